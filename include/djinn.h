@@ -1,0 +1,162 @@
+/*
+ * djinn.h -- C ABI of the B200-native DjiNN hot path: the batched DNN forward pass
+ * (inference) that serves the Tonic Suite networks.
+ *
+ * The calls follow the paper's statement of the service (sec 3.1):
+ *   - "At initialization, DjiNN loads the pre-trained model associated with each
+ *     application into memory, giving all worker threads read-only access to this
+ *     data" (L84)                                      -> djinn_load_net / djinn_free
+ *   - "DjiNN executes the DNN inference pass, which generates a prediction using the
+ *     pre-processed input from the application, and returns the prediction result"
+ *     (L71); image apps return a classification, ASR/NLP probability vectors
+ *     (Table 3)                              -> djinn_forward (out_mode)
+ *   - batching "stack[s] multiple inputs into a larger matrix" (L185)
+ *                                                      -> `rows` of djinn_forward
+ *   - "supporting more applications simply requires providing DjiNN a pretrained
+ *     neural network model" (L78)                      -> any net description in the
+ *                                                         supported layer subset
+ *
+ * Conventions (all calls):
+ *   - Return 0 (DJINN_OK) on success, a negative DJINN_E_* code on failure; the
+ *     message of the last failure on the calling thread is djinn_last_error().
+ *     No C++ exception ever crosses this boundary.
+ *   - Pointers are borrowed for the duration of the call only; the library copies
+ *     what it keeps.  The library owns every device allocation it makes (weight
+ *     arena, per-stream workspaces) until djinn_free.
+ *   - Everything the network computes runs in this library's sm_100a kernels; there
+ *     is no CPU fallback.  A process without a usable sm_100 device gets
+ *     DJINN_E_CUDA from djinn_load_net.
+ */
+#ifndef DJINN_H
+#define DJINN_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define DJINN_API __attribute__((visibility("default")))
+#else
+#define DJINN_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct djinn_net djinn_net;   /* opaque; owned by the library until djinn_free */
+
+enum {
+  DJINN_OK = 0,
+  DJINN_E_INVAL = -1,        /* bad argument (null pointer, bad enum, rows < 0)            */
+  DJINN_E_PARSE = -2,        /* net description does not parse                             */
+  DJINN_E_SHAPE = -3,        /* layer shapes inconsistent / unsupported geometry           */
+  DJINN_E_WEIGHTS = -4,      /* weight blob length does not match the description          */
+  DJINN_E_NOMEM = -5,        /* device or host allocation failed                           */
+  DJINN_E_CUDA = -6,         /* CUDA runtime/driver error (also: no sm_100 device)         */
+  DJINN_E_UNSUPPORTED = -7   /* layer type / option not supported                          */
+};
+
+/* Compute path.  FP32: SIMT FFMA kernels, fp32 storage (exact fp32 accumulation, no TF32).
+ * BF16 / FP16: tcgen05 tensor-core kernels, 16-bit operands and activations, fp32
+ * accumulation in TMEM, fp32 bias, fp32 logits and probabilities. */
+enum { DJINN_FP32 = 0, DJINN_BF16 = 1, DJINN_FP16 = 2 };
+
+/* Memory kind of a caller buffer. */
+enum { DJINN_MEM_HOST = 0, DJINN_MEM_DEVICE = 1 };
+
+/* Output of djinn_forward.
+ * PROB:   float32 [rows, out_dim] softmax probabilities (default; Table 3 "probability vectors")
+ * ARGMAX: int32   [rows] index of the largest logit, ties -> lowest index (Table 3 "classification")
+ * LOGITS: float32 [rows, out_dim] pre-softmax scores of the last layer */
+enum { DJINN_OUT_PROB = 0, DJINN_OUT_ARGMAX = 1, DJINN_OUT_LOGITS = 2 };
+
+/*
+ * djinn_load_net -- parse a net description, pack its weights on `device`, and
+ * prepare kernels and workspaces for batches of up to `max_rows` rows.
+ *
+ *   desc, desc_len : net description text, a subset of Caffe prototxt:
+ *                    `name`, `rows_per_query`, and a linear chain of `layer { ... }`
+ *                    of types Input (first), Convolution (num_output, kernel_size,
+ *                    stride, pad, group), LocallyConnected (num_output, kernel_size,
+ *                    stride), InnerProduct (num_output), ReLU, Sigmoid, TanH, HardTanh,
+ *                    LRN (local_size, alpha, beta, k; ACROSS_CHANNELS), Pooling
+ *                    (pool MAX|AVE, kernel_size, stride, pad; Caffe ceil geometry),
+ *                    Dropout (identity at inference), Softmax (last).  Copied.
+ *   weights        : canonical blob, little-endian float32: for each parametrised layer
+ *                    in file order its weights then its bias, C-order, shapes
+ *                      Convolution      W[Co][Ci/group][k][k],  b[Co]
+ *                      LocallyConnected W[OH][OW][Co][Ci][k][k], b[Co][OH][OW]
+ *                      InnerProduct     W[No][K] with K in Caffe (c,h,w) order, b[No]
+ *                    May be NULL: the weight arena is then left uninitialised, to be
+ *                    filled through djinn_weight_arena (e.g. an NCCL broadcast from a
+ *                    rank that loaded the same description with weights).
+ *   n_floats       : number of floats in `weights` (checked: DJINN_E_WEIGHTS).
+ *   weights_mem    : DJINN_MEM_HOST or DJINN_MEM_DEVICE (where `weights` lives).
+ *   device         : CUDA device ordinal the net lives on.
+ *   precision      : DJINN_FP32 | DJINN_BF16 | DJINN_FP16.  16-bit paths round the
+ *                    weights to nearest-even at load.
+ *   max_rows       : largest batch (rows) processed in one internal pass; larger
+ *                    djinn_forward calls are split into chunks of max_rows.  > 0.
+ *   out            : receives the net handle.
+ */
+DJINN_API int djinn_load_net(const char* desc, size_t desc_len, const float* weights, size_t n_floats,
+                   int weights_mem, int device, int precision, int64_t max_rows,
+                   djinn_net** out);
+
+/*
+ * djinn_forward -- run the forward pass of `rows` stacked queries' rows.
+ *
+ *   input     : float32 [rows, in_elems_per_row] in Caffe NCHW order per row
+ *               (Table 3 sizes imply fp32 inputs).  Host or device (in_mem).
+ *   rows      : number of rows (>= 0; 0 is a no-op).
+ *   output    : per out_mode (see DJINN_OUT_*), host or device (out_mem); must hold
+ *               rows * out_elems_per_row floats (PROB/LOGITS) or rows int32 (ARGMAX).
+ *   stream    : cudaStream_t to run on (NULL = legacy default stream).  The call is
+ *               asynchronous with respect to the host for device buffers; with host
+ *               buffers the copies are enqueued on the same stream and the caller must
+ *               synchronise the stream (djinn_sync) before reading `output` or reusing
+ *               `input`.
+ * Thread safety: concurrent calls on one net are safe when they use different streams
+ * (weights are read-only; each stream gets its own workspace).  Not concurrent with
+ * djinn_free.
+ */
+DJINN_API int djinn_forward(djinn_net* net, const float* input, int64_t rows, int in_mem,
+                  void* output, int out_mem, int out_mode, void* stream);
+
+/* djinn_sync -- synchronise `stream` and surface asynchronous CUDA errors as
+ * DJINN_E_CUDA. */
+DJINN_API int djinn_sync(djinn_net* net, void* stream);
+
+/* djinn_free -- release every allocation of the net.  NULL is OK. */
+DJINN_API int djinn_free(djinn_net* net);
+
+/* djinn_net_info -- any pointer may be NULL.
+ *   in_elems_per_row : product of the Input shape (e.g. 3*227*227)
+ *   out_elems_per_row: classes of the last layer
+ *   n_params         : number of floats in the canonical weight blob
+ *   n_layers         : layers excluding Input and Softmax */
+DJINN_API int djinn_net_info(const djinn_net* net, int64_t* in_elems_per_row, int64_t* out_elems_per_row,
+                   int64_t* n_params, int64_t* n_layers);
+
+/* djinn_weight_arena -- device pointer and size of the packed weight arena (one
+ * allocation), for the one-time weight broadcast of the multi-GPU harness
+ * (SURVEY.md sec 8(e)).  Nets loaded from the same description, precision and
+ * max_rows have byte-identical arena layouts. */
+DJINN_API int djinn_weight_arena(djinn_net* net, void** dev_ptr, size_t* bytes);
+
+/* djinn_plan_info -- human-readable description of the execution plan (kernels, tile
+ * shapes, buffer sizes); `buf` receives a NUL-terminated string, truncated to `cap`.
+ * Returns the full length (excluding NUL) or a negative error. */
+DJINN_API int djinn_plan_info(const djinn_net* net, char* buf, size_t cap);
+
+/* djinn_last_error -- thread-local message of the last failure ("" if none). */
+DJINN_API const char* djinn_last_error(void);
+
+/* djinn_kernel_launches -- number of kernels the library launched on this process
+ * since load (for the bench's gpu_launches claim). */
+DJINN_API int64_t djinn_kernel_launches(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DJINN_H */

@@ -1,0 +1,182 @@
+"""B200-native DjiNN hot path: Python binding of libdjinn (include/djinn.h).
+
+The binding only marshals arguments: every step of the forward pass runs in the
+library's sm_100a kernels.  There is no CPU fallback -- importing works without a
+GPU, but loading a net without the built library or without an sm_100 device
+raises ``DjinnError``.
+
+PyTorch is used for device memory and streams only (BASELINE.json north_star).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libdjinn.so")
+NETS_DIR = os.path.join(_HERE, "nets")
+
+DJINN_OK, DJINN_E_INVAL, DJINN_E_PARSE, DJINN_E_SHAPE, DJINN_E_WEIGHTS = 0, -1, -2, -3, -4
+DJINN_E_NOMEM, DJINN_E_CUDA, DJINN_E_UNSUPPORTED = -5, -6, -7
+DJINN_FP32, DJINN_BF16, DJINN_FP16 = 0, 1, 2
+DJINN_MEM_HOST, DJINN_MEM_DEVICE = 0, 1
+DJINN_OUT_PROB, DJINN_OUT_ARGMAX, DJINN_OUT_LOGITS = 0, 1, 2
+PRECISION = {"fp32": DJINN_FP32, "bf16": DJINN_BF16, "fp16": DJINN_FP16}
+EXPORTS = ["djinn_load_net", "djinn_forward", "djinn_sync", "djinn_free", "djinn_net_info",
+           "djinn_weight_arena", "djinn_plan_info", "djinn_last_error", "djinn_kernel_launches"]
+
+
+class DjinnError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"djinn error {code}: {msg}")
+        self.code = code
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libdjinn.so (built in-tree by build.py).  Fails loudly if it is missing."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise DjinnError(DJINN_E_CUDA, f"{LIB_PATH} not built; run __graft_entry__.build()")
+        L = ctypes.CDLL(LIB_PATH)
+        P, I, I64, SZ = ctypes.c_void_p, ctypes.c_int, ctypes.c_int64, ctypes.c_size_t
+        L.djinn_load_net.argtypes = [ctypes.c_char_p, SZ, P, SZ, I, I, I, I64, ctypes.POINTER(P)]
+        L.djinn_forward.argtypes = [P, P, I64, I, P, I, I, P]
+        L.djinn_sync.argtypes = [P, P]
+        L.djinn_free.argtypes = [P]
+        L.djinn_net_info.argtypes = [P] + [ctypes.POINTER(I64)] * 4
+        L.djinn_weight_arena.argtypes = [P, ctypes.POINTER(P), ctypes.POINTER(SZ)]
+        L.djinn_plan_info.argtypes = [P, ctypes.c_char_p, SZ]
+        L.djinn_last_error.restype = ctypes.c_char_p
+        L.djinn_last_error.argtypes = []
+        L.djinn_kernel_launches.restype = I64
+        L.djinn_kernel_launches.argtypes = []
+        for f in EXPORTS[:-2]:
+            getattr(L, f).restype = I
+        _lib = L
+    return _lib
+
+
+def _check(rc: int) -> int:
+    if rc < 0:
+        raise DjinnError(rc, lib().djinn_last_error().decode())
+    return rc
+
+
+def _ptr_mem(t):
+    """(pointer, memory kind) of a torch tensor or numpy array."""
+    if isinstance(t, np.ndarray):
+        return t.ctypes.data, DJINN_MEM_HOST
+    return t.data_ptr(), (DJINN_MEM_DEVICE if t.is_cuda else DJINN_MEM_HOST)
+
+
+# ----------------------------------------------------------------- C-ABI mirrors
+def djinn_load_net(desc: str, weights, precision: int, max_rows: int, device: int = 0) -> int:
+    """Mirror of djinn_load_net.  ``weights``: float32 numpy array / torch tensor or None."""
+    d = desc.encode()
+    h = ctypes.c_void_p()
+    if weights is None:
+        wp, n, mem = None, 0, DJINN_MEM_HOST
+    else:
+        if isinstance(weights, np.ndarray):
+            weights = np.ascontiguousarray(weights, dtype=np.float32)
+        wp, mem = _ptr_mem(weights)
+        n = int(weights.size if isinstance(weights, np.ndarray) else weights.numel())
+    _check(lib().djinn_load_net(d, len(d), wp, n, mem, device, precision, max_rows, ctypes.byref(h)))
+    return h.value
+
+
+def djinn_forward(net: int, inp, rows: int, out, out_mode: int, stream: Optional[int] = None) -> None:
+    ip, imem = _ptr_mem(inp)
+    op, omem = _ptr_mem(out)
+    _check(lib().djinn_forward(net, ip, rows, imem, op, omem, out_mode, stream))
+
+
+def djinn_sync(net: int, stream: Optional[int] = None) -> None:
+    _check(lib().djinn_sync(net, stream))
+
+
+def djinn_free(net: int) -> None:
+    _check(lib().djinn_free(net))
+
+
+def djinn_net_info(net: int):
+    v = [ctypes.c_int64() for _ in range(4)]
+    _check(lib().djinn_net_info(net, *[ctypes.byref(x) for x in v]))
+    return tuple(x.value for x in v)
+
+
+def djinn_weight_arena(net: int):
+    p, n = ctypes.c_void_p(), ctypes.c_size_t()
+    _check(lib().djinn_weight_arena(net, ctypes.byref(p), ctypes.byref(n)))
+    return p.value, n.value
+
+
+def djinn_plan_info(net: int) -> str:
+    n = _check(lib().djinn_plan_info(net, None, 0))
+    buf = ctypes.create_string_buffer(n + 1)
+    _check(lib().djinn_plan_info(net, buf, n + 1))
+    return buf.value.decode()
+
+
+def djinn_kernel_launches() -> int:
+    return int(lib().djinn_kernel_launches())
+
+
+# ----------------------------------------------------------------- convenience
+def net_description(app: str) -> str:
+    with open(os.path.join(NETS_DIR, f"{app}.prototxt")) as f:
+        return f.read()
+
+
+class DjinnNet:
+    """A loaded Tonic network (owns the library handle)."""
+
+    def __init__(self, desc: str, weights, precision: str = "bf16", max_rows: int = 1024,
+                 device: int = 0):
+        self.precision = precision
+        self.max_rows = max_rows
+        self.device = device
+        self.handle = djinn_load_net(desc, weights, PRECISION[precision], max_rows, device)
+        self.in_elems, self.out_elems, self.n_params, self.n_layers = djinn_net_info(self.handle)
+
+    def forward(self, x, out_mode: int = DJINN_OUT_PROB, out=None, stream=None, sync: bool = True):
+        """x: float32 [rows, ...] torch tensor (cuda or cpu) or numpy array.  Returns the
+        output tensor (on x's device for torch cuda inputs unless ``out`` is given)."""
+        import torch
+        rows = int(x.shape[0])
+        if out is None:
+            dev = x.device if (isinstance(x, torch.Tensor) and x.is_cuda) else "cpu"
+            if out_mode == DJINN_OUT_ARGMAX:
+                out = torch.empty(rows, dtype=torch.int32, device=dev)
+            else:
+                out = torch.empty(rows, self.out_elems, dtype=torch.float32, device=dev)
+        if stream is None and isinstance(x, torch.Tensor) and x.is_cuda:
+            stream = torch.cuda.current_stream(x.device).cuda_stream
+        djinn_forward(self.handle, x, rows, out, out_mode, stream)
+        if sync:
+            djinn_sync(self.handle, stream)
+        return out
+
+    def arena(self):
+        return djinn_weight_arena(self.handle)
+
+    def plan(self) -> str:
+        return djinn_plan_info(self.handle)
+
+    def close(self):
+        if self.handle:
+            djinn_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

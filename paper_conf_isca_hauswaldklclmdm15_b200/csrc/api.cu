@@ -1,0 +1,182 @@
+// C ABI of libdjinn (include/djinn.h).  Argument validation, error translation
+// (no exception crosses the boundary), device selection, thread-local error message.
+#include <string.h>
+
+#include <string>
+
+#include "../../include/djinn.h"
+#include "net.h"
+
+struct djinn_net {
+  djinn::Net impl;
+};
+
+namespace {
+thread_local std::string g_err;
+
+int fail(int code, const std::string& msg) {
+  g_err = msg;
+  return code;
+}
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+template <typename F>
+int guarded(F&& f) {
+  try {
+    g_err.clear();
+    return f();
+  } catch (const djinn::Error& e) {
+    return fail(e.code, e.what());
+  } catch (const std::bad_alloc&) {
+    return fail(DJINN_E_NOMEM, "host allocation failed");
+  } catch (const std::exception& e) {
+    return fail(DJINN_E_INVAL, e.what());
+  } catch (...) {
+    return fail(DJINN_E_INVAL, "unknown error");
+  }
+}
+}  // namespace
+
+extern "C" {
+
+int djinn_load_net(const char* desc, size_t desc_len, const float* weights, size_t n_floats, int weights_mem,
+                   int device, int precision, int64_t max_rows, djinn_net** out) {
+  return guarded([&]() -> int {
+    if (!out) return fail(DJINN_E_INVAL, "out is NULL");
+    *out = nullptr;
+    if (!desc) return fail(DJINN_E_INVAL, "desc is NULL");
+    if (precision < DJINN_FP32 || precision > DJINN_FP16) return fail(DJINN_E_INVAL, "bad precision");
+    if (weights_mem != DJINN_MEM_HOST && weights_mem != DJINN_MEM_DEVICE) return fail(DJINN_E_INVAL, "bad weights_mem");
+    if (max_rows <= 0) return fail(DJINN_E_INVAL, "max_rows must be > 0");
+    if (max_rows > (int64_t)1 << 31) return fail(DJINN_E_INVAL, "max_rows too large");
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+      cudaGetLastError();
+      return fail(DJINN_E_CUDA, "no CUDA device");
+    }
+    if (device < 0 || device >= ndev) return fail(DJINN_E_INVAL, "bad device ordinal");
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) return fail(DJINN_E_CUDA, "cudaGetDeviceProperties");
+    if (prop.major != 10) return fail(DJINN_E_CUDA, "libdjinn is built for sm_100a (B200); device is sm_" +
+                                                        std::to_string(prop.major) + std::to_string(prop.minor));
+    DeviceGuard dg(device);
+    std::unique_ptr<djinn_net> net(new djinn_net);
+    djinn::Net& n = net->impl;
+    n.device = device;
+    n.precision = precision;
+    n.dt = precision == DJINN_FP32 ? djinn::DT_F32 : precision == DJINN_BF16 ? djinn::DT_BF16 : djinn::DT_F16;
+    n.max_rows = max_rows;
+    n.build(std::string(desc, desc_len));
+    if (weights && n_floats != (size_t)n.n_params)
+      return fail(DJINN_E_WEIGHTS, "weight blob has " + std::to_string(n_floats) + " floats, description needs " +
+                                       std::to_string(n.n_params));
+    if (cudaMalloc(&n.arena, n.arena_bytes) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(DJINN_E_NOMEM, "weight arena allocation (" + std::to_string(n.arena_bytes) + " B)");
+    }
+    // per-layer tile choice and B tensor maps over the arena
+    for (djinn::Op& o : n.ops) {
+      if (o.kind != djinn::OP_GEMM || n.dt == djinn::DT_F32) continue;
+      djinn::GemmGeom g = o.g;
+      g.M = (int)(n.max_rows * o.ohw);
+      o.bn = djinn::tc_pick_bn(g);
+      uint64_t dims[3] = {(uint64_t)g.Kpad, (uint64_t)g.N, (uint64_t)g.Z};
+      uint64_t strides[2] = {(uint64_t)g.Kpad * 2, (uint64_t)g.N * g.Kpad * 2};
+      uint32_t box[3] = {64, (uint32_t)o.bn, 1};
+      djinn::encode_tmap(&o.tmB, n.dt, (uint8_t*)n.arena + o.w_off, 3, dims, strides, box);
+    }
+    if (weights) n.load_weights(weights, n_floats, weights_mem);
+    *out = net.release();
+    return DJINN_OK;
+  });
+}
+
+int djinn_forward(djinn_net* net, const float* input, int64_t rows, int in_mem, void* output, int out_mem,
+                  int out_mode, void* stream) {
+  return guarded([&]() -> int {
+    if (!net) return fail(DJINN_E_INVAL, "net is NULL");
+    if (rows < 0) return fail(DJINN_E_INVAL, "rows < 0");
+    if (rows == 0) return DJINN_OK;
+    if (!input || !output) return fail(DJINN_E_INVAL, "input/output is NULL");
+    if (in_mem != DJINN_MEM_HOST && in_mem != DJINN_MEM_DEVICE) return fail(DJINN_E_INVAL, "bad in_mem");
+    if (out_mem != DJINN_MEM_HOST && out_mem != DJINN_MEM_DEVICE) return fail(DJINN_E_INVAL, "bad out_mem");
+    if (out_mode < DJINN_OUT_PROB || out_mode > DJINN_OUT_LOGITS) return fail(DJINN_E_INVAL, "bad out_mode");
+    DeviceGuard dg(net->impl.device);
+    net->impl.forward(input, rows, in_mem, output, out_mem, out_mode, (cudaStream_t)stream);
+    return DJINN_OK;
+  });
+}
+
+int djinn_sync(djinn_net* net, void* stream) {
+  return guarded([&]() -> int {
+    if (!net) return fail(DJINN_E_INVAL, "net is NULL");
+    DeviceGuard dg(net->impl.device);
+    cudaError_t e = cudaStreamSynchronize((cudaStream_t)stream);
+    if (e == cudaSuccess) e = cudaGetLastError();
+    if (e != cudaSuccess) {
+      net->impl.poisoned = true;
+      return fail(DJINN_E_CUDA, std::string("asynchronous CUDA error: ") + cudaGetErrorString(e));
+    }
+    return DJINN_OK;
+  });
+}
+
+int djinn_free(djinn_net* net) {
+  return guarded([&]() -> int {
+    if (!net) return DJINN_OK;
+    DeviceGuard dg(net->impl.device);
+    delete net;
+    return DJINN_OK;
+  });
+}
+
+int djinn_net_info(const djinn_net* net, int64_t* in_elems, int64_t* out_elems, int64_t* n_params,
+                   int64_t* n_layers) {
+  return guarded([&]() -> int {
+    if (!net) return fail(DJINN_E_INVAL, "net is NULL");
+    if (in_elems) *in_elems = net->impl.in_elems;
+    if (out_elems) *out_elems = net->impl.out_elems;
+    if (n_params) *n_params = net->impl.n_params;
+    if (n_layers) *n_layers = net->impl.n_layers;
+    return DJINN_OK;
+  });
+}
+
+int djinn_weight_arena(djinn_net* net, void** dev_ptr, size_t* bytes) {
+  return guarded([&]() -> int {
+    if (!net || !dev_ptr || !bytes) return fail(DJINN_E_INVAL, "NULL argument");
+    *dev_ptr = net->impl.arena;
+    *bytes = net->impl.arena_bytes;
+    return DJINN_OK;
+  });
+}
+
+int djinn_plan_info(const djinn_net* net, char* buf, size_t cap) {
+  return guarded([&]() -> int {
+    if (!net) return fail(DJINN_E_INVAL, "net is NULL");
+    std::string s = net->impl.plan_string();
+    if (buf && cap) {
+      size_t k = s.size() < cap - 1 ? s.size() : cap - 1;
+      memcpy(buf, s.data(), k);
+      buf[k] = 0;
+    }
+    return (int)s.size();
+  });
+}
+
+const char* djinn_last_error(void) { return g_err.c_str(); }
+
+int64_t djinn_kernel_launches(void) { return djinn::launch_counter(); }
+
+}  // extern "C"

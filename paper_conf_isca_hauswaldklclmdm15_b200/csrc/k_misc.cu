@@ -1,0 +1,234 @@
+// Memory-bound kernels of the hot path:
+//   K0 input pack, K4 LRN, K5 pooling, K6 softmax/argmax.
+// All activations are NHWC with channel pitch Cp; math is fp32 whatever the storage type.
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
+#include <float.h>
+
+#include "kernels.h"
+
+namespace djinn {
+
+template <typename T> __device__ __forceinline__ float ld(const T* p);
+template <> __device__ __forceinline__ float ld<float>(const float* p) { return *p; }
+template <> __device__ __forceinline__ float ld<__half>(const __half* p) { return __half2float(*p); }
+template <> __device__ __forceinline__ float ld<__nv_bfloat16>(const __nv_bfloat16* p) {
+  return __bfloat162float(*p);
+}
+template <typename T> __device__ __forceinline__ T cvt(float v);
+template <> __device__ __forceinline__ float cvt<float>(float v) { return v; }
+template <> __device__ __forceinline__ __half cvt<__half>(float v) { return __float2half_rn(v); }
+template <> __device__ __forceinline__ __nv_bfloat16 cvt<__nv_bfloat16>(float v) {
+  return __float2bfloat16_rn(v);
+}
+
+static inline int nblocks(int64_t n, int t) { return (int)((n + t - 1) / t); }
+
+// ------------------------------------------------------------------------------------------
+// K0: fp32 NCHW [rows][C][H][W] -> NHWC [rows][H][W][Cp] (16-bit), 8 channels per thread.
+// Index order (row, chunk, pixel) with pixel fastest: reads are coalesced along pixels.
+template <typename T>
+__global__ void pack16_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int C,
+                              int HW, int Cp) {
+  const int chunks = Cp / 8;
+  const int64_t total = rows * chunks * (int64_t)HW;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int pix = (int)(i % HW);
+    const int64_t t = i / HW;
+    const int ch = (int)(t % chunks);
+    const int64_t r = t / chunks;
+    const float* src = x + (r * C) * (int64_t)HW + pix;
+    __align__(16) T v[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int c = ch * 8 + j;
+      v[j] = cvt<T>(c < C ? __ldg(src + (int64_t)c * HW) : 0.f);
+    }
+    *reinterpret_cast<uint4*>(y + (r * HW + pix) * Cp + ch * 8) = *reinterpret_cast<uint4*>(v);
+  }
+}
+
+// fp32 storage: one element per thread, (row, pixel, c) order -> coalesced writes.
+__global__ void pack32_kernel(const float* __restrict__ x, float* __restrict__ y, int64_t rows,
+                              int C, int HW, int Cp) {
+  const int64_t total = rows * (int64_t)HW * Cp;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int c = (int)(i % Cp);
+    const int64_t t = i / Cp;
+    const int pix = (int)(t % HW);
+    const int64_t r = t / HW;
+    y[i] = c < C ? __ldg(x + (r * C + c) * (int64_t)HW + pix) : 0.f;
+  }
+}
+
+cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int Cp,
+                              int dt, cudaStream_t st) {
+  const int HW = H * W;
+  const int T = 256;
+  if (dt == DT_F32) {
+    int64_t n = rows * (int64_t)HW * Cp;
+    pack32_kernel<<<min(nblocks(n, T), 148 * 32), T, 0, st>>>(x, (float*)y, rows, C, HW, Cp);
+  } else {
+    int64_t n = rows * (int64_t)(Cp / 8) * HW;
+    if (dt == DT_F16)
+      pack16_kernel<__half><<<min(nblocks(n, T), 148 * 32), T, 0, st>>>(x, (__half*)y, rows, C, HW, Cp);
+    else
+      pack16_kernel<__nv_bfloat16>
+          <<<min(nblocks(n, T), 148 * 32), T, 0, st>>>(x, (__nv_bfloat16*)y, rows, C, HW, Cp);
+  }
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------
+// K4: Caffe LRN across channels.  y = x * (k + alpha/size * sum_{window} x^2)^-beta.
+// One thread per (pixel, channel); the channel window is contiguous in NHWC.
+template <typename T>
+__global__ void lrn_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t pixels, int C, int Cp,
+                           int size, float alpha_over_n, float beta, float k) {
+  const int half = (size - 1) / 2;
+  const int64_t total = pixels * Cp;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int c = (int)(i % Cp);
+    if (c >= C) { y[i] = cvt<T>(0.f); continue; }
+    const T* px = x + (i - c);
+    const int lo = max(c - half, 0), hi = min(c + half, C - 1);
+    float s = 0.f;
+    for (int cc = lo; cc <= hi; ++cc) { const float v = ld(px + cc); s += v * v; }
+    const float v = ld(px + c);
+    y[i] = cvt<T>(v * powf(k + alpha_over_n * s, -beta));
+  }
+}
+
+cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, int size, float alpha,
+                       float beta, float k, int dt, cudaStream_t st) {
+  const int T = 256;
+  const int64_t n = pixels * Cp;
+  const int g = min(nblocks(n, T), 148 * 32);
+  const float an = alpha / size;
+  if (dt == DT_F32) lrn_kernel<float><<<g, T, 0, st>>>((const float*)x, (float*)y, pixels, C, Cp, size, an, beta, k);
+  else if (dt == DT_F16) lrn_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, pixels, C, Cp, size, an, beta, k);
+  else lrn_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, pixels, C, Cp, size, an, beta, k);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------
+// K5: Caffe pooling (MAX / AVE), ceil geometry; window clipped to the image, AVE divisor is
+// the window area clipped to H+pad but not to the image.
+template <typename T>
+__global__ void pool_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t rows, int Cp, int H,
+                            int W, int OH, int OW, int kern, int stride, int pad, int is_max) {
+  const int64_t total = rows * (int64_t)OH * OW * Cp;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int c = (int)(i % Cp);
+    int64_t t = i / Cp;
+    const int ox = (int)(t % OW);
+    t /= OW;
+    const int oy = (int)(t % OH);
+    const int64_t r = t / OH;
+    int hs = oy * stride - pad, ws = ox * stride - pad;
+    int he = min(hs + kern, H + pad), we = min(ws + kern, W + pad);
+    const float area = (float)((he - hs) * (we - ws));
+    hs = max(hs, 0); ws = max(ws, 0); he = min(he, H); we = min(we, W);
+    const T* base = x + r * (int64_t)H * W * Cp + c;
+    float acc = is_max ? -FLT_MAX : 0.f;
+    for (int h = hs; h < he; ++h)
+      for (int w = ws; w < we; ++w) {
+        const float v = ld(base + ((int64_t)h * W + w) * Cp);
+        acc = is_max ? fmaxf(acc, v) : acc + v;
+      }
+    y[i] = cvt<T>(is_max ? acc : acc / area);
+  }
+}
+
+cudaError_t launch_pool(const void* x, void* y, int64_t rows, int C, int Cp, int H, int W, int OH,
+                        int OW, int kernel, int stride, int pad, int is_max, int dt, cudaStream_t st) {
+  (void)C;
+  const int T = 256;
+  const int64_t n = rows * (int64_t)OH * OW * Cp;
+  const int g = min(nblocks(n, T), 148 * 32);
+  if (dt == DT_F32) pool_kernel<float><<<g, T, 0, st>>>((const float*)x, (float*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
+  else if (dt == DT_F16) pool_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
+  else pool_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------
+// K6: row softmax p_i = exp(z_i - max) / sum_j exp(z_j - max); argmax (ties -> lowest index).
+// One CTA of 256 threads per row.
+__device__ __forceinline__ void argmax_combine(float& v, int& i, float v2, int i2) {
+  if (v2 > v || (v2 == v && i2 < i)) { v = v2; i = i2; }
+}
+
+__global__ void softmax_kernel(const float* __restrict__ z, int64_t rows, int N, int pitch,
+                               void* __restrict__ out, int mode) {
+  __shared__ float s_v[32];
+  __shared__ int s_i[32];
+  const int64_t r = blockIdx.x;
+  if (r >= rows) return;
+  const float* zr = z + r * pitch;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  if (mode == 2) {
+    float* o = (float*)out + r * N;
+    for (int i = threadIdx.x; i < N; i += blockDim.x) o[i] = zr[i];
+    return;
+  }
+  float m = -FLT_MAX;
+  int mi = 0x7fffffff;
+  for (int i = threadIdx.x; i < N; i += blockDim.x) argmax_combine(m, mi, zr[i], i);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    const float v2 = __shfl_xor_sync(0xffffffffu, m, o);
+    const int i2 = __shfl_xor_sync(0xffffffffu, mi, o);
+    argmax_combine(m, mi, v2, i2);
+  }
+  if (lane == 0) { s_v[wid] = m; s_i[wid] = mi; }
+  __syncthreads();
+  if (wid == 0) {
+    m = lane < nw ? s_v[lane] : -FLT_MAX;
+    mi = lane < nw ? s_i[lane] : 0x7fffffff;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+      const float v2 = __shfl_xor_sync(0xffffffffu, m, o);
+      const int i2 = __shfl_xor_sync(0xffffffffu, mi, o);
+      argmax_combine(m, mi, v2, i2);
+    }
+    if (lane == 0) { s_v[0] = m; s_i[0] = mi; }
+  }
+  __syncthreads();
+  m = s_v[0];
+  mi = s_i[0];
+  if (mode == 1) {
+    if (threadIdx.x == 0) ((int*)out)[r] = mi;
+    return;
+  }
+  __syncthreads();
+  float s = 0.f;
+  for (int i = threadIdx.x; i < N; i += blockDim.x) s += expf(zr[i] - m);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if (lane == 0) s_v[wid] = s;
+  __syncthreads();
+  if (wid == 0) {
+    s = lane < nw ? s_v[lane] : 0.f;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (lane == 0) s_v[0] = s;
+  }
+  __syncthreads();
+  const float inv = 1.f / s_v[0];
+  float* o = (float*)out + r * N;
+  for (int i = threadIdx.x; i < N; i += blockDim.x) o[i] = expf(zr[i] - m) * inv;
+}
+
+cudaError_t launch_softmax(const float* logits, int64_t rows, int N, int pitch, void* out, int mode,
+                           cudaStream_t st) {
+  if (rows <= 0) return cudaSuccess;
+  softmax_kernel<<<(unsigned)rows, 256, 0, st>>>(logits, rows, N, pitch, out, mode);
+  return cudaGetLastError();
+}
+
+}  // namespace djinn

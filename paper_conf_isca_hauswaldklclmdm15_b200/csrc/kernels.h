@@ -1,0 +1,73 @@
+// Kernel launch interface of libdjinn (host side).  Every function enqueues work on
+// `stream` and returns cudaError_t of the launch.  Layouts: activations are NHWC per
+// row with a channel pitch Cp (PAPER.md L63-65 layers; DESIGN.md sec 4 "data layout").
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace djinn {
+
+enum DType { DT_F32 = 0, DT_BF16 = 1, DT_F16 = 2 };
+enum Act { ACT_NONE = 0, ACT_RELU = 1, ACT_SIGMOID = 2, ACT_TANH = 3, ACT_HARDTANH = 4 };
+enum GemmMode { GM_DENSE = 0, GM_CONV = 1, GM_LC = 2 };
+
+// One convolution / locally-connected / fully-connected layer as an implicit GEMM:
+//   Y[pix(m), goff + n] = act( bias + sum_k A[m,k] * B[z][n][k] )
+// m enumerates output pixels (conv: (img,oy,ox); LC: img at location z; dense: row),
+// k enumerates (ky, kx, c) with c fastest (NHWC), z = group (conv) or location (LC).
+struct GemmGeom {
+  int mode;
+  int M;              // GEMM rows
+  int N;              // valid output channels per z (Cog / Co / No)
+  int Z;              // groups (conv), locations (LC) or 1
+  int K;              // valid K (conv/LC: KH*KW*Cgp; dense: row length)
+  int Kpad;           // K rounded up to the k-block (64) -- B row length
+  // gather geometry (conv / LC)
+  int H, W, Cp_in;    // input image per row and its channel pitch
+  int OH, OW;
+  int KH, KW, stride, pad;
+  int Cgp;            // channels per group used in K (multiple of 8 on 16-bit paths)
+  int cin_goff;       // input channel offset between groups
+  // dense A
+  int a_pitch;        // dense: elements per A row
+  // output
+  int out_pitch;      // elements per output pixel (Cp_out) or per row (dense)
+  int cout_goff;      // output channel offset between groups
+  int write_cols;     // columns written per z: valid N plus zero-filled pad up to here
+  int bias_zstride;   // bias elements between z (LC: Co per location; conv: Cog)
+  int act;
+  int out_f32;        // 1: fp32 output (logits), 0: same 16-bit type as input
+};
+
+// --- pack (K0): fp32 NCHW rows -> NHWC with channel pitch Cp, type dt -------------------
+cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int Cp,
+                              int dt, cudaStream_t st);
+
+// --- SIMT fp32 implicit GEMM (K7; exact fp32 FFMA accumulation) --------------------------
+// B: [Z][N][K] fp32 (K unpadded), bias fp32.
+cudaError_t launch_simt_gemm(const GemmGeom& g, const float* A, const float* B, const float* bias,
+                             float* Y, cudaStream_t st);
+
+// --- tcgen05 tensor-core implicit GEMM (K1/K2/K3) -----------------------------------------
+// tmB: 3D tensor map over B [Z][N][Kpad] (16-bit, SWIZZLE_128B, box {64, BN, 1}).
+// tmA: 2D tensor map over dense A [M][a_pitch] (box {64, 128}); unused for gather modes.
+int tc_pick_bn(const GemmGeom& g);
+cudaError_t launch_tc_gemm(const GemmGeom& g, int bn, int dt, const CUtensorMap* tmA,
+                           const CUtensorMap* tmB, const void* A, const float* bias, void* Y,
+                           cudaStream_t st);
+
+// --- LRN across channels (K4), NHWC ----------------------------------------------------------
+cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, int size, float alpha,
+                       float beta, float k, int dt, cudaStream_t st);
+
+// --- pooling (K5), NHWC, Caffe ceil geometry ------------------------------------------------
+cudaError_t launch_pool(const void* x, void* y, int64_t rows, int C, int Cp, int H, int W, int OH,
+                        int OW, int kernel, int stride, int pad, int is_max, int dt, cudaStream_t st);
+
+// --- softmax / argmax / logits copy (K6) ----------------------------------------------------
+// logits fp32 [rows][pitch]; mode 0: prob fp32 [rows][N]; 1: argmax int32 [rows]; 2: logits copy.
+cudaError_t launch_softmax(const float* logits, int64_t rows, int N, int pitch, void* out, int mode,
+                           cudaStream_t st);
+
+}  // namespace djinn

@@ -1,0 +1,582 @@
+// Host runtime of libdjinn: prototxt-subset parser, shape inference, execution plan,
+// weight packing into one device arena, per-stream workspaces and the forward driver.
+//
+// Service model (sec 3.1): DjiNN "loads the pre-trained model associated with
+// each application into memory, giving all worker threads read-only access" (L84);
+// the DNN library is Caffe's configurable layer framework (L77-78), so the description
+// format is a Caffe-prototxt subset.  Batching stacks queries into larger matrices (L185).
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
+#include <string.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cctype>
+#include <sstream>
+
+#include "../../include/djinn.h"
+#include "net.h"
+
+namespace djinn {
+
+// ============================================================================ parser
+const std::string* PNode::get(const std::string& k) const {
+  auto it = scalars.find(k);
+  return (it == scalars.end() || it->second.empty()) ? nullptr : &it->second[0];
+}
+const PNode* PNode::block(const std::string& k) const {
+  auto it = blocks.find(k);
+  return (it == blocks.end() || it->second.empty()) ? nullptr : &it->second[0];
+}
+int PNode::geti(const std::string& k, int def) const {
+  const std::string* s = get(k);
+  if (!s) return def;
+  char* end = nullptr;
+  long v = strtol(s->c_str(), &end, 10);
+  if (!end || *end) throw Error(DJINN_E_PARSE, "field '" + k + "' is not an integer: " + *s);
+  return (int)v;
+}
+double PNode::getf(const std::string& k, double def) const {
+  const std::string* s = get(k);
+  if (!s) return def;
+  char* end = nullptr;
+  double v = strtod(s->c_str(), &end);
+  if (!end || *end) throw Error(DJINN_E_PARSE, "field '" + k + "' is not a number: " + *s);
+  return v;
+}
+std::string PNode::gets(const std::string& k, const std::string& def) const {
+  const std::string* s = get(k);
+  return s ? *s : def;
+}
+
+namespace {
+struct Lexer {
+  const std::string& t;
+  size_t i = 0;
+  explicit Lexer(const std::string& s) : t(s) {}
+  bool next(std::string& tok) {
+    for (;;) {
+      while (i < t.size() && isspace((unsigned char)t[i])) ++i;
+      if (i < t.size() && t[i] == '#') {
+        while (i < t.size() && t[i] != '\n') ++i;
+        continue;
+      }
+      break;
+    }
+    if (i >= t.size()) return false;
+    char c = t[i];
+    if (c == '{' || c == '}' || c == ':') { tok.assign(1, c); ++i; return true; }
+    if (c == '"') {
+      size_t j = t.find('"', i + 1);
+      if (j == std::string::npos) throw Error(DJINN_E_PARSE, "unterminated string");
+      tok = t.substr(i, j - i + 1);
+      i = j + 1;
+      return true;
+    }
+    size_t j = i;
+    while (j < t.size() && !isspace((unsigned char)t[j]) && t[j] != '{' && t[j] != '}' && t[j] != ':' &&
+           t[j] != '"' && t[j] != '#')
+      ++j;
+    tok = t.substr(i, j - i);
+    i = j;
+    return true;
+  }
+};
+
+void parse_block(Lexer& lx, PNode& node, bool top) {
+  std::string key, tok;
+  while (lx.next(key)) {
+    if (key == "}") {
+      if (top) throw Error(DJINN_E_PARSE, "unbalanced '}'");
+      return;
+    }
+    if (key == "{" || key == ":") throw Error(DJINN_E_PARSE, "expected a field name, got '" + key + "'");
+    if (!lx.next(tok)) throw Error(DJINN_E_PARSE, "unexpected end after '" + key + "'");
+    if (tok == ":") {
+      if (!lx.next(tok)) throw Error(DJINN_E_PARSE, "missing value for '" + key + "'");
+    }
+    if (tok == "{") {
+      PNode child;
+      parse_block(lx, child, false);
+      node.blocks[key].push_back(std::move(child));
+    } else {
+      if (tok == "}" || tok == ":") throw Error(DJINN_E_PARSE, "bad value for '" + key + "'");
+      if (tok.size() >= 2 && tok[0] == '"') tok = tok.substr(1, tok.size() - 2);
+      node.scalars[key].push_back(tok);
+    }
+  }
+  if (!top) throw Error(DJINN_E_PARSE, "missing '}'");
+}
+}  // namespace
+
+PNode parse_prototxt(const std::string& text) {
+  PNode root;
+  Lexer lx(text);
+  parse_block(lx, root, true);
+  return root;
+}
+
+// ============================================================================ helpers
+std::atomic<int64_t>& launch_counter() {
+  static std::atomic<int64_t> c{0};
+  return c;
+}
+
+static void ck(cudaError_t e, const char* what) {
+  if (e != cudaSuccess) throw Error(DJINN_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static EncodeTiledFn encode_fn() {
+  static EncodeTiledFn fn = nullptr;
+  if (!fn) {
+    cudaDriverEntryPointQueryResult q;
+    void* p = nullptr;
+    ck(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q), "cuTensorMapEncodeTiled lookup");
+    if (q != cudaDriverEntryPointSuccess || !p) throw Error(DJINN_E_CUDA, "cuTensorMapEncodeTiled unavailable");
+    fn = (EncodeTiledFn)p;
+  }
+  return fn;
+}
+
+void encode_tmap(CUtensorMap* m, int dt, const void* base, int rank, const uint64_t* dims, const uint64_t* strides_bytes,
+                 const uint32_t* box) {
+  cuuint64_t d[5], s[4];
+  cuuint32_t b[5], es[5];
+  for (int i = 0; i < rank; ++i) { d[i] = dims[i]; b[i] = box[i]; es[i] = 1; }
+  for (int i = 0; i + 1 < rank; ++i) s[i] = strides_bytes[i];
+  const CUtensorMapDataType ty = dt == DT_F16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16;
+  CUresult r = encode_fn()(m, ty, (cuuint32_t)rank, const_cast<void*>(base), d, s, b, es,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) throw Error(DJINN_E_CUDA, "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")");
+}
+
+static inline int rup(int v, int m) { return (v + m - 1) / m * m; }
+static inline size_t rupz(size_t v, size_t m) { return (v + m - 1) / m * m; }
+
+// ============================================================================ plan
+static int act_of(const std::string& t) {
+  if (t == "ReLU") return ACT_RELU;
+  if (t == "Sigmoid") return ACT_SIGMOID;
+  if (t == "TanH") return ACT_TANH;
+  if (t == "HardTanh") return ACT_HARDTANH;
+  return -1;
+}
+
+void Net::build(const std::string& desc) {
+  PNode root = parse_prototxt(desc);
+  name = root.gets("name", "");
+  rows_per_query = root.geti("rows_per_query", 1);
+  auto it = root.blocks.find("layer");
+  if (it == root.blocks.end() || it->second.empty()) throw Error(DJINN_E_PARSE, "no layers");
+  for (const PNode& L : it->second) {
+    LayerSpec s;
+    s.name = L.gets("name", "");
+    s.type = L.gets("type", "");
+    if (s.type == "Input") {
+      const PNode* ip = L.block("input_param");
+      const PNode* sh = ip ? ip->block("shape") : nullptr;
+      if (!sh) throw Error(DJINN_E_PARSE, "Input without input_param.shape");
+      auto d = sh->scalars.find("dim");
+      if (d == sh->scalars.end()) throw Error(DJINN_E_PARSE, "Input shape without dims");
+      for (auto& v : d->second) s.dims.push_back(atoi(v.c_str()));
+    } else if (s.type == "Convolution" || s.type == "LocallyConnected" || s.type == "InnerProduct") {
+      const char* pn = s.type == "Convolution" ? "convolution_param"
+                       : s.type == "LocallyConnected" ? "local_param" : "inner_product_param";
+      const PNode* p = L.block(pn);
+      if (!p) throw Error(DJINN_E_PARSE, s.name + ": missing " + pn);
+      s.num_output = p->geti("num_output", 0);
+      s.kernel = p->geti("kernel_size", 0);
+      s.stride = p->geti("stride", 1);
+      s.pad = p->geti("pad", 0);
+      s.group = p->geti("group", 1);
+    } else if (s.type == "Pooling") {
+      const PNode* p = L.block("pooling_param");
+      if (!p) throw Error(DJINN_E_PARSE, s.name + ": missing pooling_param");
+      std::string m = p->gets("pool", "MAX");
+      if (m != "MAX" && m != "AVE") throw Error(DJINN_E_UNSUPPORTED, s.name + ": pool " + m);
+      s.pool_max = m == "MAX";
+      s.kernel = p->geti("kernel_size", 0);
+      s.stride = p->geti("stride", 1);
+      s.pad = p->geti("pad", 0);
+    } else if (s.type == "LRN") {
+      const PNode* p = L.block("lrn_param");
+      s.lrn_size = p ? p->geti("local_size", 5) : 5;
+      s.alpha = p ? (float)p->getf("alpha", 1.0) : 1.f;
+      s.beta = p ? (float)p->getf("beta", 0.75) : 0.75f;
+      s.lrn_k = p ? (float)p->getf("k", 1.0) : 1.f;
+      if (p && p->gets("norm_region", "ACROSS_CHANNELS") != "ACROSS_CHANNELS")
+        throw Error(DJINN_E_UNSUPPORTED, s.name + ": only ACROSS_CHANNELS LRN");
+    } else if (act_of(s.type) >= 0 || s.type == "Dropout" || s.type == "Softmax") {
+    } else {
+      throw Error(DJINN_E_UNSUPPORTED, "layer type '" + s.type + "'");
+    }
+    layers.push_back(s);
+  }
+  if (layers[0].type != "Input") throw Error(DJINN_E_SHAPE, "first layer must be Input");
+  if (layers.back().type != "Softmax") throw Error(DJINN_E_UNSUPPORTED, "last layer must be Softmax");
+
+  const bool f16 = dt != DT_F32;
+  auto pitch = [&](int c) { return f16 ? rup(c, 8) : c; };
+  const std::vector<int>& d = layers[0].dims;
+  Shape cur;
+  if (d.size() == 1) { cur.C = d[0]; }
+  else if (d.size() == 3) { cur.C = d[0]; cur.H = d[1]; cur.W = d[2]; }
+  else throw Error(DJINN_E_SHAPE, "Input must have 1 or 3 dims");
+  if (cur.C <= 0 || cur.H <= 0 || cur.W <= 0) throw Error(DJINN_E_SHAPE, "bad Input dims");
+  cur.Cp = pitch(cur.C);
+  in_elems = (int64_t)cur.C * cur.H * cur.W;
+
+  Op pk;
+  pk.kind = OP_PACK;
+  pk.name = "pack";
+  pk.in = cur;
+  pk.out = cur;
+  pk.in_buf = -1;
+  pk.out_buf = 0;
+  ops.push_back(pk);
+  int curbuf = 0;
+  n_layers = 0;
+  n_params = 0;
+  size_t arena_off = 0;
+
+  for (size_t i = 1; i < layers.size(); ++i) {
+    const LayerSpec& L = layers[i];
+    if (L.type != "Softmax") ++n_layers;
+    if (L.type == "Dropout") continue;
+    if (L.type == "Softmax") {
+      if (i + 1 != layers.size()) throw Error(DJINN_E_UNSUPPORTED, "Softmax must be the last layer");
+      if (ops.back().kind != OP_GEMM || ops.back().out_buf != 2)
+        throw Error(DJINN_E_UNSUPPORTED, "Softmax must follow an InnerProduct");
+      Op sm;
+      sm.kind = OP_SOFTMAX;
+      sm.name = L.name;
+      sm.in = cur;
+      sm.out = cur;
+      sm.in_buf = 2;
+      ops.push_back(sm);
+      continue;
+    }
+    if (act_of(L.type) >= 0) throw Error(DJINN_E_UNSUPPORTED, L.name + ": activation must follow a weighted layer");
+    if (L.type == "LRN") {
+      Op o;
+      o.kind = OP_LRN;
+      o.name = L.name;
+      o.in = o.out = cur;
+      o.in_buf = curbuf;
+      o.out_buf = curbuf = 1 - curbuf;
+      o.lrn_size = L.lrn_size;
+      o.alpha = L.alpha;
+      o.beta = L.beta;
+      o.lrn_k = L.lrn_k;
+      if (cur.H * cur.W < 1) throw Error(DJINN_E_SHAPE, L.name);
+      ops.push_back(o);
+      continue;
+    }
+    if (L.type == "Pooling") {
+      if (L.kernel <= 0 || L.stride <= 0 || L.pad < 0 || L.pad >= L.kernel) throw Error(DJINN_E_SHAPE, L.name + ": bad pooling");
+      Op o;
+      o.kind = OP_POOL;
+      o.name = L.name;
+      o.in = cur;
+      auto pout = [&](int in) {
+        int out = (int)((in + 2 * L.pad - L.kernel + L.stride - 1) / L.stride) + 1;  // ceil
+        if (in + 2 * L.pad - L.kernel < 0) out = 1;
+        if (L.pad > 0 && (out - 1) * L.stride >= in + L.pad) --out;
+        return out;
+      };
+      o.out = cur;
+      o.out.H = pout(cur.H);
+      o.out.W = pout(cur.W);
+      o.kernel = L.kernel;
+      o.stride = L.stride;
+      o.pad = L.pad;
+      o.is_max = L.pool_max;
+      o.in_buf = curbuf;
+      o.out_buf = curbuf = 1 - curbuf;
+      cur = o.out;
+      ops.push_back(o);
+      continue;
+    }
+    // ---- weighted layers: Convolution / LocallyConnected / InnerProduct ----
+    int act = ACT_NONE;
+    size_t j = i + 1;
+    if (j < layers.size() && act_of(layers[j].type) >= 0) {
+      act = act_of(layers[j].type);
+      ++j;
+      ++n_layers;
+      i = j - 1;
+    }
+    size_t nx = i + 1;
+    while (nx < layers.size() && layers[nx].type == "Dropout") ++nx;
+    const bool last = nx < layers.size() && layers[nx].type == "Softmax";
+    Op o;
+    o.kind = OP_GEMM;
+    o.name = L.name;
+    o.in = cur;
+    o.in_buf = curbuf;
+    GemmGeom& g = o.g;
+    memset(&g, 0, sizeof(g));
+    g.act = act;
+    g.stride = 1;
+    g.KH = g.KW = 1;
+    if (L.num_output <= 0) throw Error(DJINN_E_SHAPE, L.name + ": num_output");
+    int64_t wcount = 0, bcount = 0;
+    if (L.type == "Convolution" || L.type == "LocallyConnected") {
+      if (L.kernel <= 0 || L.stride <= 0 || L.pad < 0) throw Error(DJINN_E_SHAPE, L.name + ": bad kernel/stride/pad");
+      const bool lc = L.type == "LocallyConnected";
+      const int grp = lc ? 1 : L.group, pad = lc ? 0 : L.pad;
+      if (lc && L.pad != 0) throw Error(DJINN_E_UNSUPPORTED, L.name + ": padded LocallyConnected");
+      if (grp <= 0 || cur.C % grp || L.num_output % grp) throw Error(DJINN_E_SHAPE, L.name + ": group does not divide channels");
+      const int Cg = cur.C / grp, Cog = L.num_output / grp;
+      if (f16 && grp > 1 && (Cg % 8 || Cog % 8))
+        throw Error(DJINN_E_UNSUPPORTED, L.name + ": grouped conv needs channels per group % 8 == 0 on 16-bit paths");
+      const int OH = (cur.H + 2 * pad - L.kernel) / L.stride + 1, OW = (cur.W + 2 * pad - L.kernel) / L.stride + 1;
+      if (cur.H + 2 * pad < L.kernel || cur.W + 2 * pad < L.kernel) throw Error(DJINN_E_SHAPE, L.name + ": kernel larger than input");
+      g.mode = lc ? GM_LC : GM_CONV;
+      g.N = Cog;
+      g.Z = lc ? OH * OW : grp;
+      g.H = cur.H; g.W = cur.W; g.Cp_in = cur.Cp;
+      g.OH = OH; g.OW = OW;
+      g.KH = g.KW = L.kernel;
+      g.stride = L.stride;
+      g.pad = pad;
+      g.Cgp = (grp == 1) ? cur.Cp : Cg;
+      g.cin_goff = Cg;
+      g.K = L.kernel * L.kernel * g.Cgp;
+      o.out.C = L.num_output; o.out.H = OH; o.out.W = OW; o.out.Cp = pitch(L.num_output);
+      g.out_pitch = o.out.Cp;
+      g.cout_goff = Cog;
+      g.write_cols = grp == 1 ? o.out.Cp : Cog;
+      g.bias_zstride = Cog;
+      o.ohw = lc ? 1 : OH * OW;
+      wcount = lc ? (int64_t)OH * OW * L.num_output * cur.C * L.kernel * L.kernel
+                  : (int64_t)L.num_output * Cg * L.kernel * L.kernel;
+      bcount = lc ? (int64_t)L.num_output * OH * OW : L.num_output;
+    } else {
+      g.mode = GM_DENSE;
+      g.N = L.num_output;
+      g.Z = 1;
+      g.K = (int)cur.per_row();
+      g.a_pitch = g.K;
+      o.out.C = L.num_output; o.out.H = 1; o.out.W = 1;
+      o.out.Cp = last ? rup(L.num_output, 8) : pitch(L.num_output);
+      g.out_pitch = o.out.Cp;
+      g.write_cols = o.out.Cp;
+      g.bias_zstride = 0;
+      wcount = (int64_t)L.num_output * cur.C * cur.H * cur.W;
+      bcount = L.num_output;
+    }
+    if (last && g.mode != GM_DENSE) throw Error(DJINN_E_UNSUPPORTED, "the layer before Softmax must be InnerProduct");
+    g.Kpad = f16 ? rup(g.K, 64) : g.K;
+    g.out_f32 = last ? 1 : 0;
+    o.out_buf = last ? 2 : 1 - curbuf;
+    if (!last) curbuf = o.out_buf;
+    if (last) out_pitch = o.out.Cp;
+    o.bn = f16 ? 0 : 64;
+    // arena placement
+    const size_t wbytes = (size_t)g.Z * g.N * g.Kpad * (f16 ? 2 : 4);
+    const size_t bfloats = g.mode == GM_DENSE ? (size_t)g.N : (size_t)g.Z * g.bias_zstride;
+    arena_off = rupz(arena_off, 1024);
+    o.w_off = arena_off;
+    arena_off += wbytes;
+    arena_off = rupz(arena_off, 256);
+    o.b_off = arena_off;
+    arena_off += bfloats * 4;
+    n_params += wcount + bcount;
+    cur = o.out;
+    ops.push_back(o);
+  }
+  out_elems = cur.C;
+  arena_bytes = rupz(arena_off, 1024);
+  for (const Op& o : ops) {
+    if (o.kind == OP_SOFTMAX || o.out_buf < 0) continue;
+    const size_t es = o.out_buf == 2 ? 4 : (f16 ? 2 : 4);
+    buf_bytes[o.out_buf] = std::max(buf_bytes[o.out_buf], (size_t)max_rows * o.out.per_row() * es);
+  }
+}
+
+// ============================================================================ weights
+void Net::load_weights(const float* w, size_t n, int mem) {
+  const bool f16 = dt != DT_F32;
+  if (n != (size_t)n_params)
+    throw Error(DJINN_E_WEIGHTS, "weight blob has " + std::to_string(n) + " floats, description needs " +
+                                     std::to_string(n_params));
+  std::vector<float> hostcopy;
+  if (mem == DJINN_MEM_DEVICE) {
+    hostcopy.resize(n);
+    ck(cudaMemcpy(hostcopy.data(), w, n * 4, cudaMemcpyDeviceToHost), "weights D2H");
+    w = hostcopy.data();
+  }
+  std::vector<uint8_t> host(arena_bytes, 0);
+  size_t off = 0;  // floats into the canonical blob
+  for (Op& o : ops) {
+    if (o.kind != OP_GEMM) continue;
+    const GemmGeom& g = o.g;
+    uint8_t* wdst = host.data() + o.w_off;
+    float* bdst = reinterpret_cast<float*>(host.data() + o.b_off);
+    auto put = [&](int64_t z, int64_t nn, int64_t k, float v) {
+      const int64_t idx = (z * g.N + nn) * g.Kpad + k;
+      if (!f16) { reinterpret_cast<float*>(wdst)[idx] = v; return; }
+      uint16_t bits;
+      if (dt == DT_BF16) { __nv_bfloat16 h = __float2bfloat16_rn(v); memcpy(&bits, &h, 2); }
+      else { __half h = __float2half_rn(v); memcpy(&bits, &h, 2); }
+      reinterpret_cast<uint16_t*>(wdst)[idx] = bits;
+    };
+    const int C = o.in.C, H = o.in.H, W = o.in.W, Cp = o.in.Cp;
+    if (g.mode == GM_CONV) {
+      const int grp = g.Z, Cg = C / grp, k = g.KH;
+      for (int co = 0; co < o.out.C; ++co)
+        for (int c = 0; c < Cg; ++c)
+          for (int ky = 0; ky < k; ++ky)
+            for (int kx = 0; kx < k; ++kx)
+              put(co / g.N, co % g.N, (int64_t)(ky * k + kx) * g.Cgp + c, w[off++]);
+      for (int co = 0; co < o.out.C; ++co) bdst[co] = w[off++];
+    } else if (g.mode == GM_LC) {
+      const int k = g.KH;
+      for (int loc = 0; loc < g.Z; ++loc)
+        for (int co = 0; co < g.N; ++co)
+          for (int c = 0; c < C; ++c)
+            for (int ky = 0; ky < k; ++ky)
+              for (int kx = 0; kx < k; ++kx)
+                put(loc, co, (int64_t)(ky * k + kx) * g.Cgp + c, w[off++]);
+      for (int co = 0; co < g.N; ++co)
+        for (int loc = 0; loc < g.Z; ++loc) bdst[(int64_t)loc * g.N + co] = w[off++];
+    } else {
+      // Caffe flattens (c, h, w); our rows are (h, w, c) with channel pitch Cp.
+      for (int nn = 0; nn < g.N; ++nn)
+        for (int c = 0; c < C; ++c)
+          for (int h = 0; h < H; ++h)
+            for (int x = 0; x < W; ++x)
+              put(0, nn, ((int64_t)h * W + x) * Cp + c, w[off++]);
+      for (int nn = 0; nn < g.N; ++nn) bdst[nn] = w[off++];
+    }
+  }
+  if (off != n) throw Error(DJINN_E_WEIGHTS, "internal: blob walk mismatch");
+  ck(cudaMemcpy(arena, host.data(), arena_bytes, cudaMemcpyHostToDevice), "weights H2D");
+}
+
+// ============================================================================ workspace
+Workspace::~Workspace() {
+  for (void* p : buf) if (p) cudaFree(p);
+  if (in_stage) cudaFree(in_stage);
+  if (out_stage) cudaFree(out_stage);
+}
+
+Net::~Net() {
+  ws.clear();
+  if (arena) cudaFree(arena);
+}
+
+Workspace* Net::workspace(cudaStream_t st) {
+  std::lock_guard<std::mutex> lk(mu);
+  auto it = ws.find(st);
+  if (it != ws.end()) return it->second.get();
+  std::unique_ptr<Workspace> w(new Workspace);
+  for (int b = 0; b < 3; ++b) {
+    if (!buf_bytes[b]) continue;
+    if (cudaMalloc(&w->buf[b], buf_bytes[b]) != cudaSuccess) throw Error(DJINN_E_NOMEM, "workspace allocation");
+    ck(cudaMemset(w->buf[b], 0, buf_bytes[b]), "workspace memset");
+  }
+  w->tmA.resize(ops.size());
+  if (dt != DT_F32) {
+    for (size_t i = 0; i < ops.size(); ++i) {
+      const Op& o = ops[i];
+      if (o.kind != OP_GEMM || o.g.mode != GM_DENSE) continue;
+      uint64_t dims[2] = {(uint64_t)o.g.a_pitch, (uint64_t)max_rows};
+      uint64_t strides[1] = {(uint64_t)o.g.a_pitch * 2};
+      uint32_t box[2] = {64, 128};
+      encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 2, dims, strides, box);
+    }
+  }
+  Workspace* r = w.get();
+  ws[st] = std::move(w);
+  return r;
+}
+
+// ============================================================================ forward
+void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_mem, int mode, cudaStream_t st) {
+  if (poisoned) throw Error(DJINN_E_CUDA, "net is poisoned by an earlier CUDA error");
+  Workspace* w = workspace(st);
+  if (in_mem == DJINN_MEM_HOST && !w->in_stage)
+    if (cudaMalloc(&w->in_stage, (size_t)max_rows * in_elems * 4) != cudaSuccess) throw Error(DJINN_E_NOMEM, "input staging");
+  if (out_mem == DJINN_MEM_HOST && !w->out_stage)
+    if (cudaMalloc(&w->out_stage, (size_t)max_rows * out_elems * 4) != cudaSuccess) throw Error(DJINN_E_NOMEM, "output staging");
+  const size_t out_row_bytes = mode == DJINN_OUT_ARGMAX ? 4 : (size_t)out_elems * 4;
+  std::atomic<int64_t>& launches = launch_counter();
+  for (int64_t r0 = 0; r0 < rows; r0 += max_rows) {
+    const int64_t n = std::min<int64_t>(max_rows, rows - r0);
+    const float* src = in + r0 * in_elems;
+    if (in_mem == DJINN_MEM_HOST) {
+      ck(cudaMemcpyAsync(w->in_stage, src, (size_t)n * in_elems * 4, cudaMemcpyHostToDevice, st), "input H2D");
+      src = w->in_stage;
+    }
+    uint8_t* dst = out_mem == DJINN_MEM_HOST ? (uint8_t*)w->out_stage : (uint8_t*)out + r0 * out_row_bytes;
+    for (size_t i = 0; i < ops.size(); ++i) {
+      const Op& o = ops[i];
+      cudaError_t e = cudaSuccess;
+      switch (o.kind) {
+        case OP_PACK:
+          e = launch_pack_input(src, w->buf[0], n, o.in.C, o.in.H, o.in.W, o.out.Cp, dt, st);
+          break;
+        case OP_GEMM: {
+          GemmGeom g = o.g;
+          g.M = (int)(n * o.ohw);
+          const void* A = w->buf[o.in_buf];
+          void* Y = w->buf[o.out_buf];
+          const uint8_t* ar = (const uint8_t*)arena;
+          if (dt == DT_F32)
+            e = launch_simt_gemm(g, (const float*)A, (const float*)(ar + o.w_off), (const float*)(ar + o.b_off),
+                                 (float*)Y, st);
+          else
+            e = launch_tc_gemm(g, o.bn, dt, &w->tmA[i], &o.tmB, A, (const float*)(ar + o.b_off), Y, st);
+          break;
+        }
+        case OP_LRN:
+          e = launch_lrn(w->buf[o.in_buf], w->buf[o.out_buf], n * o.in.H * o.in.W, o.in.C, o.in.Cp, o.lrn_size,
+                         o.alpha, o.beta, o.lrn_k, dt, st);
+          break;
+        case OP_POOL:
+          e = launch_pool(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.H, o.in.W, o.out.H, o.out.W,
+                          o.kernel, o.stride, o.pad, o.is_max, dt, st);
+          break;
+        case OP_SOFTMAX:
+          e = launch_softmax((const float*)w->buf[2], n, (int)out_elems, out_pitch, dst, mode, st);
+          break;
+      }
+      ++launches;
+      if (e != cudaSuccess) {
+        poisoned = true;
+        throw Error(DJINN_E_CUDA, o.name + ": " + cudaGetErrorString(e));
+      }
+    }
+    if (out_mem == DJINN_MEM_HOST)
+      ck(cudaMemcpyAsync((uint8_t*)out + r0 * out_row_bytes, w->out_stage, (size_t)n * out_row_bytes,
+                         cudaMemcpyDeviceToHost, st),
+         "output D2H");
+  }
+}
+
+std::string Net::plan_string() const {
+  std::ostringstream s;
+  static const char* kinds[] = {"pack", "gemm", "lrn", "pool", "softmax"};
+  static const char* modes[] = {"dense", "conv", "local"};
+  s << "net " << name << " precision " << (dt == DT_F32 ? "fp32" : dt == DT_BF16 ? "bf16" : "fp16") << " max_rows "
+    << max_rows << " arena " << arena_bytes << " B params " << n_params << "\n";
+  for (const Op& o : ops) {
+    s << "  " << kinds[o.kind] << " " << o.name << " in " << o.in.C << "x" << o.in.H << "x" << o.in.W << "/p" << o.in.Cp
+      << " -> " << o.out.C << "x" << o.out.H << "x" << o.out.W << "/p" << o.out.Cp << " buf " << o.in_buf << "->"
+      << o.out_buf;
+    if (o.kind == OP_GEMM)
+      s << " [" << modes[o.g.mode] << " N=" << o.g.N << " Z=" << o.g.Z << " K=" << o.g.K << " Kpad=" << o.g.Kpad
+        << " act=" << o.g.act << " bn=" << o.bn << (o.g.out_f32 ? " fp32-out" : "") << "]";
+    s << "\n";
+  }
+  return s.str();
+}
+
+}  // namespace djinn

@@ -1,0 +1,107 @@
+// Host-side runtime of libdjinn: net-description parser, execution plan, weight arena,
+// per-stream workspaces.  The service model is PAPER.md sec 3.1 (L77-84): a pretrained
+// model is loaded once and shared read-only by all concurrent requests.
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <stdexcept>
+#include <string>
+#include <vector>
+
+#include "kernels.h"
+
+namespace djinn {
+
+struct Error : std::runtime_error {
+  int code;
+  Error(int c, const std::string& m) : std::runtime_error(m), code(c) {}
+};
+
+// ---- parsed description (subset of Caffe prototxt) --------------------------------------
+struct PNode {
+  std::map<std::string, std::vector<std::string>> scalars;
+  std::map<std::string, std::vector<PNode>> blocks;
+  const std::string* get(const std::string& k) const;
+  const PNode* block(const std::string& k) const;
+  int geti(const std::string& k, int def) const;
+  double getf(const std::string& k, double def) const;
+  std::string gets(const std::string& k, const std::string& def) const;
+};
+PNode parse_prototxt(const std::string& text);  // throws Error(DJINN_E_PARSE)
+
+struct LayerSpec {
+  std::string name, type;
+  int num_output = 0, kernel = 0, stride = 1, pad = 0, group = 1;
+  bool pool_max = true;
+  int lrn_size = 5;
+  float alpha = 1.f, beta = 0.75f, lrn_k = 1.f;
+  std::vector<int> dims;
+};
+
+enum OpKind { OP_PACK, OP_GEMM, OP_LRN, OP_POOL, OP_SOFTMAX };
+
+struct Shape { int C = 0, H = 1, W = 1, Cp = 0; int64_t per_row() const { return (int64_t)H * W * Cp; } };
+
+struct Op {
+  OpKind kind;
+  std::string name;
+  Shape in, out;
+  int in_buf = 0, out_buf = 0;  // 0/1 ping-pong, 2 logits, -1 external input
+  // gemm
+  GemmGeom g{};
+  int bn = 0;
+  size_t w_off = 0, b_off = 0;  // bytes into the weight arena
+  CUtensorMap tmB{};
+  int ohw = 1;                  // output pixels per row (conv M = rows * ohw)
+  // lrn
+  int lrn_size = 5;
+  float alpha = 0, beta = 0, lrn_k = 1;
+  // pool
+  int kernel = 0, stride = 1, pad = 0, is_max = 1;
+};
+
+struct Workspace {
+  void* buf[3] = {nullptr, nullptr, nullptr};
+  float* in_stage = nullptr;
+  void* out_stage = nullptr;
+  std::vector<CUtensorMap> tmA;  // per op (dense gemm) over its input buffer
+  ~Workspace();
+};
+
+struct Net {
+  int device = 0;
+  int precision = 0;  // DJINN_FP32 / BF16 / FP16
+  int dt = DT_F32;
+  int64_t max_rows = 0;
+  std::string name;
+  int rows_per_query = 1;
+  std::vector<LayerSpec> layers;
+  std::vector<Op> ops;
+  int64_t in_elems = 0, out_elems = 0, n_params = 0, n_layers = 0;
+  int out_pitch = 0;  // logits pitch
+  void* arena = nullptr;
+  size_t arena_bytes = 0;
+  size_t buf_bytes[3] = {0, 0, 0};
+  std::mutex mu;
+  std::map<cudaStream_t, std::unique_ptr<Workspace>> ws;
+  bool poisoned = false;
+  ~Net();
+
+  void build(const std::string& desc);                          // parse + plan
+  void load_weights(const float* w, size_t n, int mem);         // pack into the arena
+  Workspace* workspace(cudaStream_t st);
+  void forward(const float* in, int64_t rows, int in_mem, void* out, int out_mem, int mode,
+               cudaStream_t st);
+  std::string plan_string() const;
+};
+
+std::atomic<int64_t>& launch_counter();
+void encode_tmap(CUtensorMap* m, int dt, const void* base, int rank, const uint64_t* dims,
+                 const uint64_t* strides_bytes, const uint32_t* box);
+
+}  // namespace djinn

@@ -1,0 +1,125 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the fp64 oracle, element by element,
+on the same seeded inputs (-m gpu).  Sizes span several tiles and a ragged tail."""
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_isca_hauswaldklclmdm15_b200 as dj
+from datagen import recipes
+
+from parity import (FP32_PROB_TOL, REL_LOGIT_TOL, TOP1_MIN, blob, compare_16bit, compare_fp32,
+                    oracle_rows)
+
+pytestmark = pytest.mark.gpu
+
+# rows per parity case: small enough for the oracle in seconds, > one M tile with a ragged tail
+ROWS = {"dig": 300, "pos": 1000, "chk": 1000, "ner": 1000, "asr": 300, "face": 6, "imc": 6}
+APPS = list(ROWS)
+
+
+def run_gpu(app, prec, x, max_rows=None, mode=dj.DJINN_OUT_LOGITS):
+    net = dj.DjinnNet(dj.net_description(app), blob(app, prec), prec, max_rows or x.shape[0])
+    xt = torch.from_numpy(x).cuda()
+    out = net.forward(xt, mode).cpu().numpy()
+    net.close()
+    return out
+
+
+@pytest.mark.parametrize("app", APPS)
+def test_fp32_path_matches_oracle(app):
+    n = ROWS[app]
+    x = recipes.gen_input_rows(app, 0, n, "fp32")
+    lg_ref, pr_ref = oracle_rows(app, x, "fp32")
+    net = dj.DjinnNet(dj.net_description(app), blob(app, "fp32"), "fp32", n)
+    xt = torch.from_numpy(x).cuda()
+    lg = net.forward(xt, dj.DJINN_OUT_LOGITS).cpu().numpy()
+    pr = net.forward(xt, dj.DJINN_OUT_PROB).cpu().numpy()
+    net.close()
+    r = compare_fp32(pr, pr_ref, lg, lg_ref)
+    print(app, "fp32", r)
+    assert r["prob_max_abs"] <= FP32_PROB_TOL, r
+
+
+@pytest.mark.parametrize("prec", ["bf16", "fp16"])
+@pytest.mark.parametrize("app", APPS)
+def test_tensor_core_path_matches_oracle(app, prec):
+    n = ROWS[app]
+    x = recipes.gen_input_rows(app, 0, n, prec)
+    lg_ref, _ = oracle_rows(app, x, prec)
+    lg = run_gpu(app, prec, x)
+    r = compare_16bit(lg, lg_ref)
+    print(app, prec, r)
+    assert r["rel_max"] <= REL_LOGIT_TOL, r
+    assert r["top1_decidable"] >= TOP1_MIN, r
+
+
+@pytest.mark.parametrize("prec", ["fp32", "bf16"])
+def test_prob_argmax_logits_modes_agree(prec):
+    app = "pos"
+    x = recipes.gen_input_rows(app, 0, 777, prec)
+    net = dj.DjinnNet(dj.net_description(app), blob(app, prec), prec, 777)
+    xt = torch.from_numpy(x).cuda()
+    lg = net.forward(xt, dj.DJINN_OUT_LOGITS)
+    pr = net.forward(xt, dj.DJINN_OUT_PROB)
+    am = net.forward(xt, dj.DJINN_OUT_ARGMAX)
+    net.close()
+    torch.testing.assert_close(pr, torch.softmax(lg.double(), 1).float(), rtol=1e-5, atol=1e-6)
+    assert torch.equal(am.long(), lg.argmax(1))
+    torch.testing.assert_close(pr.sum(1), torch.ones(777, device=pr.device), rtol=0, atol=1e-5)
+
+
+def test_chunking_and_host_buffers_match_device_path():
+    """rows > max_rows is processed in chunks; host input/output equals device I/O bitwise."""
+    app, prec = "dig", "bf16"
+    x = recipes.gen_input_rows(app, 0, 250, prec)
+    net = dj.DjinnNet(dj.net_description(app), blob(app, prec), prec, 64)
+    dev = net.forward(torch.from_numpy(x).cuda(), dj.DJINN_OUT_PROB).cpu()
+    host_out = torch.empty(250, 10)
+    s = torch.cuda.Stream()
+    dj.djinn_forward(net.handle, torch.from_numpy(x).pin_memory(), 250, host_out, dj.DJINN_OUT_PROB,
+                     s.cuda_stream)
+    dj.djinn_sync(net.handle, s.cuda_stream)
+    net.close()
+    full = run_gpu(app, prec, x, max_rows=250, mode=dj.DJINN_OUT_PROB)
+    assert torch.equal(dev, host_out)
+    np.testing.assert_array_equal(dev.numpy(), full)
+
+
+def test_rows_zero_and_error_paths():
+    net = dj.DjinnNet(dj.net_description("pos"), blob("pos", "bf16"), "bf16", 16)
+    out = torch.empty(0, 45, device="cuda")
+    dj.djinn_forward(net.handle, torch.empty(0, 300, device="cuda"), 0, out, dj.DJINN_OUT_PROB)
+    with pytest.raises(dj.DjinnError) as e:
+        dj.djinn_forward(net.handle, torch.empty(4, 300, device="cuda"), -1, out, dj.DJINN_OUT_PROB)
+    assert e.value.code == dj.DJINN_E_INVAL
+    net.close()
+    with pytest.raises(dj.DjinnError) as e:
+        dj.DjinnNet("layer { name: 'x' type: 'Input' ", None, "bf16", 16)
+    assert e.value.code == dj.DJINN_E_PARSE
+    with pytest.raises(dj.DjinnError) as e:
+        dj.DjinnNet(dj.net_description("pos"), np.zeros(10, np.float32), "bf16", 16)
+    assert e.value.code == dj.DJINN_E_WEIGHTS
+    bad = dj.net_description("pos").replace('type: "HardTanh"', 'type: "Swish"')
+    with pytest.raises(dj.DjinnError) as e:
+        dj.DjinnNet(bad, None, "bf16", 16)
+    assert e.value.code == dj.DJINN_E_UNSUPPORTED
+
+
+def test_concurrent_streams_share_read_only_weights():
+    """Two streams on one net (read-only sharing across workers)."""
+    app, prec = "asr", "bf16"
+    x = recipes.gen_input_rows(app, 0, 256, prec)
+    net = dj.DjinnNet(dj.net_description(app), blob(app, prec), prec, 256)
+    xt = torch.from_numpy(x).cuda()
+    ref = net.forward(xt, dj.DJINN_OUT_LOGITS)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    o1 = torch.empty_like(ref)
+    o2 = torch.empty_like(ref)
+    torch.cuda.synchronize()
+    for _ in range(3):
+        dj.djinn_forward(net.handle, xt, 256, o1, dj.DJINN_OUT_LOGITS, s1.cuda_stream)
+        dj.djinn_forward(net.handle, xt, 256, o2, dj.DJINN_OUT_LOGITS, s2.cuda_stream)
+    dj.djinn_sync(net.handle, s1.cuda_stream)
+    dj.djinn_sync(net.handle, s2.cuda_stream)
+    net.close()
+    assert torch.equal(o1, ref) and torch.equal(o2, ref)
