@@ -1,0 +1,345 @@
+"""bench.py -- queries/s of the B200-native DjiNN forward pass on the Tonic Suite.
+
+Metric (BASELINE.json): queries/sec per Tonic app at 1/2/4/8 B200, plus % tensor peak
+(GEMM) / % HBM BW.  A query is a Table 3 unit: IMC 1 image, DIG 100
+images, FACE 1 image, ASR 548 frames, POS/CHK/NER a 28-word sentence.
+
+One step = one batch of EVERY Tonic app through the whole hot path (Table 5
+"MIXED" service workload, L308), per GPU at the BASELINE.json config batch:
+    IMC 1024 images, FACE 256 images, ASR 8192 frames, POS/CHK/NER 4096 windows each,
+    DIG 16 queries (1600 images)
+Inputs are device-resident when the timed region starts (the paper's PCIe-bypass
+measurement, L251); ``e2e`` repeats the step through host buffers (pinned H2D of the
+inputs and D2H of the probabilities inside the timed region).  Weak scaling: each rank
+serves its own shard of queries with a full model replica; the only collective is the
+one-time weight-arena broadcast (L231 "no communication between GPUs").
+
+Usage:  python bench.py [--gpus N] [--steps K] [--warmup W] [--precision bf16|fp16|fp32]
+        python bench.py --impl reference ...     (the fp64 CPU oracle on a bounded sample)
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from datagen import recipes  # noqa: E402
+
+APPS = ["imc", "face", "asr", "pos", "chk", "ner", "dig"]
+BATCH_ROWS = {"imc": 1024, "face": 256, "asr": 8192, "pos": 4096, "chk": 4096, "ner": 4096, "dig": 1600}
+ROWS_PER_QUERY = recipes.ROWS_PER_QUERY
+METRIC = "queries/sec per Tonic app at 1/2/4/8 B200; % tensor peak (GEMM) / % HBM BW"
+# oracle sample per app for the CPU baseline / reference arm (rows)
+CPU_SAMPLE = {"imc": 1, "face": 1, "asr": 64, "pos": 28, "chk": 28, "ner": 28, "dig": 10}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return {"hbm_gbs": d["hbm_gbs"], "tflops": d["bf16_tflops"], "tflops_sustained": d["bf16_tflops_sustained"],
+                "src": "measured (MEASURED_PEAKS.json)"}
+    return {"hbm_gbs": 6650.0, "tflops": 1590.0, "tflops_sustained": 1400.0, "src": "fallback (B200_PROFILING.md)"}
+
+
+def queries_per_step(world: int = 1) -> float:
+    return world * sum(BATCH_ROWS[a] / ROWS_PER_QUERY[a] for a in APPS)
+
+
+# ------------------------------------------------------------------ clocks sampler
+class ClockSampler:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 5 + i and r[5 + i] == "Active"})
+        pw = [float(r[3]) for r in self.rows if r[3].replace(".", "").isdigit()]
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows), "power_w_max": max(pw) if pw else None}
+
+
+# ------------------------------------------------------------------ CPU oracle leg
+def run_oracle_sample(apps=APPS, threads=None):
+    """Time the fp64 oracle (as it stands) on CPU_SAMPLE rows of each app.
+    Returns (mixed-workload queries/s extrapolated from per-app s/row, detail)."""
+    from oracle import OracleNet
+    from oracle.calibrate import net_text
+    detail = {}
+    step_s = 0.0
+    for app in apps:
+        net = OracleNet(net_text(app))
+        W = recipes.gen_weights(app, "fp32")
+        n = CPU_SAMPLE[app]
+        x = recipes.gen_input_rows(app, 0, n, "fp32")
+        t0 = time.perf_counter()
+        net.forward(x, W)
+        dt = time.perf_counter() - t0
+        s_per_row = dt / n
+        detail[app] = {"rows": n, "seconds": dt, "queries_per_s": 1.0 / (s_per_row * ROWS_PER_QUERY[app])}
+        step_s += s_per_row * BATCH_ROWS[app]
+    return queries_per_step() / step_s, detail
+
+
+def reference_arm(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    cores = os.cpu_count()
+    for _ in range(args.warmup):
+        run_oracle_sample()
+    vals = []
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        v, detail = run_oracle_sample()
+        vals.append(v)
+    wall = time.perf_counter() - t0
+    value = statistics.median(vals)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * wall / max(1, args.steps),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": "tonic-mixed (Table 5 MIXED): one batch of every app per step",
+                       "batch_rows": BATCH_ROWS, "oracle_sample_rows": CPU_SAMPLE},
+            "cpu_baseline": {"value": value, "unit": "queries/s", "cores": cores, "kind": "oracle",
+                             "sample": "per step: " + ", ".join(f"{a} {CPU_SAMPLE[a]} rows" for a in APPS)
+                                       + "; extrapolated to the mixed step by measured seconds/row"},
+            "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "per_app_queries_per_s": {a: d["queries_per_s"] for a, d in detail.items()}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ GPU arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
+    ap.add_argument("--precision", default=os.environ.get("DJINN_BENCH_PRECISION", "bf16"),
+                    choices=["bf16", "fp16", "fp32"])
+    ap.add_argument("--apps", default=",".join(APPS))
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--profile-json", default=None, help="write per-op timings here")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return reference_arm(args)
+    assert args.warmup >= 3 or os.environ.get("DJINN_BENCH_ALLOW_SHORT"), "W >= 3 warm-up steps required"
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_isca_hauswaldklclmdm15_b200 as dj
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    apps = [a for a in args.apps.split(",") if a]
+    grid = args.precision
+    stream = torch.cuda.Stream()
+    sh = stream.cuda_stream
+
+    # ---- load every app: rank 0 packs the weights, others receive the arena (C1 broadcast)
+    nets, inputs, outputs = {}, {}, {}
+    for app in apps:
+        rows = BATCH_ROWS[app]
+        w = recipes.flat_blob(recipes.gen_weights(app, grid)) if rank == 0 else None
+        net = dj.DjinnNet(dj.net_description(app), w, grid, rows, local)
+        if world > 1:
+            ptr, nbytes = net.arena()
+
+            class _Arena:
+                __cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (ptr, False), "version": 3}
+            dist.broadcast(torch.as_tensor(_Arena(), device="cuda"), src=0)
+        nets[app] = net
+        x = recipes.gen_input_rows(app, rank * rows, rows, grid)          # this rank's shard
+        inputs[app] = torch.from_numpy(x).cuda()
+        outputs[app] = torch.empty(rows, net.out_elems, device="cuda")
+        del w
+    torch.cuda.synchronize()
+
+    def step():
+        for app in apps:
+            dj.djinn_forward(nets[app].handle, inputs[app], BATCH_ROWS[app], outputs[app], dj.DJINN_OUT_PROB, sh)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def timed(fn, k):
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(k):
+            fn()
+        e1.record(stream)
+        barrier()
+        ms = e0.elapsed_time(e1)
+        if world > 1:
+            t = torch.tensor([ms], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = t.item()
+        return ms
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    for app in apps:
+        dj.djinn_profile(nets[app].handle, True)
+    l0 = dj.djinn_kernel_launches()
+    with ClockSampler(local) as clk:
+        ms = timed(step, args.steps)
+    launches = dj.djinn_kernel_launches() - l0
+    ms_per_step = ms / args.steps
+    qps = sum(BATCH_ROWS[a] / ROWS_PER_QUERY[a] for a in apps) * world / (ms_per_step / 1e3)
+
+    # ---- per-op device times over the timed region -> dominant kernel roofline
+    peaks = load_peaks()
+    ops = []
+    for app in apps:
+        prof = dj.djinn_profile_read(nets[app].handle, reset=True)
+        dj.djinn_profile(nets[app].handle, False)
+        for i, (t, c) in enumerate(prof):
+            if c == 0:
+                continue
+            info = dj.djinn_op_info(nets[app].handle, i)
+            rows = BATCH_ROWS[app]
+            flops = info["flops_per_row"] * rows
+            byts = info["bytes_per_row"] * rows + info["weight_bytes"]
+            avg_s = t / c / 1e3
+            t_tc = flops / (peaks["tflops_sustained"] * 1e12)
+            t_hbm = byts / (peaks["hbm_gbs"] * 1e9)
+            ops.append({"app": app, "op": info["name"], "kind": info["kind"], "ms_total": t, "launches": c,
+                        "avg_us": avg_s * 1e6, "flops": flops, "bytes": byts,
+                        "tflops": flops / avg_s / 1e12, "gbs": byts / avg_s / 1e9,
+                        "bound": "tensor" if t_tc >= t_hbm else "hbm",
+                        "roofline_us": max(t_tc, t_hbm) * 1e6})
+    ops.sort(key=lambda o: -o["ms_total"])
+    step_total = sum(o["ms_total"] for o in ops)
+    top = ops[0]
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        with open(tpath) as f:
+            traffic = json.load(f).get(f"{top['app']}/{top['op']}", {}).get("dram_bytes_per_launch")
+    if top["bound"] == "tensor":
+        roof = {"bound": "tensor", "achieved": top["tflops"], "peak": peaks["tflops_sustained"], "unit": "TFLOP/s"}
+    else:
+        roof = {"bound": "hbm", "achieved": top["gbs"], "peak": peaks["hbm_gbs"], "unit": "GB/s"}
+    roof["frac"] = roof["achieved"] / roof["peak"]
+    roof.update({"traffic": traffic, "kernel": f"{top['app']}/{top['op']}", "share_of_step": top["ms_total"] / step_total,
+                 "algorithmic_flops": top["flops"], "algorithmic_bytes": top["bytes"],
+                 "peak_src": peaks["src"] + (" sustained bf16" if top["bound"] == "tensor" else " copy BW")})
+
+    # ---- per-app isolated throughput
+    per_app = {}
+    for app in apps:
+        k = max(3, args.steps // 2)
+        t = timed(lambda a=app: dj.djinn_forward(nets[a].handle, inputs[a], BATCH_ROWS[a], outputs[a],
+                                                 dj.DJINN_OUT_PROB, sh), k) / k
+        q = BATCH_ROWS[app] / ROWS_PER_QUERY[app] * world
+        rl = sum(o["roofline_us"] for o in ops if o["app"] == app) / 1e3
+        per_app[app] = {"queries_per_s": q / (t / 1e3), "ms_per_batch": t, "batch_rows": BATCH_ROWS[app],
+                        "roofline_ms": rl, "roofline_frac": rl / t}
+
+    # ---- e2e: public API with pinned HOST buffers (H2D + D2H inside the timed region)
+    e2e = None
+    if not args.no_e2e:
+        hin = {a: inputs[a].cpu().pin_memory() for a in apps}
+        hout = {a: torch.empty(BATCH_ROWS[a], nets[a].out_elems).pin_memory() for a in apps}
+
+        def step_host():
+            for a in apps:
+                dj.djinn_forward(nets[a].handle, hin[a], BATCH_ROWS[a], hout[a], dj.DJINN_OUT_PROB, sh)
+        for _ in range(2):
+            step_host()
+        k = max(3, args.steps // 4)
+        t = timed(step_host, k) / k
+        e2e = {"value": sum(BATCH_ROWS[a] / ROWS_PER_QUERY[a] for a in apps) * world / (t / 1e3), "unit": "queries/s",
+               "ms_per_step": t, "h2d_bytes_per_step": int(sum(hin[a].numel() * 4 for a in apps)),
+               "d2h_bytes_per_step": int(sum(hout[a].numel() * 4 for a in apps))}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        v, detail = run_oracle_sample(apps)
+        cpu = {"value": v, "unit": "queries/s", "cores": os.cpu_count(), "kind": "oracle",
+               "sample": "one oracle pass over " + ", ".join(f"{a} {CPU_SAMPLE[a]} rows" for a in apps)
+                         + "; mixed-step rate extrapolated from measured seconds/row",
+               "per_app_queries_per_s": {a: d["queries_per_s"] for a, d in detail.items()}}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": qps, "unit": "queries/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": {"bf16": "bf16", "fp16": "f16", "fp32": "f32"}[grid],
+                "data": "synthetic (seeded LSUV-calibrated weights, Table 3 input shapes)",
+                "config": {"workload": "tonic-mixed (Table 5 MIXED): one batch of every app per step per GPU",
+                           "batch_rows_per_gpu": {a: BATCH_ROWS[a] for a in apps},
+                           "queries_per_step_per_gpu": sum(BATCH_ROWS[a] / ROWS_PER_QUERY[a] for a in apps),
+                           "l2": "step working set (~2 GB of inputs/activations) >> 126 MB L2",
+                           "parallelism": f"replica x{world}, query shards, no per-step collective"},
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
+                "clocks": clk.summary(), "per_app": per_app,
+                "top_ops": [{k: o[k] for k in ("app", "op", "kind", "ms_total", "avg_us", "tflops", "gbs", "bound",
+                                               "roofline_us")} for o in ops[:12]]}
+        print(json.dumps(line), flush=True)
+        if args.profile_json:
+            with open(args.profile_json, "w") as f:
+                json.dump({"ops": ops, "per_app": per_app}, f, indent=1)
+    for n in nets.values():
+        n.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -149,6 +149,27 @@ DJINN_API int djinn_weight_arena(djinn_net* net, void** dev_ptr, size_t* bytes);
  * Returns the full length (excluding NUL) or a negative error. */
 DJINN_API int djinn_plan_info(const djinn_net* net, char* buf, size_t cap);
 
+/* djinn_profile -- enable (1) / disable (0) per-op device timing of subsequent
+ * djinn_forward calls on this net: a CUDA event is recorded on the forward's stream
+ * before each kernel and after the last one (PAPER.md L151-173 profiles per kernel,
+ * weighted by kernel time).  Enabling clears earlier records. */
+DJINN_API int djinn_profile(djinn_net* net, int enable);
+
+/* djinn_profile_read -- synchronise the recorded events and return, per op of the plan
+ * (index 0..n_ops-1), the summed device milliseconds and the number of timed launches.
+ * ms / count may be NULL; at most `cap` entries are written.  reset != 0 clears the
+ * records.  Returns n_ops or a negative error. */
+DJINN_API int djinn_profile_read(djinn_net* net, double* ms, int64_t* count, int cap, int reset);
+
+/* djinn_op_info -- static description of plan op `op` (0 <= op < n_ops):
+ *   name (NUL-terminated, truncated to name_cap), kind (0 pack, 1 gemm, 2 lrn, 3 pool,
+ *   4 softmax), and its ALGORITHMIC work per row of the batch: flops (2 per
+ *   multiply-add, real unpadded dimensions), activation bytes read + written at the
+ *   path's storage width, and the bytes of weights + bias it must read once per launch.
+ * Any output pointer may be NULL.  Returns n_ops or a negative error. */
+DJINN_API int djinn_op_info(const djinn_net* net, int op, char* name, size_t name_cap, int* kind,
+                            double* flops_per_row, double* bytes_per_row, double* weight_bytes);
+
 /* djinn_last_error -- thread-local message of the last failure ("" if none). */
 DJINN_API const char* djinn_last_error(void);
 

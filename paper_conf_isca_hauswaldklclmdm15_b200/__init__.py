@@ -26,7 +26,9 @@ DJINN_MEM_HOST, DJINN_MEM_DEVICE = 0, 1
 DJINN_OUT_PROB, DJINN_OUT_ARGMAX, DJINN_OUT_LOGITS = 0, 1, 2
 PRECISION = {"fp32": DJINN_FP32, "bf16": DJINN_BF16, "fp16": DJINN_FP16}
 EXPORTS = ["djinn_load_net", "djinn_forward", "djinn_sync", "djinn_free", "djinn_net_info",
-           "djinn_weight_arena", "djinn_plan_info", "djinn_last_error", "djinn_kernel_launches"]
+           "djinn_weight_arena", "djinn_plan_info", "djinn_profile", "djinn_profile_read", "djinn_op_info",
+           "djinn_last_error", "djinn_kernel_launches"]
+OP_KINDS = ["pack", "gemm", "lrn", "pool", "softmax"]
 
 
 class DjinnError(RuntimeError):
@@ -53,6 +55,11 @@ def lib() -> ctypes.CDLL:
         L.djinn_net_info.argtypes = [P] + [ctypes.POINTER(I64)] * 4
         L.djinn_weight_arena.argtypes = [P, ctypes.POINTER(P), ctypes.POINTER(SZ)]
         L.djinn_plan_info.argtypes = [P, ctypes.c_char_p, SZ]
+        D = ctypes.c_double
+        L.djinn_profile.argtypes = [P, I]
+        L.djinn_profile_read.argtypes = [P, ctypes.POINTER(D), ctypes.POINTER(I64), I, I]
+        L.djinn_op_info.argtypes = [P, I, ctypes.c_char_p, SZ, ctypes.POINTER(I), ctypes.POINTER(D),
+                                    ctypes.POINTER(D), ctypes.POINTER(D)]
         L.djinn_last_error.restype = ctypes.c_char_p
         L.djinn_last_error.argtypes = []
         L.djinn_kernel_launches.restype = I64
@@ -125,6 +132,29 @@ def djinn_plan_info(net: int) -> str:
     return buf.value.decode()
 
 
+def djinn_profile(net: int, enable: bool) -> None:
+    _check(lib().djinn_profile(net, 1 if enable else 0))
+
+
+def djinn_profile_read(net: int, reset: bool = True):
+    """[(ms_total, launches)] per plan op."""
+    n = _check(lib().djinn_profile_read(net, None, None, 0, 0))
+    ms = (ctypes.c_double * n)()
+    cnt = (ctypes.c_int64 * n)()
+    _check(lib().djinn_profile_read(net, ms, cnt, n, 1 if reset else 0))
+    return [(ms[i], cnt[i]) for i in range(n)]
+
+
+def djinn_op_info(net: int, op: int) -> dict:
+    name = ctypes.create_string_buffer(128)
+    kind = ctypes.c_int()
+    f, b, w = ctypes.c_double(), ctypes.c_double(), ctypes.c_double()
+    n = _check(lib().djinn_op_info(net, op, name, 128, ctypes.byref(kind), ctypes.byref(f), ctypes.byref(b),
+                                   ctypes.byref(w)))
+    return {"index": op, "n_ops": n, "name": name.value.decode(), "kind": OP_KINDS[kind.value],
+            "flops_per_row": f.value, "bytes_per_row": b.value, "weight_bytes": w.value}
+
+
 def djinn_kernel_launches() -> int:
     return int(lib().djinn_kernel_launches())
 
@@ -169,6 +199,10 @@ class DjinnNet:
 
     def plan(self) -> str:
         return djinn_plan_info(self.handle)
+
+    def ops(self):
+        n = djinn_op_info(self.handle, 0)["n_ops"]
+        return [djinn_op_info(self.handle, i) for i in range(n)]
 
     def close(self):
         if self.handle:

@@ -175,6 +175,65 @@ int djinn_plan_info(const djinn_net* net, char* buf, size_t cap) {
   });
 }
 
+int djinn_profile(djinn_net* net, int enable) {
+  return guarded([&]() -> int {
+    if (!net) return fail(DJINN_E_INVAL, "net is NULL");
+    std::lock_guard<std::mutex> lk(net->impl.mu);
+    net->impl.prof_clear();
+    net->impl.profile = enable != 0;
+    return DJINN_OK;
+  });
+}
+
+int djinn_profile_read(djinn_net* net, double* ms, int64_t* count, int cap, int reset) {
+  return guarded([&]() -> int {
+    if (!net) return fail(DJINN_E_INVAL, "net is NULL");
+    djinn::Net& n = net->impl;
+    DeviceGuard dg(n.device);
+    std::lock_guard<std::mutex> lk(n.mu);
+    const int nops = (int)n.ops.size();
+    std::vector<double> acc(nops, 0.0);
+    std::vector<int64_t> cnt(nops, 0);
+    for (const djinn::ProfRec& r : n.prof_recs) {
+      if (cudaEventSynchronize(n.prof_events[r.first + r.n_ops]) != cudaSuccess)
+        return fail(DJINN_E_CUDA, "profile event synchronize");
+      for (int i = 0; i < r.n_ops && i < nops; ++i) {
+        float t = 0.f;
+        if (cudaEventElapsedTime(&t, n.prof_events[r.first + i], n.prof_events[r.first + i + 1]) != cudaSuccess)
+          return fail(DJINN_E_CUDA, "cudaEventElapsedTime");
+        acc[i] += t;
+        cnt[i] += 1;
+      }
+    }
+    for (int i = 0; i < nops && i < cap; ++i) {
+      if (ms) ms[i] = acc[i];
+      if (count) count[i] = cnt[i];
+    }
+    if (reset) n.prof_clear();
+    return nops;
+  });
+}
+
+int djinn_op_info(const djinn_net* net, int op, char* name, size_t name_cap, int* kind, double* flops_per_row,
+                  double* bytes_per_row, double* weight_bytes) {
+  return guarded([&]() -> int {
+    if (!net) return fail(DJINN_E_INVAL, "net is NULL");
+    const djinn::Net& n = net->impl;
+    if (op < 0 || op >= (int)n.ops.size()) return fail(DJINN_E_INVAL, "op index out of range");
+    const djinn::Op& o = n.ops[op];
+    if (name && name_cap) {
+      size_t k = o.name.size() < name_cap - 1 ? o.name.size() : name_cap - 1;
+      memcpy(name, o.name.data(), k);
+      name[k] = 0;
+    }
+    if (kind) *kind = (int)o.kind;
+    if (flops_per_row) *flops_per_row = o.flops_row;
+    if (bytes_per_row) *bytes_per_row = o.bytes_row;
+    if (weight_bytes) *weight_bytes = o.weight_bytes;
+    return (int)n.ops.size();
+  });
+}
+
 const char* djinn_last_error(void) { return g_err.c_str(); }
 
 int64_t djinn_kernel_launches(void) { return djinn::launch_counter(); }

@@ -25,27 +25,45 @@ template <> __device__ __forceinline__ __nv_bfloat16 cvt<__nv_bfloat16>(float v)
 static inline int nblocks(int64_t n, int t) { return (int)((n + t - 1) / t); }
 
 // ------------------------------------------------------------------------------------------
-// K0: fp32 NCHW [rows][C][H][W] -> NHWC [rows][H][W][Cp] (16-bit), 8 channels per thread.
-// Index order (row, chunk, pixel) with pixel fastest: reads are coalesced along pixels.
+// K0: fp32 NCHW [rows][C][H][W] -> NHWC [rows][Ho][Wo][Cp] (16-bit), 8 channels per thread,
+// with the optional first-layer transforms (space-to-depth, kx-unroll) that give the first
+// convolution a dense, 16-element-aligned K (DESIGN.md sec 5 "first layer").
 template <typename T>
-__global__ void pack16_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int C,
-                              int HW, int Cp) {
+__global__ void pack16_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int C, int H, int W,
+                              int mode, int f, int Ho, int Wo, int Cp) {
   const int chunks = Cp / 8;
-  const int64_t total = rows * chunks * (int64_t)HW;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
-       i += (int64_t)gridDim.x * blockDim.x) {
-    const int pix = (int)(i % HW);
-    const int64_t t = i / HW;
-    const int ch = (int)(t % chunks);
-    const int64_t r = t / chunks;
-    const float* src = x + (r * C) * (int64_t)HW + pix;
-    __align__(16) T v[8];
+  const int per_row = Ho * Wo * chunks;  // 32-bit index math inside a row
+  for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
+    const float* src = x + r * C * (int64_t)H * W;
+    T* dst = y + r * (int64_t)per_row * 8;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < per_row; i += gridDim.x * blockDim.x) {
+      const int ch = i % chunks;
+      const int pix = i / chunks;
+      const int yo = pix / Wo, xo = pix - (pix / Wo) * Wo;
+      __align__(16) T v[8];
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const int c = ch * 8 + j;
-      v[j] = cvt<T>(c < C ? __ldg(src + (int64_t)c * HW) : 0.f);
+      for (int j = 0; j < 8; ++j) {
+        const int cc = ch * 8 + j;
+        int c = cc, yy = yo, xx = xo;
+        bool ok;
+        if (mode == 0) {
+          ok = cc < C;
+        } else if (mode == 1) {
+          const int d = cc / C;
+          c = cc - d * C;
+          yy = yo * f + d / f;
+          xx = xo * f + d % f;
+          ok = d < f * f && yy < H && xx < W;
+        } else {
+          const int kx = cc / C;
+          c = cc - kx * C;
+          xx = xo + kx;
+          ok = kx < f && xx < W;
+        }
+        v[j] = cvt<T>(ok ? __ldg(src + (c * H + yy) * W + xx) : 0.f);
+      }
+      *reinterpret_cast<uint4*>(dst + i * 8) = *reinterpret_cast<uint4*>(v);
     }
-    *reinterpret_cast<uint4*>(y + (r * HW + pix) * Cp + ch * 8) = *reinterpret_cast<uint4*>(v);
   }
 }
 
@@ -63,20 +81,19 @@ __global__ void pack32_kernel(const float* __restrict__ x, float* __restrict__ y
   }
 }
 
-cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int Cp,
-                              int dt, cudaStream_t st) {
-  const int HW = H * W;
+cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f,
+                              int Ho, int Wo, int Cp, int dt, cudaStream_t st) {
   const int T = 256;
   if (dt == DT_F32) {
-    int64_t n = rows * (int64_t)HW * Cp;
-    pack32_kernel<<<min(nblocks(n, T), 148 * 32), T, 0, st>>>(x, (float*)y, rows, C, HW, Cp);
+    int64_t n = rows * (int64_t)H * W * Cp;
+    pack32_kernel<<<min(nblocks(n, T), 148 * 32), T, 0, st>>>(x, (float*)y, rows, C, H * W, Cp);
   } else {
-    int64_t n = rows * (int64_t)(Cp / 8) * HW;
+    const int per_row = Ho * Wo * (Cp / 8);
+    dim3 g(min(nblocks(per_row, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
     if (dt == DT_F16)
-      pack16_kernel<__half><<<min(nblocks(n, T), 148 * 32), T, 0, st>>>(x, (__half*)y, rows, C, HW, Cp);
+      pack16_kernel<__half><<<g, T, 0, st>>>(x, (__half*)y, rows, C, H, W, mode, f, Ho, Wo, Cp);
     else
-      pack16_kernel<__nv_bfloat16>
-          <<<min(nblocks(n, T), 148 * 32), T, 0, st>>>(x, (__nv_bfloat16*)y, rows, C, HW, Cp);
+      pack16_kernel<__nv_bfloat16><<<g, T, 0, st>>>(x, (__nv_bfloat16*)y, rows, C, H, W, mode, f, Ho, Wo, Cp);
   }
   return cudaGetLastError();
 }
@@ -144,10 +161,55 @@ __global__ void pool_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t 
   }
 }
 
+// 16-bit storage: 8 channels (16 B) per thread, fp32 math.
+template <typename T>
+__global__ void pool16_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t rows, int Cp, int H, int W,
+                              int OH, int OW, int kern, int stride, int pad, int is_max) {
+  const int chunks = Cp / 8;
+  const int per_row = OH * OW * chunks;
+  for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
+    const T* xr = x + r * (int64_t)H * W * Cp;
+    T* yr = y + r * (int64_t)per_row * 8;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < per_row; i += gridDim.x * blockDim.x) {
+      const int ch = i % chunks;
+      const int pix = i / chunks;
+      const int oy = pix / OW, ox = pix - (pix / OW) * OW;
+      int hs = oy * stride - pad, ws = ox * stride - pad;
+      int he = min(hs + kern, H + pad), we = min(ws + kern, W + pad);
+      const float area = (float)((he - hs) * (we - ws));
+      hs = max(hs, 0); ws = max(ws, 0); he = min(he, H); we = min(we, W);
+      const T* base = xr + ch * 8;
+      float acc[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) acc[j] = is_max ? -FLT_MAX : 0.f;
+      for (int h = hs; h < he; ++h)
+        for (int w = ws; w < we; ++w) {
+          const uint4 u = __ldg(reinterpret_cast<const uint4*>(base + (h * W + w) * Cp));
+          const T* v = reinterpret_cast<const T*>(&u);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) acc[j] = is_max ? fmaxf(acc[j], ld(v + j)) : acc[j] + ld(v + j);
+        }
+      __align__(16) T o[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) o[j] = cvt<T>(is_max ? acc[j] : acc[j] / area);
+      *reinterpret_cast<uint4*>(yr + i * 8) = *reinterpret_cast<const uint4*>(o);
+    }
+  }
+}
+
 cudaError_t launch_pool(const void* x, void* y, int64_t rows, int C, int Cp, int H, int W, int OH,
                         int OW, int kernel, int stride, int pad, int is_max, int dt, cudaStream_t st) {
   (void)C;
   const int T = 256;
+  if (dt != DT_F32 && Cp % 8 == 0) {
+    const int per_row = OH * OW * (Cp / 8);
+    dim3 g(min(nblocks(per_row, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
+    if (dt == DT_F16)
+      pool16_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
+    else
+      pool16_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
+    return cudaGetLastError();
+  }
   const int64_t n = rows * (int64_t)OH * OW * Cp;
   const int g = min(nblocks(n, T), 148 * 32);
   if (dt == DT_F32) pool_kernel<float><<<g, T, 0, st>>>((const float*)x, (float*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);

@@ -1,20 +1,28 @@
 // K1/K2/K3: tcgen05 tensor-core implicit GEMM for fully-connected, convolution and
-// locally-connected layers with bias + activation fused in the epilogue.
+// locally-connected layers, bias + activation (+ optional LRN) fused in the epilogue.
 //
 // What it computes ("each neuron computes a weighted sum of its inputs";
 // L65: "the learned weights are kernels that are convolved with the image"; L185:
 // batching "increases the dimensions of the matrix multiplication"):
 //     Y[pix(m), goff(z) + n] = act( bias[z][n] + sum_k A[m,k] * B[z][n][k] )
-// with A gathered from the NHWC activations (implicit im2col) or read densely, B the
-// packed weights [Z][N][Kpad] (K-major), fp32 accumulation in TMEM.
+// A = the NHWC activations seen through an implicit im2col, B = packed weights
+// [Z][N][Kpad] (K-major, k = (ky, kx, c) with c fastest), fp32 accumulation in TMEM.
 //
-// Structure (Blackwell-native):
-//   warps 0-3  epilogue: tcgen05.ld TMEM -> registers, +bias, activation, 16-bit/fp32 stores
-//   warp  4    TMA producer: B tiles (3D tensor map, SWIZZLE_128B), dense A tiles (2D map)
-//   warp  5    TMEM allocator + single-thread tcgen05.mma issuer (M=128, N=BN, K=16)
-//   warps 6-9  (conv/LC) A gather producers: cp.async 16-byte chunks of 8 channels into the
-//              SWIZZLE_128B K-major layout, proxy-fenced, mbarrier-signalled
-// Ring of STAGES smem stages with full/empty mbarriers; tcgen05.commit frees a stage.
+// Blackwell structure:
+//   * persistent CTAs (grid <= #SMs), static tile striding; a tile = (m block of 128 rows,
+//     n block of BN columns, a group of zf z-slices accumulated side by side in TMEM)
+//   * warp 8: TMA producer.  A arrives in chunks of cw channels (one TMA box each):
+//       conv  -> im2col-mode TMA (the hardware walks 128 output pixels, applies the
+//                filter offset (kx,ky), zero-fills the padding)
+//       LC    -> tiled 4D TMA box {cw, 1, 1, 128 images} at the tap's input pixel
+//       dense -> tiled 2D TMA box {64, 128 rows}
+//     B arrives as a 3D tiled box {64, BN, 1}, SWIZZLE_128B.
+//   * warp 9: TMEM allocator + single-thread tcgen05.mma issuer (M=128, N=BN, K=16),
+//     tcgen05.commit frees smem stages and publishes finished accumulators
+//   * warps 0-7: epilogue, tcgen05.ld TMEM -> registers, +bias, activation, optional
+//     Caffe LRN across the pixel's channels, 16-bit / fp32 vector stores.  Warps w and w+4
+//     share TMEM lane quarter w%4 and split the columns; accumulators are double-buffered
+//     in TMEM so the epilogue of tile t overlaps the MMAs of tile t+1.
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
@@ -26,9 +34,7 @@ namespace djinn {
 namespace {
 
 constexpr int BM = 128, BK = 64;
-constexpr int TMA_WARP = 4, MMA_WARP = 5, GATHER_WARP0 = 6;
-constexpr int GATHER_THREADS = 128;
-constexpr int LAG = 2;  // cp.async groups kept in flight per gather thread
+constexpr int EPI_WARPS = 8, TMA_WARP = 8, MMA_WARP = 9, NUM_THREADS = 320;
 
 template <int BN>
 struct Cfg {
@@ -36,14 +42,11 @@ struct Cfg {
   static constexpr int B_BYTES = BN * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int STAGES = (200 * 1024) / STAGE_BYTES > 8 ? 8 : (200 * 1024) / STAGE_BYTES;
-  static constexpr int TMEM_COLS = BN < 32 ? 32 : BN;
-  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 256;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 512;
 };
 
 // ---------------------------------------------------------------- PTX helpers
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-  return (uint32_t)__cvta_generic_to_shared(p);
-}
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
 }
@@ -51,8 +54,7 @@ __device__ __forceinline__ void mbar_arrive(uint32_t bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
 __device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes)
-               : "memory");
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   uint32_t done, iters = 0;
@@ -64,52 +66,54 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
         : "=r"(done)
         : "r"(bar), "r"(parity)
         : "memory");
-    if (++iters > (1u << 26)) __trap();  // a lost arrival must fault, never hang the GPU
+    if (++iters > (1u << 28)) __trap();  // a lost arrival must fault, never hang the GPU
   } while (!done);
 }
-__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0,
-                                            int c1) {
+__device__ __forceinline__ void tma_2d(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1) {
   asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
-          dst),
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
       "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1)
       : "memory");
 }
-__device__ __forceinline__ void tma_load_3d(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0,
-                                            int c1, int c2) {
+__device__ __forceinline__ void tma_3d(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1, int c2) {
   asm volatile(
       "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(
           dst),
       "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
       : "memory");
 }
-__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, uint32_t src_bytes) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes)
-               : "memory");
+__device__ __forceinline__ void tma_4d(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1, int c2,
+                                       int c3) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], [%2];" ::"r"(
+          dst),
+      "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+      : "memory");
 }
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() {
-  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+// im2col mode: coordinates {c, w, h, n} = channel and the filter window's top-left input
+// position of the first of the 128 output pixels; offsets {kx, ky} select the tap.
+__device__ __forceinline__ void tma_im2col_4d(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c, int w,
+                                              int h, int n, uint16_t ox, uint16_t oy) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.im2col.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(dst),
+      "l"((uint64_t)map), "r"(bar), "r"(c), "r"(w), "r"(h), "r"(n), "h"(ox), "h"(oy)
+      : "memory");
 }
-__device__ __forceinline__ void fence_proxy_async() {
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
-__device__ __forceinline__ void tc_fence_before() {
-  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-}
-__device__ __forceinline__ void tc_fence_after() {
-  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+// UMMA shared-memory descriptor of a K-major swizzled tile: rows of `row_bytes` (32/64/128),
+// 8-row core groups `8*row_bytes` apart (SBO), LBO unused (1), version 1 (sm_100),
+// layout type SW32 = 6, SW64 = 4, SW128 = 2.
+__device__ __forceinline__ uint64_t sdesc(uint32_t saddr, int row_bytes) {
+  const uint64_t layout = row_bytes == 128 ? 2 : (row_bytes == 64 ? 4 : 6);
+  return (uint64_t)((saddr & 0x3FFFFu) >> 4) | ((uint64_t)1 << 16) | ((uint64_t)((8 * row_bytes) >> 4) << 32) |
+         ((uint64_t)1 << 46) | (layout << 61);
 }
 
-// UMMA shared-memory descriptor, K-major, SWIZZLE_128B canonical layout: rows of 128 B,
-// 8-row core groups 1024 B apart (SBO), LBO unused (1), version 1 (sm_100), layout 2.
-__device__ __forceinline__ uint64_t sdesc_sw128(uint32_t saddr) {
-  return (uint64_t)((saddr & 0x3FFFFu) >> 4) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
-         ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
-}
-
-// Instruction descriptor, kind::f16: D fp32, A/B fp16 (0) or bf16 (1), both K-major.
+// Instruction descriptor, kind::f16: D fp32, A/B fp16 (0) or bf16 (1), both K-major, M=128.
 template <int BN, bool BF16>
 __device__ __forceinline__ uint32_t idesc_f16() {
   const uint32_t ab = BF16 ? 1u : 0u;
@@ -125,27 +129,31 @@ __device__ __forceinline__ void mma_f16(uint32_t d_tmem, uint64_t adesc, uint64_
       : "memory");
 }
 __device__ __forceinline__ void mma_commit(uint32_t bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar)
-               : "memory");
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
 }
-
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
   asm volatile(
       "tcgen05.ld.sync.aligned.32x32b.x16.b32 "
       "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
-        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
-        "=r"(r[14]), "=r"(r[15])
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
       : "r"(taddr));
 }
 __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 
+__device__ __forceinline__ float tanh_approx(float v) {
+  float r;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(r) : "f"(v));
+  return r;
+}
+// Activations on MUFU (16-bit storage tolerates their ~2^-11..2^-21 relative error).
 __device__ __forceinline__ float act_fast(float v, int act) {
   switch (act) {
-    case ACT_RELU: return v > 0.f ? v : 0.f;
-    case ACT_SIGMOID: return 1.f / (1.f + __expf(-v));
-    case ACT_TANH: return tanhf(v);
+    case ACT_RELU: return fmaxf(v, 0.f);
+    case ACT_SIGMOID: return __fdividef(1.f, 1.f + __expf(-v));
+    case ACT_TANH: return tanh_approx(v);
     case ACT_HARDTANH: return fminf(fmaxf(v, -1.f), 1.f);
+    case ACT_SIGMOID_C: return __fdividef(1.f, 1.f + __expf(-v)) - 0.5f;  // sigma - 1/2 (abs. err ~1e-7)
     default: return v;
   }
 }
@@ -161,40 +169,81 @@ __device__ __forceinline__ uint32_t pack2(float a, float b) {
   }
 }
 
+template <bool BF16>
+__device__ __forceinline__ void store16(const GemmGeom& g, void* Y, int64_t off, const float (&v)[16], int nvalid8) {
+  if (g.out_f32) {
+    float* yp = reinterpret_cast<float*>(Y) + off;
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+      if (h < nvalid8) {
+        reinterpret_cast<float4*>(yp + 8 * h)[0] = make_float4(v[8 * h], v[8 * h + 1], v[8 * h + 2], v[8 * h + 3]);
+        reinterpret_cast<float4*>(yp + 8 * h)[1] = make_float4(v[8 * h + 4], v[8 * h + 5], v[8 * h + 6], v[8 * h + 7]);
+      }
+  } else {
+    uint16_t* yp = reinterpret_cast<uint16_t*>(Y) + off;
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+      if (h < nvalid8)
+        *reinterpret_cast<uint4*>(yp + 8 * h) =
+            make_uint4(pack2<BF16>(v[8 * h], v[8 * h + 1]), pack2<BF16>(v[8 * h + 2], v[8 * h + 3]),
+                       pack2<BF16>(v[8 * h + 4], v[8 * h + 5]), pack2<BF16>(v[8 * h + 6], v[8 * h + 7]));
+  }
+}
+
+struct TileCoord {
+  int m0, n0, z0;
+};
+__device__ __forceinline__ TileCoord tile_coord(int t, int mt, int nt) {
+  TileCoord c;
+  c.m0 = (t % mt) * BM;
+  t /= mt;
+  c.n0 = (t % nt);
+  c.z0 = t / nt;
+  return c;
+}
+
 // ---------------------------------------------------------------- the kernel
-template <int BN, bool GATHER, bool BF16>
-__global__ void __launch_bounds__(GATHER ? 320 : 192, 1)
+template <int BN, bool BF16>
+__global__ void __launch_bounds__(NUM_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                   const GemmGeom g, const uint16_t* __restrict__ A, const float* __restrict__ bias,
-                   void* __restrict__ Y) {
+                   const GemmGeom g, const float* __restrict__ bias, void* __restrict__ Y) {
   using C = Cfg<BN>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + C::STAGES * C::A_BYTES;
   uint64_t* bars = reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * C::STAGES + 1);
+  // bars: full[STAGES], empty[STAGES], tfull[2], tempty[2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * C::STAGES + 4);
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + C::STAGES);
-  const uint32_t tmem_full = smem_u32(bars + 2 * C::STAGES);
+  const uint32_t tfull0 = smem_u32(bars + 2 * C::STAGES), tempty0 = smem_u32(bars + 2 * C::STAGES + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int m0 = blockIdx.x * BM, n0 = blockIdx.y * BN, z = blockIdx.z;
   const int num_kb = g.Kpad / BK;
+  const int mt = (g.M + BM - 1) / BM, nt = (g.N + BN - 1) / BN, zt = g.Z / g.zf;
+  const int tiles = mt * nt * zt;
+  const int slot_cols = g.zf * BN;
+  const int nslots = 2 * slot_cols <= 512 ? 2 : 1;
+  int tcols = 32;
+  while (tcols < nslots * slot_cols) tcols <<= 1;
 
   if (warp == TMA_WARP && lane == 0) {
     for (int s = 0; s < C::STAGES; ++s) {
-      mbar_init(full0 + 8 * s, GATHER ? 1 + GATHER_THREADS : 1);
+      mbar_init(full0 + 8 * s, 1);
       mbar_init(empty0 + 8 * s, 1);
     }
-    mbar_init(tmem_full, 1);
+    for (int s = 0; s < 2; ++s) {
+      mbar_init(tfull0 + 8 * s, 1);
+      mbar_init(tempty0 + 8 * s, EPI_WARPS);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     fence_proxy_async();
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmA) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmB) : "memory");
-    if (!GATHER) asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmA) : "memory");
   }
   if (warp == MMA_WARP) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                 "r"((uint32_t)C::TMEM_COLS)
+                 "r"((uint32_t)tcols)
                  : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
@@ -205,170 +254,264 @@ __global__ void __launch_bounds__(GATHER ? 320 : 192, 1)
 
   if (warp == TMA_WARP) {
     if (lane == 0) {
-      for (int kb = 0; kb < num_kb; ++kb) {
-        const int s = kb % C::STAGES;
-        const uint32_t ph = (kb / C::STAGES) & 1;
-        mbar_wait(empty0 + 8 * s, ph ^ 1);
-        mbar_arrive_expect_tx(full0 + 8 * s, C::B_BYTES + (GATHER ? 0 : C::A_BYTES));
-        tma_load_3d(smem_u32(sB + s * C::B_BYTES), &tmB, full0 + 8 * s, kb * BK, n0, z);
-        if (!GATHER) tma_load_2d(smem_u32(sA + s * C::A_BYTES), &tmA, full0 + 8 * s, kb * BK, m0);
+      const int cw = g.cw, cbytes = BM * cw * 2, cpt = g.Cgp / cw;
+      const int nchunks_k = g.K / cw;  // valid chunks along K
+      int it = 0;
+      for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
+        const TileCoord tc = tile_coord(t, mt, nt);
+        // first output pixel of the tile (conv): top-left of its filter window in input coords
+        int img = 0, wy = 0, wx = 0;
+        if (g.mode == GM_CONV) {
+          img = tc.m0 / (g.OH * g.OW);
+          const int rem = tc.m0 - img * g.OH * g.OW;
+          const int oy = rem / g.OW, ox = rem - (rem / g.OW) * g.OW;
+          wy = oy * g.stride - g.pad;
+          wx = ox * g.stride - g.pad;
+        }
+        for (int zi = 0; zi < g.zf; ++zi) {
+          const int z = tc.z0 * g.zf + zi;
+          for (int kb = 0; kb < num_kb; ++kb, ++it) {
+            const int s = it % C::STAGES;
+            const uint32_t ph = (it / C::STAGES) & 1;
+            mbar_wait(empty0 + 8 * s, ph ^ 1);
+            const uint32_t fb = full0 + 8 * s;
+            mbar_arrive_expect_tx(fb, C::A_BYTES + C::B_BYTES);
+            const uint32_t a_dst = smem_u32(sA + s * C::A_BYTES);
+            if (g.mode == GM_DENSE) {
+              tma_2d(a_dst, &tmA, fb, kb * BK, tc.m0);
+            } else {
+              for (int j = 0; j < BK / cw; ++j) {
+                const int q = kb * (BK / cw) + j;
+                int c, kx = 0, ky = 0;
+                if (q < nchunks_k) {
+                  const int tap = q / cpt;
+                  c = (q - tap * cpt) * cw + (g.mode == GM_CONV ? z * g.cin_goff : 0);
+                  ky = tap / g.KW;
+                  kx = tap - ky * g.KW;
+                } else {
+                  c = g.Cp_in;  // past the channel extent: TMA zero-fills the K tail
+                }
+                const uint32_t dst = a_dst + j * cbytes;
+                if (g.mode == GM_CONV) {
+                  tma_im2col_4d(dst, &tmA, fb, c, wx, wy, img, (uint16_t)kx, (uint16_t)ky);
+                } else {  // LC: rows are images at the fixed output location z
+                  const int oy = z / g.OW, ox = z - (z / g.OW) * g.OW;
+                  tma_4d(dst, &tmA, fb, c, ox * g.stride + kx, oy * g.stride + ky, tc.m0);
+                }
+              }
+            }
+            tma_3d(smem_u32(sB + s * C::B_BYTES), &tmB, fb, kb * BK, tc.n0 * BN, z);
+          }
+        }
       }
     }
     __syncwarp();
   } else if (warp == MMA_WARP) {
     if (lane == 0) {
       const uint32_t idesc = idesc_f16<BN, BF16>();
-      for (int kb = 0; kb < num_kb; ++kb) {
-        const int s = kb % C::STAGES;
-        const uint32_t ph = (kb / C::STAGES) & 1;
-        mbar_wait(full0 + 8 * s, ph);
+      const int cw = g.mode == GM_DENSE ? 64 : g.cw, cbytes = BM * cw * 2;
+      int it = 0, lt = 0;
+      for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++lt) {
+        const int slot = nslots == 2 ? (lt & 1) : 0;
+        const uint32_t use = nslots == 2 ? (uint32_t)(lt >> 1) : (uint32_t)lt;
+        mbar_wait(tempty0 + 8 * slot, (use & 1) ^ 1);
         tc_fence_after();
-        const uint64_t ad = sdesc_sw128(smem_u32(sA + s * C::A_BYTES));
-        const uint64_t bd = sdesc_sw128(smem_u32(sB + s * C::B_BYTES));
+        for (int zi = 0; zi < g.zf; ++zi) {
+          const uint32_t d = tmem + (uint32_t)(slot * slot_cols + zi * BN);
+          for (int kb = 0; kb < num_kb; ++kb, ++it) {
+            const int s = it % C::STAGES;
+            const uint32_t ph = (it / C::STAGES) & 1;
+            mbar_wait(full0 + 8 * s, ph);
+            tc_fence_after();
+            const uint32_t a0 = smem_u32(sA + s * C::A_BYTES);
+            const uint64_t bd = sdesc(smem_u32(sB + s * C::B_BYTES), 128);
 #pragma unroll
-        for (int k = 0; k < BK / 16; ++k)  // advance 16 elements = 32 B = 2 descriptor units
-          mma_f16(tmem, ad + 2 * k, bd + 2 * k, idesc, (kb | k) != 0);
-        mma_commit(empty0 + 8 * s);
+            for (int k = 0; k < BK / 16; ++k) {
+              const int e = k * 16;  // element offset of this K step inside the stage
+              const uint64_t ad = sdesc(a0 + (e / cw) * cbytes + (e % cw) * 2, cw * 2);
+              mma_f16(d, ad, bd + 2 * k, idesc, (kb | k) != 0);
+            }
+            mma_commit(empty0 + 8 * s);
+          }
+        }
+        mma_commit(tfull0 + 8 * slot);
       }
-      mma_commit(tmem_full);
     }
     __syncwarp();
-  } else if (GATHER && warp >= GATHER_WARP0) {
-    // ---- implicit im2col producer: thread -> (chunk j, rows r0 + 16 i) ----
-    const int gt = threadIdx.x - GATHER_WARP0 * 32;
-    const int j = gt & 7, r0 = gt >> 3;
-    int img[8], iy0[8], ix0[8];
+  } else {
+    // ---- epilogue (warps 0-7): TMEM -> registers -> bias + act (+ LRN) -> global ----
+    const int quarter = warp & 3, half = warp >> 2;
+    int lt = 0;
+    const uint32_t lane_base = (uint32_t)(quarter * 32) << 16;
+    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++lt) {
+      const TileCoord tc = tile_coord(t, mt, nt);
+      const int slot = nslots == 2 ? (lt & 1) : 0;
+      const uint32_t use = nslots == 2 ? (uint32_t)(lt >> 1) : (uint32_t)lt;
+      mbar_wait(tfull0 + 8 * slot, use & 1);
+      tc_fence_after();
+      const int m = tc.m0 + quarter * 32 + lane;
+      const bool mok = m < g.M;
+      const uint32_t tbase = tmem + lane_base + (uint32_t)(slot * slot_cols);
+      if (g.epi_lrn) {
+        // Channels c = zi * N + n (N == BN when zf > 1) live in columns zi*BN + n.  The LRN
+        // window is clipped to [0, Ctot); values beyond are zero, so zero-padding is exact.
+        // Warp half h processes 16-channel chunks [ib, ie) with a one-chunk halo each side.
+        const int N = g.N, Ctot = g.zf * N;
+        const int nch = (Ctot + 15) / 16, per = (nch + 1) / 2;
+        const int ib = half * per, ie = min(nch, ib + per);
+        const int64_t obase = (int64_t)m * g.out_pitch;
+        float cur[16], nxt[16];
+        float pm2 = 0.f, pm1 = 0.f;
+        auto load_chunk = [&](int i, float (&v)[16]) {
+          const int c0 = i * 16;
+          const int zi = c0 / N, n0 = c0 - zi * N;
+          uint32_t r[16];
+          tmem_ld16(tbase + (uint32_t)(zi * BN + n0), r);
+          tmem_wait_ld();
 #pragma unroll
-    for (int i = 0; i < 8; ++i) {
-      const int m = m0 + r0 + 16 * i;
-      int im = m, oy, ox;
-      if (g.mode == GM_CONV) {
-        im = m / (g.OH * g.OW);
-        const int rem = m - im * g.OH * g.OW;
-        oy = rem / g.OW;
-        ox = rem - oy * g.OW;
+          for (int j = 0; j < 16; ++j) {
+            const int c = c0 + j;
+            v[j] = c < Ctot ? act_fast(__uint_as_float(r[j]) + __ldg(bias + c), g.act) : 0.f;
+          }
+        };
+        if (ib < ie) {
+          if (ib > 0) {
+            load_chunk(ib - 1, cur);
+            pm2 = cur[14] * cur[14];
+            pm1 = cur[15] * cur[15];
+          }
+          load_chunk(ib, cur);
+        }
+        for (int i = ib; i < ie; ++i) {
+          if (i + 1 < nch) {
+            load_chunk(i + 1, nxt);
+          } else {
+#pragma unroll
+            for (int j = 0; j < 16; ++j) nxt[j] = 0.f;
+          }
+          float sq[20];
+          sq[0] = pm2;
+          sq[1] = pm1;
+#pragma unroll
+          for (int j = 0; j < 16; ++j) sq[2 + j] = cur[j] * cur[j];
+          sq[18] = nxt[0] * nxt[0];
+          sq[19] = nxt[1] * nxt[1];
+          float o[16];
+#pragma unroll
+          for (int j = 0; j < 16; ++j) {
+            const float s5 = sq[j] + sq[j + 1] + sq[j + 2] + sq[j + 3] + sq[j + 4];  // window c-2 .. c+2
+            o[j] = cur[j] * __powf(g.lrn_k + g.lrn_alpha_over_n * s5, -g.lrn_beta);
+          }
+          pm2 = sq[16];
+          pm1 = sq[17];
+          if (mok) {
+            const int c0 = i * 16;
+            const int nvalid8 = min(2, (g.write_cols - c0 + 7) / 8);
+            if (nvalid8 > 0) store16<BF16>(g, Y, obase + c0, o, nvalid8);
+          }
+#pragma unroll
+          for (int j = 0; j < 16; ++j) cur[j] = nxt[j];
+        }
       } else {
-        oy = z / g.OW;
-        ox = z - oy * g.OW;
-      }
-      img[i] = im;
-      iy0[i] = m < g.M ? oy * g.stride - g.pad : -(1 << 28);
-      ix0[i] = ox * g.stride - g.pad;
-    }
-    const int CPT = g.Cgp >> 3;
-    const int cin = (g.mode == GM_CONV) ? z * g.cin_goff : 0;
-    const uint32_t swz = (uint32_t)((j ^ (r0 & 7)) << 4);
-    const uint16_t* Ab = A + cin;
-    for (int kb = 0; kb < num_kb; ++kb) {
-      const int s = kb % C::STAGES;
-      const uint32_t ph = (kb / C::STAGES) & 1;
-      mbar_wait(empty0 + 8 * s, ph ^ 1);
-      const int q = kb * 8 + j;
-      const bool kval = q * 8 < g.K;
-      const int tap = q / CPT, c8 = q - tap * CPT;
-      const int ky = tap / g.KW, kx = tap - ky * g.KW;
-      const uint32_t dst = smem_u32(sA + s * C::A_BYTES) + swz;
-#pragma unroll
-      for (int i = 0; i < 8; ++i) {
-        const int r = r0 + 16 * i;
-        const int iy = iy0[i] + ky, ix = ix0[i] + kx;
-        const bool ok = kval && iy >= 0 && iy < g.H && ix >= 0 && ix < g.W;
-        const uint16_t* src =
-            ok ? Ab + (((int64_t)img[i] * g.H + iy) * g.W + ix) * g.Cp_in + c8 * 8 : A;
-        cp_async16(dst + r * 128, src, ok ? 16u : 0u);
-      }
-      cp_async_commit();
-      if (kb >= LAG) {
-        cp_async_wait<LAG>();
-        fence_proxy_async();
-        mbar_arrive(full0 + 8 * ((kb - LAG) % C::STAGES));
-      }
-    }
-    cp_async_wait<0>();
-    fence_proxy_async();
-    for (int kb = num_kb - LAG < 0 ? 0 : num_kb - LAG; kb < num_kb; ++kb)
-      mbar_arrive(full0 + 8 * (kb % C::STAGES));
-  } else if (warp < 4) {
-    // ---- epilogue: TMEM -> registers -> bias + act -> global ----
-    mbar_wait(tmem_full, 0);
-    tc_fence_after();
-    const int row = warp * 32 + lane;
-    const int m = m0 + row;
-    const int64_t pix = (g.mode == GM_LC) ? (int64_t)m * g.OH * g.OW + z : (int64_t)m;
-    const int goff = (g.mode == GM_CONV) ? z * g.cout_goff : 0;
-    const float* bz = bias + (int64_t)z * g.bias_zstride;
+        // columns of each z-slice split between the two warps of a lane quarter
+        const int cols = BN >= 32 ? BN / 2 : BN;
+        const int cbeg = BN >= 32 ? half * cols : 0;
+        const bool active = BN >= 32 || half == 0;
+        for (int zi = 0; zi < g.zf && active; ++zi) {
+          const int z = tc.z0 * g.zf + zi;
+          const int64_t pix = (g.mode == GM_LC) ? (int64_t)m * g.OH * g.OW + z : (int64_t)m;
+          const int goff = (g.mode == GM_CONV) ? z * g.cout_goff : 0;
+          const float* bz = bias + (int64_t)z * g.bias_zstride;
+          const int nb0 = tc.n0 * BN;
 #pragma unroll 1
-    for (int c = 0; c < BN; c += 16) {
-      uint32_t r[16];
-      tmem_ld16(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c, r);
-      tmem_wait_ld();
-      const int nb = n0 + c;
-      if (m < g.M && nb < g.write_cols) {
-        float v[16];
+          for (int c = cbeg; c < cbeg + cols; c += 32) {
+            const int two = (c + 16 < cbeg + cols) ? 2 : 1;
+            uint32_t r[2][16];
+            tmem_ld16(tbase + (uint32_t)(zi * BN + c), r[0]);
+            if (two == 2) tmem_ld16(tbase + (uint32_t)(zi * BN + c + 16), r[1]);
+            tmem_wait_ld();
 #pragma unroll
-        for (int t = 0; t < 16; ++t) {
-          const int n = nb + t;
-          v[t] = n < g.N ? act_fast(__uint_as_float(r[t]) + __ldg(bz + n), g.act) : 0.f;
-        }
-        if (g.out_f32) {
-          float* yp = reinterpret_cast<float*>(Y) + pix * g.out_pitch + goff + nb;
+            for (int hh = 0; hh < 2; ++hh) {
+              if (hh >= two) break;
+              const int nb = nb0 + c + 16 * hh;
+              if (mok && nb < g.write_cols) {
+                float v[16];
+                if (nb + 16 <= g.N) {
+                  float b[16];
 #pragma unroll
-          for (int h = 0; h < 2; ++h)
-            if (nb + 8 * h < g.write_cols) {
-              reinterpret_cast<float4*>(yp + 8 * h)[0] = make_float4(v[8 * h], v[8 * h + 1], v[8 * h + 2], v[8 * h + 3]);
-              reinterpret_cast<float4*>(yp + 8 * h)[1] = make_float4(v[8 * h + 4], v[8 * h + 5], v[8 * h + 6], v[8 * h + 7]);
+                  for (int q = 0; q < 4; ++q) *reinterpret_cast<float4*>(b + 4 * q) = __ldg(reinterpret_cast<const float4*>(bz + nb) + q);
+#pragma unroll
+                  for (int j = 0; j < 16; ++j) v[j] = act_fast(__uint_as_float(r[hh][j]) + b[j], g.act);
+                } else {
+#pragma unroll
+                  for (int j = 0; j < 16; ++j) {
+                    const int n = nb + j;
+                    v[j] = n < g.N ? act_fast(__uint_as_float(r[hh][j]) + __ldg(bz + n), g.act) : 0.f;
+                  }
+                }
+                store16<BF16>(g, Y, pix * g.out_pitch + goff + nb, v, min(2, (g.write_cols - nb + 7) / 8));
+              }
             }
-        } else {
-          uint16_t* yp = reinterpret_cast<uint16_t*>(Y) + pix * g.out_pitch + goff + nb;
-#pragma unroll
-          for (int h = 0; h < 2; ++h)
-            if (nb + 8 * h < g.write_cols)
-              *reinterpret_cast<uint4*>(yp + 8 * h) =
-                  make_uint4(pack2<BF16>(v[8 * h], v[8 * h + 1]), pack2<BF16>(v[8 * h + 2], v[8 * h + 3]),
-                             pack2<BF16>(v[8 * h + 4], v[8 * h + 5]), pack2<BF16>(v[8 * h + 6], v[8 * h + 7]));
+          }
         }
       }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(tempty0 + 8 * slot);
     }
   }
   tc_fence_before();
   __syncthreads();
   if (warp == MMA_WARP) {
     tc_fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"((uint32_t)C::TMEM_COLS)
-                 : "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"((uint32_t)tcols) : "memory");
   }
 }
 
-template <int BN, bool GATHER, bool BF16>
-cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtensorMap* tmB, const void* A,
-                        const float* bias, void* Y, cudaStream_t st) {
+int g_num_sms = 0;
+
+template <int BN, bool BF16>
+cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtensorMap* tmB, const float* bias, void* Y,
+                        cudaStream_t st) {
   using C = Cfg<BN>;
   static bool attr_set = false;  // benign race: idempotent attribute set
-  auto kern = tc_gemm_kernel<BN, GATHER, BF16>;
+  auto kern = tc_gemm_kernel<BN, BF16>;
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  dim3 grid((g.M + BM - 1) / BM, (g.N + BN - 1) / BN, g.Z);
-  kern<<<grid, GATHER ? 320 : 192, C::SMEM, st>>>(*tmA, *tmB, g, reinterpret_cast<const uint16_t*>(A), bias, Y);
+  const int64_t tiles = (int64_t)((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN) * (g.Z / g.zf);
+  const int grid = (int)(tiles < tc_num_sms() ? tiles : tc_num_sms());
+  kern<<<grid, NUM_THREADS, C::SMEM, st>>>(*tmA, *tmB, g, bias, Y);
   return cudaGetLastError();
 }
 
-template <bool GATHER, bool BF16>
-cudaError_t launch_bn(const GemmGeom& g, int bn, const CUtensorMap* tmA, const CUtensorMap* tmB, const void* A,
-                      const float* bias, void* Y, cudaStream_t st) {
+template <bool BF16>
+cudaError_t launch_bn(const GemmGeom& g, int bn, const CUtensorMap* tmA, const CUtensorMap* tmB, const float* bias,
+                      void* Y, cudaStream_t st) {
   switch (bn) {
-    case 16: return launch_inst<16, GATHER, BF16>(g, tmA, tmB, A, bias, Y, st);
-    case 32: return launch_inst<32, GATHER, BF16>(g, tmA, tmB, A, bias, Y, st);
-    case 64: return launch_inst<64, GATHER, BF16>(g, tmA, tmB, A, bias, Y, st);
-    case 128: return launch_inst<128, GATHER, BF16>(g, tmA, tmB, A, bias, Y, st);
-    case 256: return launch_inst<256, GATHER, BF16>(g, tmA, tmB, A, bias, Y, st);
+    case 16: return launch_inst<16, BF16>(g, tmA, tmB, bias, Y, st);
+    case 32: return launch_inst<32, BF16>(g, tmA, tmB, bias, Y, st);
+    case 64: return launch_inst<64, BF16>(g, tmA, tmB, bias, Y, st);
+    case 128: return launch_inst<128, BF16>(g, tmA, tmB, bias, Y, st);
+    case 256: return launch_inst<256, BF16>(g, tmA, tmB, bias, Y, st);
     default: return cudaErrorInvalidValue;
   }
 }
 
 }  // namespace
+
+int tc_num_sms() {
+  if (!g_num_sms) {
+    int dev = 0, n = 148;
+    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess)
+      g_num_sms = n;
+    else
+      g_num_sms = 148;
+  }
+  return g_num_sms;
+}
 
 int tc_pick_bn(const GemmGeom& g) {
   const int n = g.N;
@@ -376,19 +519,14 @@ int tc_pick_bn(const GemmGeom& g) {
   if (n <= 32) return 32;
   if (n <= 64) return 64;
   if (n <= 128) return 128;
-  const int64_t mt = (g.M + BM - 1) / BM;
-  const int64_t ctas256 = mt * ((n + 255) / 256) * g.Z;
-  return ctas256 >= 2 * 148 ? 256 : 128;
+  return 256;
 }
 
 cudaError_t launch_tc_gemm(const GemmGeom& g, int bn, int dt, const CUtensorMap* tmA, const CUtensorMap* tmB,
-                           const void* A, const float* bias, void* Y, cudaStream_t st) {
-  const bool gather = g.mode != GM_DENSE;
-  if (dt == DT_BF16)
-    return gather ? launch_bn<true, true>(g, bn, tmA, tmB, A, bias, Y, st)
-                  : launch_bn<false, true>(g, bn, tmA, tmB, A, bias, Y, st);
-  return gather ? launch_bn<true, false>(g, bn, tmA, tmB, A, bias, Y, st)
-                : launch_bn<false, false>(g, bn, tmA, tmB, A, bias, Y, st);
+                           const float* bias, void* Y, cudaStream_t st) {
+  if (g.M <= 0) return cudaSuccess;
+  if (dt == DT_BF16) return launch_bn<true>(g, bn, tmA, tmB, bias, Y, st);
+  return launch_bn<false>(g, bn, tmA, tmB, bias, Y, st);
 }
 
 }  // namespace djinn

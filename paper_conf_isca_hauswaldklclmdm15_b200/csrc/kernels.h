@@ -9,7 +9,10 @@
 namespace djinn {
 
 enum DType { DT_F32 = 0, DT_BF16 = 1, DT_F16 = 2 };
-enum Act { ACT_NONE = 0, ACT_RELU = 1, ACT_SIGMOID = 2, ACT_TANH = 3, ACT_HARDTANH = 4 };
+// ACT_SIGMOID_C stores sigma(x) - 1/2 ("centered" storage, an exact reparametrisation: the
+// consumer's bias absorbs + 1/2 * rowsum(W)); it keeps 16-bit activations near 0 where their
+// relative precision is best.
+enum Act { ACT_NONE = 0, ACT_RELU = 1, ACT_SIGMOID = 2, ACT_TANH = 3, ACT_HARDTANH = 4, ACT_SIGMOID_C = 5 };
 enum GemmMode { GM_DENSE = 0, GM_CONV = 1, GM_LC = 2 };
 
 // One convolution / locally-connected / fully-connected layer as an implicit GEMM:
@@ -38,11 +41,20 @@ struct GemmGeom {
   int bias_zstride;   // bias elements between z (LC: Co per location; conv: Cog)
   int act;
   int out_f32;        // 1: fp32 output (logits), 0: same 16-bit type as input
+  // tensor-core path only
+  int cw;             // A chunk width in elements (16 / 32 / 64): one TMA box per chunk
+  int zf;             // z values fused per CTA (groups computed by one CTA; TMEM columns zf*BN)
+  int epi_lrn;        // 1: Caffe LRN across the zf*N channels of a pixel in the epilogue
+  int lrn_size;
+  float lrn_alpha_over_n, lrn_beta, lrn_k;
 };
 
 // --- pack (K0): fp32 NCHW rows -> NHWC with channel pitch Cp, type dt -------------------
-cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int Cp,
-                              int dt, cudaStream_t st);
+// mode 0: y[r][h][w][c] = x[r][c][h][w];  mode 1 (space-to-depth by f):
+// y[r][ty][tx][(dy*f+dx)*C + c] = x[r][c][f*ty+dy][f*tx+dx];  mode 2 (kx-unroll of width f):
+// y[r][h][w][kx*C + c] = x[r][c][h][w+kx].  Out-of-range sources and pad channels are 0.
+cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f,
+                              int Ho, int Wo, int Cp, int dt, cudaStream_t st);
 
 // --- SIMT fp32 implicit GEMM (K7; exact fp32 FFMA accumulation) --------------------------
 // B: [Z][N][K] fp32 (K unpadded), bias fp32.
@@ -51,11 +63,14 @@ cudaError_t launch_simt_gemm(const GemmGeom& g, const float* A, const float* B, 
 
 // --- tcgen05 tensor-core implicit GEMM (K1/K2/K3) -----------------------------------------
 // tmB: 3D tensor map over B [Z][N][Kpad] (16-bit, SWIZZLE_128B, box {64, BN, 1}).
-// tmA: 2D tensor map over dense A [M][a_pitch] (box {64, 128}); unused for gather modes.
+// tmA: conv -> 4D im2col map over the NHWC input (channelsPerPixel = cw, 128 pixels);
+//      LC   -> 4D tiled map over the NHWC input, box {cw, 1, 1, 128};
+//      dense-> 2D tiled map over [rows][a_pitch], box {64, 128}.
+// Swizzle of A boxes: cw*2 bytes (32B / 64B / 128B).
 int tc_pick_bn(const GemmGeom& g);
+int tc_num_sms();
 cudaError_t launch_tc_gemm(const GemmGeom& g, int bn, int dt, const CUtensorMap* tmA,
-                           const CUtensorMap* tmB, const void* A, const float* bias, void* Y,
-                           cudaStream_t st);
+                           const CUtensorMap* tmB, const float* bias, void* Y, cudaStream_t st);
 
 // --- LRN across channels (K4), NHWC ----------------------------------------------------------
 cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, int size, float alpha,

@@ -142,17 +142,47 @@ static EncodeTiledFn encode_fn() {
   return fn;
 }
 
+static CUtensorMapSwizzle swizzle_for(int row_bytes) {
+  return row_bytes >= 128 ? CU_TENSOR_MAP_SWIZZLE_128B : row_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
+}
+
 void encode_tmap(CUtensorMap* m, int dt, const void* base, int rank, const uint64_t* dims, const uint64_t* strides_bytes,
-                 const uint32_t* box) {
+                 const uint32_t* box, int swizzle_bytes) {
   cuuint64_t d[5], s[4];
   cuuint32_t b[5], es[5];
   for (int i = 0; i < rank; ++i) { d[i] = dims[i]; b[i] = box[i]; es[i] = 1; }
   for (int i = 0; i + 1 < rank; ++i) s[i] = strides_bytes[i];
   const CUtensorMapDataType ty = dt == DT_F16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16;
   CUresult r = encode_fn()(m, ty, (cuuint32_t)rank, const_cast<void*>(base), d, s, b, es,
-                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle_for(swizzle_bytes),
                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) throw Error(DJINN_E_CUDA, "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")");
+}
+
+typedef CUresult (*EncodeIm2colFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const int*, const int*, cuuint32_t, cuuint32_t, const cuuint32_t*,
+                                   CUtensorMapInterleave, CUtensorMapSwizzle, CUtensorMapL2promotion,
+                                   CUtensorMapFloatOOBfill);
+
+void encode_im2col(CUtensorMap* m, int dt, const void* base, const uint64_t* dims, const uint64_t* strides_bytes,
+                   const int* lower_wh, const int* upper_wh, int channels, int pixels, const uint32_t* elem_strides) {
+  static EncodeIm2colFn fn = nullptr;
+  if (!fn) {
+    cudaDriverEntryPointQueryResult q;
+    void* p = nullptr;
+    ck(cudaGetDriverEntryPoint("cuTensorMapEncodeIm2col", &p, cudaEnableDefault, &q), "cuTensorMapEncodeIm2col lookup");
+    if (q != cudaDriverEntryPointSuccess || !p) throw Error(DJINN_E_CUDA, "cuTensorMapEncodeIm2col unavailable");
+    fn = (EncodeIm2colFn)p;
+  }
+  cuuint64_t d[4], s[3];
+  cuuint32_t es[4];
+  for (int i = 0; i < 4; ++i) { d[i] = dims[i]; es[i] = elem_strides[i]; }
+  for (int i = 0; i < 3; ++i) s[i] = strides_bytes[i];
+  const CUtensorMapDataType ty = dt == DT_F16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16;
+  CUresult r = fn(m, ty, 4, const_cast<void*>(base), d, s, lower_wh, upper_wh, (cuuint32_t)channels, (cuuint32_t)pixels, es,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle_for(channels * 2), CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) throw Error(DJINN_E_CUDA, "cuTensorMapEncodeIm2col failed (" + std::to_string((int)r) + ")");
 }
 
 static inline int rup(int v, int m) { return (v + m - 1) / m * m; }
@@ -221,7 +251,9 @@ void Net::build(const std::string& desc) {
   if (layers.back().type != "Softmax") throw Error(DJINN_E_UNSUPPORTED, "last layer must be Softmax");
 
   const bool f16 = dt != DT_F32;
-  auto pitch = [&](int c) { return f16 ? rup(c, 8) : c; };
+  // 16-bit activations: channel pitch a multiple of 16 so every conv's K splits into TMA
+  // chunks of 16/32/64 channels (one swizzle atom row of 32/64/128 B)
+  auto pitch = [&](int c) { return f16 ? rup(c, 16) : c; };
   const std::vector<int>& d = layers[0].dims;
   Shape cur;
   if (d.size() == 1) { cur.C = d[0]; }
@@ -333,10 +365,12 @@ void Net::build(const std::string& desc) {
       if (lc && L.pad != 0) throw Error(DJINN_E_UNSUPPORTED, L.name + ": padded LocallyConnected");
       if (grp <= 0 || cur.C % grp || L.num_output % grp) throw Error(DJINN_E_SHAPE, L.name + ": group does not divide channels");
       const int Cg = cur.C / grp, Cog = L.num_output / grp;
-      if (f16 && grp > 1 && (Cg % 8 || Cog % 8))
-        throw Error(DJINN_E_UNSUPPORTED, L.name + ": grouped conv needs channels per group % 8 == 0 on 16-bit paths");
+      if (f16 && grp > 1 && (Cg % 16 || Cog % 8))
+        throw Error(DJINN_E_UNSUPPORTED, L.name + ": grouped conv needs Cin/group % 16 == 0 and Cout/group % 8 == 0 on 16-bit paths");
       const int OH = (cur.H + 2 * pad - L.kernel) / L.stride + 1, OW = (cur.W + 2 * pad - L.kernel) / L.stride + 1;
       if (cur.H + 2 * pad < L.kernel || cur.W + 2 * pad < L.kernel) throw Error(DJINN_E_SHAPE, L.name + ": kernel larger than input");
+      o.orig_in = cur;
+      o.orig_k = L.kernel;
       g.mode = lc ? GM_LC : GM_CONV;
       g.N = Cog;
       g.Z = lc ? OH * OW : grp;
@@ -347,13 +381,58 @@ void Net::build(const std::string& desc) {
       g.pad = pad;
       g.Cgp = (grp == 1) ? cur.Cp : Cg;
       g.cin_goff = Cg;
-      g.K = L.kernel * L.kernel * g.Cgp;
+      // First layer with few channels on the tensor-core path: repack the input so that K
+      // is dense.  Strided kernels: space-to-depth by the stride (k x k / s  ->  ceil(k/s)^2
+      // taps over s*s*C channels, stride 1).  Stride 1: unroll kx into channels (k x k -> k x 1).
+      if (f16 && !lc && grp == 1 && ops.size() == 1 && cur.C < 16 && pad == 0) {
+        Op& pk = ops[0];
+        const int f = L.stride, k = L.kernel;
+        if (f > 1) {
+          const int Hs = (cur.H + f - 1) / f, Ws = (cur.W + f - 1) / f, ks = (k + f - 1) / f;
+          if (Hs - ks + 1 >= OH && Ws - ks + 1 >= OW) {
+            pk.xform = o.xform = 1;
+            pk.xf = o.xf = f;
+            pk.out.C = f * f * cur.C; pk.out.H = Hs; pk.out.W = Ws; pk.out.Cp = pitch(f * f * cur.C);
+            g.H = Hs; g.W = Ws; g.Cp_in = g.Cgp = pk.out.Cp;
+            g.KH = g.KW = ks;
+            g.stride = 1;
+          }
+        } else {
+          pk.xform = o.xform = 2;
+          pk.xf = o.xf = k;
+          pk.out.C = k * cur.C; pk.out.H = cur.H; pk.out.W = cur.W - k + 1; pk.out.Cp = pitch(k * cur.C);
+          g.H = cur.H; g.W = cur.W - k + 1; g.Cp_in = g.Cgp = pk.out.Cp;
+          g.KH = k; g.KW = 1;
+        }
+        if (pk.xform) { o.in = pk.out; }
+      }
+      g.K = g.KH * g.KW * g.Cgp;
       o.out.C = L.num_output; o.out.H = OH; o.out.W = OW; o.out.Cp = pitch(L.num_output);
       g.out_pitch = o.out.Cp;
       g.cout_goff = Cog;
       g.write_cols = grp == 1 ? o.out.Cp : Cog;
       g.bias_zstride = Cog;
       o.ohw = lc ? 1 : OH * OW;
+      g.zf = 1;
+      g.cw = g.Cgp % 64 == 0 ? 64 : (g.Cgp % 32 == 0 ? 32 : 16);
+      // Caffe LRN right after (the activation of) this conv: fuse it into the epilogue when one
+      // tile holds every channel of a pixel (all groups side by side in TMEM).
+      if (f16 && !lc && i + 1 < layers.size() && layers[i + 1].type == "LRN" && layers[i + 1].lrn_size == 5) {
+        const int bn = tc_pick_bn(g);
+        if (Cog <= 256 && (grp == 1 || bn == Cog) && grp * bn <= 256) {
+          const LayerSpec& R = layers[i + 1];
+          g.epi_lrn = 1;
+          g.zf = grp;
+          g.lrn_size = R.lrn_size;
+          g.lrn_alpha_over_n = R.alpha / R.lrn_size;
+          g.lrn_beta = R.beta;
+          g.lrn_k = R.lrn_k;
+          g.write_cols = o.out.Cp;
+          o.name += "+" + R.name;
+          ++i;
+          ++n_layers;
+        }
+      }
       wcount = lc ? (int64_t)OH * OW * L.num_output * cur.C * L.kernel * L.kernel
                   : (int64_t)L.num_output * Cg * L.kernel * L.kernel;
       bcount = lc ? (int64_t)L.num_output * OH * OW : L.num_output;
@@ -363,6 +442,8 @@ void Net::build(const std::string& desc) {
       g.Z = 1;
       g.K = (int)cur.per_row();
       g.a_pitch = g.K;
+      g.zf = 1;
+      g.cw = 64;
       o.out.C = L.num_output; o.out.H = 1; o.out.W = 1;
       o.out.Cp = last ? rup(L.num_output, 8) : pitch(L.num_output);
       g.out_pitch = o.out.Cp;
@@ -393,6 +474,42 @@ void Net::build(const std::string& desc) {
   }
   out_elems = cur.C;
   arena_bytes = rupz(arena_off, 1024);
+  // Centered sigmoid storage on 16-bit paths: a sigmoid layer feeding a dense layer stores
+  // sigma(x) - 1/2 and the consumer's bias absorbs 1/2 * rowsum(W) (exact reparametrisation).
+  if (f16)
+    for (size_t i = 0; i + 1 < ops.size(); ++i)
+      if (ops[i].kind == OP_GEMM && ops[i].g.act == ACT_SIGMOID && ops[i + 1].kind == OP_GEMM &&
+          ops[i + 1].g.mode == GM_DENSE) {
+        ops[i].g.act = ACT_SIGMOID_C;
+        ops[i + 1].fold_half = true;
+      }
+  // algorithmic work per op (real, unpadded dimensions)
+  const double es = f16 ? 2.0 : 4.0;
+  for (Op& o : ops) {
+    const Shape& oin = (o.kind == OP_GEMM && o.g.mode != GM_DENSE) ? o.orig_in : o.in;
+    const double in_e = (double)oin.C * oin.H * oin.W, out_e = (double)o.out.C * o.out.H * o.out.W;
+    switch (o.kind) {
+      case OP_PACK: o.bytes_row = in_e * 4 + in_e * es; break;
+      case OP_GEMM: {
+        const GemmGeom& g = o.g;
+        double kreal;
+        if (g.mode == GM_DENSE) kreal = in_e;
+        else if (g.mode == GM_LC) kreal = (double)o.orig_k * o.orig_k * oin.C;
+        else kreal = (double)o.orig_k * o.orig_k * (oin.C / (g.zf > 1 ? g.zf : g.Z));
+        o.flops_row = 2.0 * out_e * kreal;
+        o.bytes_row = in_e * es + out_e * (g.out_f32 ? 4.0 : es);
+        const double nb = g.mode == GM_DENSE ? g.N : (double)g.Z * g.bias_zstride;
+        o.weight_bytes = (g.mode == GM_LC ? (double)g.Z * g.N * kreal
+                                          : (g.mode == GM_CONV ? (double)o.out.C * kreal : (double)g.N * kreal)) * es +
+                         nb * 4;
+        if (g.mode == GM_CONV && g.zf > 1) o.flops_row = 2.0 * out_e * kreal;
+        break;
+      }
+      case OP_LRN: o.bytes_row = 2 * in_e * es; break;
+      case OP_POOL: o.bytes_row = in_e * es + out_e * es; break;
+      case OP_SOFTMAX: o.bytes_row = 2.0 * in_e * 4; break;
+    }
+  }
   for (const Op& o : ops) {
     if (o.kind == OP_SOFTMAX || o.out_buf < 0) continue;
     const size_t es = o.out_buf == 2 ? 4 : (f16 ? 2 : 4);
@@ -419,22 +536,35 @@ void Net::load_weights(const float* w, size_t n, int mem) {
     const GemmGeom& g = o.g;
     uint8_t* wdst = host.data() + o.w_off;
     float* bdst = reinterpret_cast<float*>(host.data() + o.b_off);
+    std::vector<double> rowsum(o.fold_half ? g.N : 0, 0.0);
     auto put = [&](int64_t z, int64_t nn, int64_t k, float v) {
       const int64_t idx = (z * g.N + nn) * g.Kpad + k;
       if (!f16) { reinterpret_cast<float*>(wdst)[idx] = v; return; }
       uint16_t bits;
-      if (dt == DT_BF16) { __nv_bfloat16 h = __float2bfloat16_rn(v); memcpy(&bits, &h, 2); }
-      else { __half h = __float2half_rn(v); memcpy(&bits, &h, 2); }
+      float r;
+      if (dt == DT_BF16) { __nv_bfloat16 h = __float2bfloat16_rn(v); memcpy(&bits, &h, 2); r = __bfloat162float(h); }
+      else { __half h = __float2half_rn(v); memcpy(&bits, &h, 2); r = __half2float(h); }
+      if (o.fold_half) rowsum[nn] += r;
       reinterpret_cast<uint16_t*>(wdst)[idx] = bits;
     };
     const int C = o.in.C, H = o.in.H, W = o.in.W, Cp = o.in.Cp;
     if (g.mode == GM_CONV) {
-      const int grp = g.Z, Cg = C / grp, k = g.KH;
+      const int grp = g.Z, C0 = o.orig_in.C, Cg = C0 / grp, k = o.orig_k;
       for (int co = 0; co < o.out.C; ++co)
         for (int c = 0; c < Cg; ++c)
           for (int ky = 0; ky < k; ++ky)
-            for (int kx = 0; kx < k; ++kx)
-              put(co / g.N, co % g.N, (int64_t)(ky * k + kx) * g.Cgp + c, w[off++]);
+            for (int kx = 0; kx < k; ++kx) {
+              int64_t kk;
+              if (o.xform == 1) {  // space-to-depth: tap (ky/f, kx/f), channel ((ky%f)*f + kx%f)*C0 + c
+                const int f = o.xf;
+                kk = (int64_t)((ky / f) * g.KW + kx / f) * g.Cgp + ((ky % f) * f + kx % f) * C0 + c;
+              } else if (o.xform == 2) {  // kx-unroll: tap ky, channel kx*C0 + c
+                kk = (int64_t)ky * g.Cgp + kx * C0 + c;
+              } else {
+                kk = (int64_t)(ky * k + kx) * g.Cgp + c;
+              }
+              put(co / g.N, co % g.N, kk, w[off++]);
+            }
       for (int co = 0; co < o.out.C; ++co) bdst[co] = w[off++];
     } else if (g.mode == GM_LC) {
       const int k = g.KH;
@@ -453,7 +583,7 @@ void Net::load_weights(const float* w, size_t n, int mem) {
           for (int h = 0; h < H; ++h)
             for (int x = 0; x < W; ++x)
               put(0, nn, ((int64_t)h * W + x) * Cp + c, w[off++]);
-      for (int nn = 0; nn < g.N; ++nn) bdst[nn] = w[off++];
+      for (int nn = 0; nn < g.N; ++nn) bdst[nn] = (float)(w[off++] + (o.fold_half ? 0.5 * rowsum[nn] : 0.0));
     }
   }
   if (off != n) throw Error(DJINN_E_WEIGHTS, "internal: blob walk mismatch");
@@ -467,7 +597,22 @@ Workspace::~Workspace() {
   if (out_stage) cudaFree(out_stage);
 }
 
+cudaEvent_t Net::prof_event() {
+  if (prof_used == prof_events.size()) {
+    cudaEvent_t e;
+    ck(cudaEventCreate(&e), "cudaEventCreate");
+    prof_events.push_back(e);
+  }
+  return prof_events[prof_used++];
+}
+
+void Net::prof_clear() {
+  prof_used = 0;
+  prof_recs.clear();
+}
+
 Net::~Net() {
+  for (cudaEvent_t e : prof_events) cudaEventDestroy(e);
   ws.clear();
   if (arena) cudaFree(arena);
 }
@@ -486,11 +631,28 @@ Workspace* Net::workspace(cudaStream_t st) {
   if (dt != DT_F32) {
     for (size_t i = 0; i < ops.size(); ++i) {
       const Op& o = ops[i];
-      if (o.kind != OP_GEMM || o.g.mode != GM_DENSE) continue;
-      uint64_t dims[2] = {(uint64_t)o.g.a_pitch, (uint64_t)max_rows};
-      uint64_t strides[1] = {(uint64_t)o.g.a_pitch * 2};
-      uint32_t box[2] = {64, 128};
-      encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 2, dims, strides, box);
+      if (o.kind != OP_GEMM) continue;
+      const GemmGeom& g = o.g;
+      if (g.mode == GM_DENSE) {
+        uint64_t dims[2] = {(uint64_t)g.a_pitch, (uint64_t)max_rows};
+        uint64_t strides[1] = {(uint64_t)g.a_pitch * 2};
+        uint32_t box[2] = {64, 128};
+        encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 2, dims, strides, box);
+        continue;
+      }
+      // NHWC input [max_rows][H][W][Cp] viewed as a 4D tensor {C, W, H, N}
+      uint64_t dims[4] = {(uint64_t)g.Cp_in, (uint64_t)g.W, (uint64_t)g.H, (uint64_t)max_rows};
+      uint64_t strides[3] = {(uint64_t)g.Cp_in * 2, (uint64_t)g.W * g.Cp_in * 2, (uint64_t)g.H * g.W * g.Cp_in * 2};
+      if (g.mode == GM_CONV) {
+        // filter-window top-left positions: w = -pad + i*stride, i < OW (same for h)
+        const int lower[2] = {-g.pad, -g.pad};
+        const int upper[2] = {-g.pad + (g.OW - 1) * g.stride - (g.W - 1), -g.pad + (g.OH - 1) * g.stride - (g.H - 1)};
+        const uint32_t estr[4] = {1, (uint32_t)g.stride, (uint32_t)g.stride, 1};
+        encode_im2col(&w->tmA[i], dt, w->buf[o.in_buf], dims, strides, lower, upper, g.cw, 128, estr);
+      } else {
+        uint32_t box[4] = {(uint32_t)g.cw, 1, 1, 128};
+        encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 4, dims, strides, box, g.cw * 2);
+      }
     }
   }
   Workspace* r = w.get();
@@ -516,12 +678,20 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
       src = w->in_stage;
     }
     uint8_t* dst = out_mem == DJINN_MEM_HOST ? (uint8_t*)w->out_stage : (uint8_t*)out + r0 * out_row_bytes;
+    if (profile) {
+      std::lock_guard<std::mutex> lk(mu);
+      prof_recs.push_back({prof_used, (int)ops.size()});
+      for (size_t i = 0; i <= ops.size(); ++i) prof_event();
+    }
+    const size_t pbase = profile ? prof_recs.back().first : 0;
     for (size_t i = 0; i < ops.size(); ++i) {
       const Op& o = ops[i];
       cudaError_t e = cudaSuccess;
+      if (profile) ck(cudaEventRecord(prof_events[pbase + i], st), "profile event");
       switch (o.kind) {
         case OP_PACK:
-          e = launch_pack_input(src, w->buf[0], n, o.in.C, o.in.H, o.in.W, o.out.Cp, dt, st);
+          e = launch_pack_input(src, w->buf[0], n, o.in.C, o.in.H, o.in.W, o.xform, o.xf, o.out.H, o.out.W, o.out.Cp,
+                                dt, st);
           break;
         case OP_GEMM: {
           GemmGeom g = o.g;
@@ -533,7 +703,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
             e = launch_simt_gemm(g, (const float*)A, (const float*)(ar + o.w_off), (const float*)(ar + o.b_off),
                                  (float*)Y, st);
           else
-            e = launch_tc_gemm(g, o.bn, dt, &w->tmA[i], &o.tmB, A, (const float*)(ar + o.b_off), Y, st);
+            e = launch_tc_gemm(g, o.bn, dt, &w->tmA[i], &o.tmB, (const float*)(ar + o.b_off), Y, st);
           break;
         }
         case OP_LRN:
@@ -554,6 +724,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
         throw Error(DJINN_E_CUDA, o.name + ": " + cudaGetErrorString(e));
       }
     }
+    if (profile) ck(cudaEventRecord(prof_events[pbase + ops.size()], st), "profile event");
     if (out_mem == DJINN_MEM_HOST)
       ck(cudaMemcpyAsync((uint8_t*)out + r0 * out_row_bytes, w->out_stage, (size_t)n * out_row_bytes,
                          cudaMemcpyDeviceToHost, st),
@@ -573,7 +744,9 @@ std::string Net::plan_string() const {
       << o.out_buf;
     if (o.kind == OP_GEMM)
       s << " [" << modes[o.g.mode] << " N=" << o.g.N << " Z=" << o.g.Z << " K=" << o.g.K << " Kpad=" << o.g.Kpad
-        << " act=" << o.g.act << " bn=" << o.bn << (o.g.out_f32 ? " fp32-out" : "") << "]";
+        << " act=" << o.g.act << " bn=" << o.bn << " cw=" << o.g.cw << " zf=" << o.g.zf << " KHxKW=" << o.g.KH << "x"
+        << o.g.KW << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << "]";
+    if (o.kind == OP_PACK && o.xform) s << " [" << (o.xform == 1 ? "space-to-depth " : "kx-unroll ") << o.xf << "]";
     s << "\n";
   }
   return s.str();

@@ -58,11 +58,24 @@ struct Op {
   size_t w_off = 0, b_off = 0;  // bytes into the weight arena
   CUtensorMap tmB{};
   int ohw = 1;                  // output pixels per row (conv M = rows * ohw)
+  bool fold_half = false;       // bias += 1/2 * rowsum(W): the producer stores sigma - 1/2
+  // first-layer input transform (PACK op and the conv it feeds): 0 none, 1 space-to-depth
+  // by xf (= conv stride), 2 kx-unroll of a stride-1 kernel of width xf
+  int xform = 0, xf = 1;
+  Shape orig_in;                // the layer's input before the transform
+  int orig_k = 0;               // original kernel size
   // lrn
   int lrn_size = 5;
   float alpha = 0, beta = 0, lrn_k = 1;
   // pool
   int kernel = 0, stride = 1, pad = 0, is_max = 1;
+  // algorithmic work (djinn_op_info): per batch row, and once per launch
+  double flops_row = 0, bytes_row = 0, weight_bytes = 0;
+};
+
+struct ProfRec {  // one timed forward chunk: events[first .. first + n_ops]
+  size_t first;
+  int n_ops;
 };
 
 struct Workspace {
@@ -90,6 +103,13 @@ struct Net {
   std::mutex mu;
   std::map<cudaStream_t, std::unique_ptr<Workspace>> ws;
   bool poisoned = false;
+  // per-op profiling (djinn_profile)
+  bool profile = false;
+  std::vector<cudaEvent_t> prof_events;
+  size_t prof_used = 0;
+  std::vector<ProfRec> prof_recs;
+  cudaEvent_t prof_event();
+  void prof_clear();
   ~Net();
 
   void build(const std::string& desc);                          // parse + plan
@@ -102,6 +122,8 @@ struct Net {
 
 std::atomic<int64_t>& launch_counter();
 void encode_tmap(CUtensorMap* m, int dt, const void* base, int rank, const uint64_t* dims,
-                 const uint64_t* strides_bytes, const uint32_t* box);
+                 const uint64_t* strides_bytes, const uint32_t* box, int swizzle_bytes = 128);
+void encode_im2col(CUtensorMap* m, int dt, const void* base, const uint64_t* dims, const uint64_t* strides_bytes,
+                   const int* lower_wh, const int* upper_wh, int channels, int pixels, const uint32_t* elem_strides);
 
 }  // namespace djinn
