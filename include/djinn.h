@@ -170,6 +170,15 @@ DJINN_API int djinn_profile_read(djinn_net* net, double* ms, int64_t* count, int
 DJINN_API int djinn_op_info(const djinn_net* net, int op, char* name, size_t name_cap, int* kind,
                             double* flops_per_row, double* bytes_per_row, double* weight_bytes);
 
+/* djinn_describe -- parse and plan `desc` for `precision` / `max_rows` WITHOUT touching a
+ * device or weights (host-side planner only): writes the plan text (as djinn_plan_info)
+ * into buf (truncated to cap) and the net's in/out elements per row, parameter and layer
+ * counts (any pointer may be NULL).  Returns the full plan length or a negative error
+ * (DJINN_E_PARSE / _SHAPE / _UNSUPPORTED / _INVAL). */
+DJINN_API int djinn_describe(const char* desc, size_t desc_len, int precision, int64_t max_rows, char* buf,
+                             size_t cap, int64_t* in_elems_per_row, int64_t* out_elems_per_row, int64_t* n_params,
+                             int64_t* n_layers);
+
 /* djinn_last_error -- thread-local message of the last failure ("" if none). */
 DJINN_API const char* djinn_last_error(void);
 

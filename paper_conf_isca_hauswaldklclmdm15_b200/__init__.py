@@ -27,7 +27,7 @@ DJINN_OUT_PROB, DJINN_OUT_ARGMAX, DJINN_OUT_LOGITS = 0, 1, 2
 PRECISION = {"fp32": DJINN_FP32, "bf16": DJINN_BF16, "fp16": DJINN_FP16}
 EXPORTS = ["djinn_load_net", "djinn_forward", "djinn_sync", "djinn_free", "djinn_net_info",
            "djinn_weight_arena", "djinn_plan_info", "djinn_profile", "djinn_profile_read", "djinn_op_info",
-           "djinn_last_error", "djinn_kernel_launches"]
+           "djinn_describe", "djinn_last_error", "djinn_kernel_launches"]
 OP_KINDS = ["pack", "gemm", "lrn", "pool", "softmax"]
 
 
@@ -60,6 +60,7 @@ def lib() -> ctypes.CDLL:
         L.djinn_profile_read.argtypes = [P, ctypes.POINTER(D), ctypes.POINTER(I64), I, I]
         L.djinn_op_info.argtypes = [P, I, ctypes.c_char_p, SZ, ctypes.POINTER(I), ctypes.POINTER(D),
                                     ctypes.POINTER(D), ctypes.POINTER(D)]
+        L.djinn_describe.argtypes = [ctypes.c_char_p, SZ, I, I64, ctypes.c_char_p, SZ] + [ctypes.POINTER(I64)] * 4
         L.djinn_last_error.restype = ctypes.c_char_p
         L.djinn_last_error.argtypes = []
         L.djinn_kernel_launches.restype = I64
@@ -153,6 +154,16 @@ def djinn_op_info(net: int, op: int) -> dict:
                                    ctypes.byref(w)))
     return {"index": op, "n_ops": n, "name": name.value.decode(), "kind": OP_KINDS[kind.value],
             "flops_per_row": f.value, "bytes_per_row": b.value, "weight_bytes": w.value}
+
+
+def djinn_describe(desc: str, precision: int, max_rows: int):
+    """Host-only planning (no device): (plan text, in_elems, out_elems, n_params, n_layers)."""
+    d = desc.encode()
+    v = [ctypes.c_int64() for _ in range(4)]
+    n = _check(lib().djinn_describe(d, len(d), precision, max_rows, None, 0, *[ctypes.byref(x) for x in v]))
+    buf = ctypes.create_string_buffer(n + 1)
+    _check(lib().djinn_describe(d, len(d), precision, max_rows, buf, n + 1, None, None, None, None))
+    return (buf.value.decode(),) + tuple(x.value for x in v)
 
 
 def djinn_kernel_launches() -> int:

@@ -234,6 +234,37 @@ int djinn_op_info(const djinn_net* net, int op, char* name, size_t name_cap, int
   });
 }
 
+int djinn_describe(const char* desc, size_t desc_len, int precision, int64_t max_rows, char* buf, size_t cap,
+                   int64_t* in_elems, int64_t* out_elems, int64_t* n_params, int64_t* n_layers) {
+  return guarded([&]() -> int {
+    if (!desc) return fail(DJINN_E_INVAL, "desc is NULL");
+    if (precision < DJINN_FP32 || precision > DJINN_FP16) return fail(DJINN_E_INVAL, "bad precision");
+    if (max_rows <= 0) return fail(DJINN_E_INVAL, "max_rows must be > 0");
+    djinn::Net n;
+    n.precision = precision;
+    n.dt = precision == DJINN_FP32 ? djinn::DT_F32 : precision == DJINN_BF16 ? djinn::DT_BF16 : djinn::DT_F16;
+    n.max_rows = max_rows;
+    n.build(std::string(desc, desc_len));
+    for (djinn::Op& o : n.ops)
+      if (o.kind == djinn::OP_GEMM && n.dt != djinn::DT_F32) {
+        djinn::GemmGeom g = o.g;
+        g.M = (int)(n.max_rows * o.ohw);
+        o.bn = djinn::tc_pick_bn(g);
+      }
+    if (in_elems) *in_elems = n.in_elems;
+    if (out_elems) *out_elems = n.out_elems;
+    if (n_params) *n_params = n.n_params;
+    if (n_layers) *n_layers = n.n_layers;
+    std::string s = n.plan_string();
+    if (buf && cap) {
+      size_t k = s.size() < cap - 1 ? s.size() : cap - 1;
+      memcpy(buf, s.data(), k);
+      buf[k] = 0;
+    }
+    return (int)s.size();
+  });
+}
+
 const char* djinn_last_error(void) { return g_err.c_str(); }
 
 int64_t djinn_kernel_launches(void) { return djinn::launch_counter(); }

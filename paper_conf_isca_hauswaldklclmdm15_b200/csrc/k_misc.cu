@@ -81,12 +81,54 @@ __global__ void pack32_kernel(const float* __restrict__ x, float* __restrict__ y
   }
 }
 
+// First-layer transforms (mode 1 space-to-depth by f, mode 2 kx-unroll of width f): one thread
+// per OUTPUT pixel writes all Cp channels; the (tap, channel) pair of each output channel is
+// tracked with incremental counters (no integer division per element).
+template <typename T>
+__global__ void pack_xform_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int C, int H, int W,
+                                  int mode, int f, int Ho, int Wo, int Cp) {
+  const int per_row = Ho * Wo;
+  for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
+    const float* src = x + r * C * (int64_t)H * W;
+    for (int pix = blockIdx.x * blockDim.x + threadIdx.x; pix < per_row; pix += gridDim.x * blockDim.x) {
+      const int yo = pix / Wo, xo = pix - (pix / Wo) * Wo;
+      T* dst = y + (r * per_row + pix) * (int64_t)Cp;
+      int a = 0, b = 0, c = 0;  // mode 1: (dy, dx, c); mode 2: (kx, -, c)
+      for (int ch = 0; ch < Cp; ch += 8) {
+        __align__(16) T v[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const int yy = mode == 1 ? yo * f + a : yo;
+          const int xx = mode == 1 ? xo * f + b : xo + a;
+          const bool ok = a < f && yy < H && xx < W;
+          v[j] = cvt<T>(ok ? __ldg(src + ((int64_t)c * H + yy) * W + xx) : 0.f);
+          if (++c == C) {
+            c = 0;
+            if (mode == 1) {
+              if (++b == f) { b = 0; ++a; }
+            } else {
+              ++a;
+            }
+          }
+        }
+        *reinterpret_cast<uint4*>(dst + ch) = *reinterpret_cast<const uint4*>(v);
+      }
+    }
+  }
+}
+
 cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f,
                               int Ho, int Wo, int Cp, int dt, cudaStream_t st) {
   const int T = 256;
   if (dt == DT_F32) {
     int64_t n = rows * (int64_t)H * W * Cp;
     pack32_kernel<<<min(nblocks(n, T), 148 * 32), T, 0, st>>>(x, (float*)y, rows, C, H * W, Cp);
+  } else if (mode != 0) {
+    dim3 g(min(nblocks(Ho * Wo, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
+    if (dt == DT_F16)
+      pack_xform_kernel<__half><<<g, T, 0, st>>>(x, (__half*)y, rows, C, H, W, mode, f, Ho, Wo, Cp);
+    else
+      pack_xform_kernel<__nv_bfloat16><<<g, T, 0, st>>>(x, (__nv_bfloat16*)y, rows, C, H, W, mode, f, Ho, Wo, Cp);
   } else {
     const int per_row = Ho * Wo * (Cp / 8);
     dim3 g(min(nblocks(per_row, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
@@ -102,32 +144,38 @@ cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int 
 // K4: Caffe LRN across channels.  y = x * (k + alpha/size * sum_{window} x^2)^-beta.
 // One thread per (pixel, channel); the channel window is contiguous in NHWC.
 template <typename T>
-__global__ void lrn_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t pixels, int C, int Cp,
-                           int size, float alpha_over_n, float beta, float k) {
+__global__ void lrn_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t pixels, int C, int Cp, int gsz,
+                           int gpitch, int size, float alpha_over_n, float beta, float k) {
   const int half = (size - 1) / 2;
   const int64_t total = pixels * Cp;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
        i += (int64_t)gridDim.x * blockDim.x) {
-    const int c = (int)(i % Cp);
-    if (c >= C) { y[i] = cvt<T>(0.f); continue; }
-    const T* px = x + (i - c);
+    const int p = (int)(i % Cp);  // storage position -> logical channel
+    const int grp = p / gpitch, cin = p - grp * gpitch;
+    const int c = grp * gsz + cin;
+    if (cin >= gsz || c >= C) { y[i] = cvt<T>(0.f); continue; }
+    const T* px = x + (i - p);
     const int lo = max(c - half, 0), hi = min(c + half, C - 1);
     float s = 0.f;
-    for (int cc = lo; cc <= hi; ++cc) { const float v = ld(px + cc); s += v * v; }
-    const float v = ld(px + c);
+    for (int cc = lo; cc <= hi; ++cc) {
+      const float v = ld(px + (cc / gsz) * gpitch + cc % gsz);
+      s += v * v;
+    }
+    const float v = ld(px + p);
     y[i] = cvt<T>(v * powf(k + alpha_over_n * s, -beta));
   }
 }
 
-cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, int size, float alpha,
-                       float beta, float k, int dt, cudaStream_t st) {
+cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, int gsz, int gpitch, int size,
+                       float alpha, float beta, float k, int dt, cudaStream_t st) {
   const int T = 256;
   const int64_t n = pixels * Cp;
   const int g = min(nblocks(n, T), 148 * 32);
   const float an = alpha / size;
-  if (dt == DT_F32) lrn_kernel<float><<<g, T, 0, st>>>((const float*)x, (float*)y, pixels, C, Cp, size, an, beta, k);
-  else if (dt == DT_F16) lrn_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, pixels, C, Cp, size, an, beta, k);
-  else lrn_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, pixels, C, Cp, size, an, beta, k);
+  if (gsz > C) { gsz = C; gpitch = Cp; }
+  if (dt == DT_F32) lrn_kernel<float><<<g, T, 0, st>>>((const float*)x, (float*)y, pixels, C, Cp, gsz, gpitch, size, an, beta, k);
+  else if (dt == DT_F16) lrn_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, pixels, C, Cp, gsz, gpitch, size, an, beta, k);
+  else lrn_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, pixels, C, Cp, gsz, gpitch, size, an, beta, k);
   return cudaGetLastError();
 }
 
@@ -286,10 +334,119 @@ __global__ void softmax_kernel(const float* __restrict__ z, int64_t rows, int N,
   for (int i = threadIdx.x; i < N; i += blockDim.x) o[i] = expf(zr[i] - m) * inv;
 }
 
+// Single pass, values held in registers: one warp per row (N <= 32*VPT).
+template <int VPT>
+__global__ void softmax_warp_kernel(const float* __restrict__ z, int64_t rows, int N, int pitch, float* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  const int64_t r = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5);
+  if (r >= rows) return;
+  const float* zr = z + r * pitch;
+  float v[VPT];
+  float m = -FLT_MAX;
+#pragma unroll
+  for (int j = 0; j < VPT; ++j) {
+    const int i = lane + 32 * j;
+    v[j] = i < N ? zr[i] : -FLT_MAX;
+    m = fmaxf(m, v[j]);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+  float s = 0.f;
+#pragma unroll
+  for (int j = 0; j < VPT; ++j) {
+    v[j] = (lane + 32 * j) < N ? expf(v[j] - m) : 0.f;
+    s += v[j];
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  const float inv = 1.f / s;
+  float* orow = out + r * N;
+#pragma unroll
+  for (int j = 0; j < VPT; ++j) {
+    const int i = lane + 32 * j;
+    if (i < N) orow[i] = v[j] * inv;
+  }
+}
+
+// Single pass for long rows (N <= 256*4*VQ, e.g. the 8000 ASR senones): one CTA of 256 threads
+// per row, float4 loads, exp values kept in registers between the reductions.
+template <int VQ>
+__global__ void softmax_block_kernel(const float* __restrict__ z, int64_t rows, int N, int pitch, float* __restrict__ out) {
+  __shared__ float red[8];
+  const int64_t r = blockIdx.x;
+  const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
+  const float* zr = z + r * pitch;
+  float4 v[VQ];
+  float m = -FLT_MAX;
+#pragma unroll
+  for (int j = 0; j < VQ; ++j) {
+    const int i = 4 * (t + 256 * j);
+    if (i + 3 < N) {
+      v[j] = *reinterpret_cast<const float4*>(zr + i);
+    } else {
+      v[j].x = i < N ? zr[i] : -FLT_MAX;
+      v[j].y = i + 1 < N ? zr[i + 1] : -FLT_MAX;
+      v[j].z = i + 2 < N ? zr[i + 2] : -FLT_MAX;
+      v[j].w = -FLT_MAX;
+    }
+    m = fmaxf(fmaxf(m, fmaxf(v[j].x, v[j].y)), fmaxf(v[j].z, v[j].w));
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+  if (lane == 0) red[wid] = m;
+  __syncthreads();
+  m = red[0];
+#pragma unroll
+  for (int k = 1; k < 8; ++k) m = fmaxf(m, red[k]);
+  __syncthreads();
+  float s = 0.f;
+#pragma unroll
+  for (int j = 0; j < VQ; ++j) {
+    const int i = 4 * (t + 256 * j);
+    v[j].x = i < N ? expf(v[j].x - m) : 0.f;
+    v[j].y = i + 1 < N ? expf(v[j].y - m) : 0.f;
+    v[j].z = i + 2 < N ? expf(v[j].z - m) : 0.f;
+    v[j].w = i + 3 < N ? expf(v[j].w - m) : 0.f;
+    s += (v[j].x + v[j].y) + (v[j].z + v[j].w);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if (lane == 0) red[wid] = s;
+  __syncthreads();
+  s = 0.f;
+#pragma unroll
+  for (int k = 0; k < 8; ++k) s += red[k];
+  const float inv = 1.f / s;
+  float* orow = out + r * N;
+  const bool vec = (N % 4) == 0;
+#pragma unroll
+  for (int j = 0; j < VQ; ++j) {
+    const int i = 4 * (t + 256 * j);
+    float4 p = make_float4(v[j].x * inv, v[j].y * inv, v[j].z * inv, v[j].w * inv);
+    if (vec && i + 3 < N) {
+      *reinterpret_cast<float4*>(orow + i) = p;
+    } else {
+      if (i < N) orow[i] = p.x;
+      if (i + 1 < N) orow[i + 1] = p.y;
+      if (i + 2 < N) orow[i + 2] = p.z;
+      if (i + 3 < N) orow[i + 3] = p.w;
+    }
+  }
+}
+
 cudaError_t launch_softmax(const float* logits, int64_t rows, int N, int pitch, void* out, int mode,
                            cudaStream_t st) {
   if (rows <= 0) return cudaSuccess;
-  softmax_kernel<<<(unsigned)rows, 256, 0, st>>>(logits, rows, N, pitch, out, mode);
+  if (mode == 0 && N <= 256 && pitch % 4 == 0) {
+    const int rpb = 8;  // rows (warps) per 256-thread block
+    const unsigned g = (unsigned)((rows + rpb - 1) / rpb);
+    if (N <= 64) softmax_warp_kernel<2><<<g, 256, 0, st>>>(logits, rows, N, pitch, (float*)out);
+    else softmax_warp_kernel<8><<<g, 256, 0, st>>>(logits, rows, N, pitch, (float*)out);
+  } else if (mode == 0 && N <= 8192 && pitch % 4 == 0) {
+    softmax_block_kernel<8><<<(unsigned)rows, 256, 0, st>>>(logits, rows, N, pitch, (float*)out);
+  } else {
+    softmax_kernel<<<(unsigned)rows, 256, 0, st>>>(logits, rows, N, pitch, out, mode);
+  }
   return cudaGetLastError();
 }
 

@@ -12,8 +12,10 @@
 //   * persistent CTAs (grid <= #SMs), static tile striding; a tile = (m block of 128 rows,
 //     n block of BN columns, a group of zf z-slices accumulated side by side in TMEM)
 //   * warp 8: TMA producer.  A arrives in chunks of cw channels (one TMA box each):
-//       conv  -> im2col-mode TMA (the hardware walks 128 output pixels, applies the
-//                filter offset (kx,ky), zero-fills the padding)
+//       conv  -> tiled 4D TMA box {cw, bx, by, bn}: the input pixels under tap (kx,ky) of
+//                a bx x by x bn block of output pixels (the M tile); out-of-bounds
+//                coordinates (the zero padding) are zero-filled by the TMA unit.  (im2col-
+//                mode TMA was measured at ~16 B/cycle/SM on B200, tiled boxes stream >90.)
 //       LC    -> tiled 4D TMA box {cw, 1, 1, 128 images} at the tap's input pixel
 //       dense -> tiled 2D TMA box {64, 128 rows}
 //     B arrives as a 3D tiled box {64, BN, 1}, SWIZZLE_128B.
@@ -158,6 +160,48 @@ __device__ __forceinline__ float act_fast(float v, int act) {
   }
 }
 
+// Bias + activation on a 16-vector: the switch is resolved once per vector, the loops are
+// branch-free (the per-element runtime switch cost ~17% of issue slots in branch resolution).
+__device__ __forceinline__ void bias_act16(float (&v)[16], const uint32_t (&r)[16], const float (&b)[16], int act) {
+#pragma unroll
+  for (int j = 0; j < 16; ++j) v[j] = __uint_as_float(r[j]) + b[j];
+  switch (act) {
+    case ACT_RELU:
+#pragma unroll
+      for (int j = 0; j < 16; ++j) v[j] = fmaxf(v[j], 0.f);
+      break;
+    case ACT_SIGMOID:
+#pragma unroll
+      for (int j = 0; j < 16; ++j) v[j] = __fdividef(1.f, 1.f + __expf(-v[j]));
+      break;
+    case ACT_SIGMOID_C:
+#pragma unroll
+      for (int j = 0; j < 16; ++j) v[j] = __fdividef(1.f, 1.f + __expf(-v[j])) - 0.5f;
+      break;
+    case ACT_TANH:
+#pragma unroll
+      for (int j = 0; j < 16; ++j) v[j] = tanh_approx(v[j]);
+      break;
+    case ACT_HARDTANH:
+#pragma unroll
+      for (int j = 0; j < 16; ++j) v[j] = fminf(fmaxf(v[j], -1.f), 1.f);
+      break;
+    default:
+      break;
+  }
+}
+
+// 16 bias values starting at n (zeros at n >= nvalid); vector loads when the chunk is full.
+__device__ __forceinline__ void load_bias16(float (&b)[16], const float* __restrict__ bz, int n, int nvalid) {
+  if (n + 16 <= nvalid) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) *reinterpret_cast<float4*>(b + 4 * q) = __ldg(reinterpret_cast<const float4*>(bz + n) + q);
+  } else {
+#pragma unroll
+    for (int j = 0; j < 16; ++j) b[j] = n + j < nvalid ? __ldg(bz + n + j) : 0.f;
+  }
+}
+
 template <bool BF16>
 __device__ __forceinline__ uint32_t pack2(float a, float b) {
   if (BF16) {
@@ -190,16 +234,46 @@ __device__ __forceinline__ void store16(const GemmGeom& g, void* Y, int64_t off,
   }
 }
 
+// Store a 16-channel chunk whose first LOGICAL channel is cglob, honouring the output's
+// grouped layout (channel c at (c/gsz)*gpitch + c%gsz); the last chunk of a group also
+// zero-fills the group's pad channels so that pads never hold stale data.
+template <bool BF16>
+__device__ __forceinline__ void store_chunk(const GemmGeom& g, void* Y, int64_t pixbase, int cglob,
+                                            const float (&v)[16], int nvalid8) {
+  const int gsz = g.out_gsz;
+  const int grp = cglob / gsz, cin = cglob - grp * gsz;
+  const int64_t gbase = pixbase + (int64_t)grp * g.out_gpitch;
+  store16<BF16>(g, Y, gbase + cin, v, nvalid8);
+  if (g.out_gpitch > gsz && cin + 16 >= gsz && !g.out_f32) {
+    uint16_t* yp = reinterpret_cast<uint16_t*>(Y) + gbase + gsz;
+    for (int e = 0; e < g.out_gpitch - gsz; e += 8) *reinterpret_cast<uint4*>(yp + e) = make_uint4(0, 0, 0, 0);
+  }
+}
+
 struct TileCoord {
-  int m0, n0, z0;
+  int m0, n0, z0;      // m0: first GEMM row (dense / LC); n0: column block; z0: z group
+  int x0, y0, i0;      // conv: first output pixel (x, y) and image of the block
 };
-__device__ __forceinline__ TileCoord tile_coord(int t, int mt, int nt) {
+__device__ __forceinline__ TileCoord tile_coord(const GemmGeom& g, int t, int mt, int nt) {
   TileCoord c;
-  c.m0 = (t % mt) * BM;
+  const int tm = t % mt;
+  c.m0 = tm * BM;
   t /= mt;
   c.n0 = (t % nt);
   c.z0 = t / nt;
+  c.x0 = c.y0 = c.i0 = 0;
+  if (g.mode == GM_CONV && g.a_tiled) {
+    const int nbx = (g.OW + g.bx - 1) / g.bx, nby = (g.OH + g.by - 1) / g.by;
+    c.x0 = (tm % nbx) * g.bx;
+    c.y0 = ((tm / nbx) % nby) * g.by;
+    c.i0 = (tm / (nbx * nby)) * g.bn;
+  }
   return c;
+}
+__device__ __forceinline__ int num_m_tiles(const GemmGeom& g) {
+  if (g.mode == GM_CONV && g.a_tiled)
+    return ((g.OW + g.bx - 1) / g.bx) * ((g.OH + g.by - 1) / g.by) * ((g.Nimg + g.bn - 1) / g.bn);
+  return (g.M + BM - 1) / BM;
 }
 
 // ---------------------------------------------------------------- the kernel
@@ -220,7 +294,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int num_kb = g.Kpad / BK;
-  const int mt = (g.M + BM - 1) / BM, nt = (g.N + BN - 1) / BN, zt = g.Z / g.zf;
+  const int mt = num_m_tiles(g), nt = (g.N + BN - 1) / BN, zt = g.Z / g.zf;
   const int tiles = mt * nt * zt;
   const int slot_cols = g.zf * BN;
   const int nslots = 2 * slot_cols <= 512 ? 2 : 1;
@@ -258,15 +332,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       const int nchunks_k = g.K / cw;  // valid chunks along K
       int it = 0;
       for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
-        const TileCoord tc = tile_coord(t, mt, nt);
-        // first output pixel of the tile (conv): top-left of its filter window in input coords
-        int img = 0, wy = 0, wx = 0;
-        if (g.mode == GM_CONV) {
+        const TileCoord tc = tile_coord(g, t, mt, nt);
+        // conv: top-left input pixel of the filter window of the tile's first output pixel
+        int wx = tc.x0 * g.stride - g.pad, wy = tc.y0 * g.stride - g.pad, img = tc.i0;
+        if (g.mode == GM_CONV && !g.a_tiled) {
           img = tc.m0 / (g.OH * g.OW);
           const int rem = tc.m0 - img * g.OH * g.OW;
-          const int oy = rem / g.OW, ox = rem - (rem / g.OW) * g.OW;
+          const int oy = rem / g.OW;
           wy = oy * g.stride - g.pad;
-          wx = ox * g.stride - g.pad;
+          wx = (rem - oy * g.OW) * g.stride - g.pad;
         }
         for (int zi = 0; zi < g.zf; ++zi) {
           const int z = tc.z0 * g.zf + zi;
@@ -293,7 +367,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 }
                 const uint32_t dst = a_dst + j * cbytes;
                 if (g.mode == GM_CONV) {
-                  tma_im2col_4d(dst, &tmA, fb, c, wx, wy, img, (uint16_t)kx, (uint16_t)ky);
+                  if (g.a_tiled) tma_4d(dst, &tmA, fb, c, wx + kx, wy + ky, img);
+                  else tma_im2col_4d(dst, &tmA, fb, c, wx, wy, img, (uint16_t)kx, (uint16_t)ky);
                 } else {  // LC: rows are images at the fixed output location z
                   const int oy = z / g.OW, ox = z - (z / g.OW) * g.OW;
                   tma_4d(dst, &tmA, fb, c, ox * g.stride + kx, oy * g.stride + ky, tc.m0);
@@ -344,13 +419,22 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     int lt = 0;
     const uint32_t lane_base = (uint32_t)(quarter * 32) << 16;
     for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++lt) {
-      const TileCoord tc = tile_coord(t, mt, nt);
+      const TileCoord tc = tile_coord(g, t, mt, nt);
       const int slot = nslots == 2 ? (lt & 1) : 0;
       const uint32_t use = nslots == 2 ? (uint32_t)(lt >> 1) : (uint32_t)lt;
+      const int r = quarter * 32 + lane;
+      int m;       // output pixel (conv) / GEMM row (dense, LC)
+      bool mok;
+      if (g.mode == GM_CONV && g.a_tiled) {
+        const int ox = tc.x0 + r % g.bx, oy = tc.y0 + (r / g.bx) % g.by, im = tc.i0 + r / (g.bx * g.by);
+        mok = ox < g.OW && oy < g.OH && im < g.Nimg;
+        m = (im * g.OH + oy) * g.OW + ox;
+      } else {
+        m = tc.m0 + r;
+        mok = m < g.M;
+      }
       mbar_wait(tfull0 + 8 * slot, use & 1);
       tc_fence_after();
-      const int m = tc.m0 + quarter * 32 + lane;
-      const bool mok = m < g.M;
       const uint32_t tbase = tmem + lane_base + (uint32_t)(slot * slot_cols);
       if (g.epi_lrn) {
         // Channels c = zi * N + n (N == BN when zf > 1) live in columns zi*BN + n.  The LRN
@@ -360,18 +444,21 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         const int nch = (Ctot + 15) / 16, per = (nch + 1) / 2;
         const int ib = half * per, ie = min(nch, ib + per);
         const int64_t obase = (int64_t)m * g.out_pitch;
+        const float ka = g.lrn_alpha_over_n, kk = g.lrn_k, nb = -g.lrn_beta;
         float cur[16], nxt[16];
         float pm2 = 0.f, pm1 = 0.f;
         auto load_chunk = [&](int i, float (&v)[16]) {
           const int c0 = i * 16;
           const int zi = c0 / N, n0 = c0 - zi * N;
-          uint32_t r[16];
-          tmem_ld16(tbase + (uint32_t)(zi * BN + n0), r);
+          float b[16];
+          load_bias16(b, bias, c0, Ctot);
+          uint32_t rr[16];
+          tmem_ld16(tbase + (uint32_t)(zi * BN + n0), rr);
           tmem_wait_ld();
+          bias_act16(v, rr, b, g.act);
+          if (c0 + 16 > Ctot) {
 #pragma unroll
-          for (int j = 0; j < 16; ++j) {
-            const int c = c0 + j;
-            v[j] = c < Ctot ? act_fast(__uint_as_float(r[j]) + __ldg(bias + c), g.act) : 0.f;
+            for (int j = 0; j < 16; ++j) v[j] = c0 + j < Ctot ? v[j] : 0.f;
           }
         };
         if (ib < ie) {
@@ -399,15 +486,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           float o[16];
 #pragma unroll
           for (int j = 0; j < 16; ++j) {
-            const float s5 = sq[j] + sq[j + 1] + sq[j + 2] + sq[j + 3] + sq[j + 4];  // window c-2 .. c+2
-            o[j] = cur[j] * __powf(g.lrn_k + g.lrn_alpha_over_n * s5, -g.lrn_beta);
+            const float s5 = (sq[j] + sq[j + 1]) + (sq[j + 2] + sq[j + 3]) + sq[j + 4];  // window c-2 .. c+2
+            o[j] = cur[j] * exp2f(nb * __log2f(fmaf(ka, s5, kk)));
           }
           pm2 = sq[16];
           pm1 = sq[17];
           if (mok) {
             const int c0 = i * 16;
             const int nvalid8 = min(2, (g.write_cols - c0 + 7) / 8);
-            if (nvalid8 > 0) store16<BF16>(g, Y, obase + c0, o, nvalid8);
+            if (nvalid8 > 0) store_chunk<BF16>(g, Y, obase, c0, o, nvalid8);
           }
 #pragma unroll
           for (int j = 0; j < 16; ++j) cur[j] = nxt[j];
@@ -425,32 +512,32 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           const int nb0 = tc.n0 * BN;
 #pragma unroll 1
           for (int c = cbeg; c < cbeg + cols; c += 32) {
-            const int two = (c + 16 < cbeg + cols) ? 2 : 1;
-            uint32_t r[2][16];
-            tmem_ld16(tbase + (uint32_t)(zi * BN + c), r[0]);
-            if (two == 2) tmem_ld16(tbase + (uint32_t)(zi * BN + c + 16), r[1]);
+            const bool two = c + 16 < cbeg + cols;
+            float b0[16], b1[16];
+            load_bias16(b0, bz, nb0 + c, g.N);  // bias loads in flight during the TMEM load
+            if (two) load_bias16(b1, bz, nb0 + c + 16, g.N);
+            uint32_t r0[16], r1[16];
+            tmem_ld16(tbase + (uint32_t)(zi * BN + c), r0);
+            if (two) tmem_ld16(tbase + (uint32_t)(zi * BN + c + 16), r1);
             tmem_wait_ld();
+            const int nb = nb0 + c;
+            if (mok && nb < g.write_cols) {
+              float v[16];
+              bias_act16(v, r0, b0, g.act);
+              if (nb + 16 > g.N) {
 #pragma unroll
-            for (int hh = 0; hh < 2; ++hh) {
-              if (hh >= two) break;
-              const int nb = nb0 + c + 16 * hh;
-              if (mok && nb < g.write_cols) {
-                float v[16];
-                if (nb + 16 <= g.N) {
-                  float b[16];
-#pragma unroll
-                  for (int q = 0; q < 4; ++q) *reinterpret_cast<float4*>(b + 4 * q) = __ldg(reinterpret_cast<const float4*>(bz + nb) + q);
-#pragma unroll
-                  for (int j = 0; j < 16; ++j) v[j] = act_fast(__uint_as_float(r[hh][j]) + b[j], g.act);
-                } else {
-#pragma unroll
-                  for (int j = 0; j < 16; ++j) {
-                    const int n = nb + j;
-                    v[j] = n < g.N ? act_fast(__uint_as_float(r[hh][j]) + __ldg(bz + n), g.act) : 0.f;
-                  }
-                }
-                store16<BF16>(g, Y, pix * g.out_pitch + goff + nb, v, min(2, (g.write_cols - nb + 7) / 8));
+                for (int j = 0; j < 16; ++j) v[j] = nb + j < g.N ? v[j] : 0.f;
               }
+              store_chunk<BF16>(g, Y, pix * g.out_pitch, goff + nb, v, min(2, (g.write_cols - nb + 7) / 8));
+            }
+            if (two && mok && nb + 16 < g.write_cols) {
+              float v[16];
+              bias_act16(v, r1, b1, g.act);
+              if (nb + 32 > g.N) {
+#pragma unroll
+                for (int j = 0; j < 16; ++j) v[j] = nb + 16 + j < g.N ? v[j] : 0.f;
+              }
+              store_chunk<BF16>(g, Y, pix * g.out_pitch, goff + nb + 16, v, min(2, (g.write_cols - nb - 16 + 7) / 8));
             }
           }
         }
@@ -481,7 +568,11 @@ cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtenso
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  const int64_t tiles = (int64_t)((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN) * (g.Z / g.zf);
+  const int64_t mtiles = (g.mode == GM_CONV && g.a_tiled)
+                             ? (int64_t)((g.OW + g.bx - 1) / g.bx) * ((g.OH + g.by - 1) / g.by) *
+                                                  ((g.Nimg + g.bn - 1) / g.bn)
+                                            : (g.M + BM - 1) / BM;
+  const int64_t tiles = mtiles * ((g.N + BN - 1) / BN) * (g.Z / g.zf);
   const int grid = (int)(tiles < tc_num_sms() ? tiles : tc_num_sms());
   kern<<<grid, NUM_THREADS, C::SMEM, st>>>(*tmA, *tmB, g, bias, Y);
   return cudaGetLastError();

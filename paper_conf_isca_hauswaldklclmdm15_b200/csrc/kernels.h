@@ -41,8 +41,13 @@ struct GemmGeom {
   int bias_zstride;   // bias elements between z (LC: Co per location; conv: Cog)
   int act;
   int out_f32;        // 1: fp32 output (logits), 0: same 16-bit type as input
+  int out_gsz, out_gpitch;  // output channel c stored at (c/out_gsz)*out_gpitch + c%out_gsz
   // tensor-core path only
   int cw;             // A chunk width in elements (16 / 32 / 64): one TMA box per chunk
+  int Nimg;           // conv: images in the batch
+  int a_tiled;        // conv: 0 = im2col-mode TMA over linear output pixels (default), 1 = tiled
+                      //       4D boxes over bx x by x bn pixel blocks (DJINN_CONV_A=tiled)
+  int bx, by, bn;     // conv: output-pixel block of one M tile (bx*by*bn == 128), x fastest
   int zf;             // z values fused per CTA (groups computed by one CTA; TMEM columns zf*BN)
   int epi_lrn;        // 1: Caffe LRN across the zf*N channels of a pixel in the epilogue
   int lrn_size;
@@ -63,7 +68,8 @@ cudaError_t launch_simt_gemm(const GemmGeom& g, const float* A, const float* B, 
 
 // --- tcgen05 tensor-core implicit GEMM (K1/K2/K3) -----------------------------------------
 // tmB: 3D tensor map over B [Z][N][Kpad] (16-bit, SWIZZLE_128B, box {64, BN, 1}).
-// tmA: conv -> 4D im2col map over the NHWC input (channelsPerPixel = cw, 128 pixels);
+// tmA: conv -> 4D tiled map over the NHWC input, box {cw, bx*s, by*s, bn}, element strides
+//              {1, s, s, 1}: the tap (kx,ky) of a bx x by x bn block of output pixels;
 //      LC   -> 4D tiled map over the NHWC input, box {cw, 1, 1, 128};
 //      dense-> 2D tiled map over [rows][a_pitch], box {64, 128}.
 // Swizzle of A boxes: cw*2 bytes (32B / 64B / 128B).
@@ -73,8 +79,9 @@ cudaError_t launch_tc_gemm(const GemmGeom& g, int bn, int dt, const CUtensorMap*
                            const CUtensorMap* tmB, const float* bias, void* Y, cudaStream_t st);
 
 // --- LRN across channels (K4), NHWC ----------------------------------------------------------
-cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, int size, float alpha,
-                       float beta, float k, int dt, cudaStream_t st);
+// Channel c of a pixel is stored at (c/gsz)*gpitch + c%gsz (grouped layouts); pads -> 0.
+cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, int gsz, int gpitch, int size,
+                       float alpha, float beta, float k, int dt, cudaStream_t st);
 
 // --- pooling (K5), NHWC, Caffe ceil geometry ------------------------------------------------
 cudaError_t launch_pool(const void* x, void* y, int64_t rows, int C, int Cp, int H, int W, int OH,

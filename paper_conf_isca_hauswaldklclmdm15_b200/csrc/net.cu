@@ -147,10 +147,10 @@ static CUtensorMapSwizzle swizzle_for(int row_bytes) {
 }
 
 void encode_tmap(CUtensorMap* m, int dt, const void* base, int rank, const uint64_t* dims, const uint64_t* strides_bytes,
-                 const uint32_t* box, int swizzle_bytes) {
+                 const uint32_t* box, int swizzle_bytes, const uint32_t* elem_strides) {
   cuuint64_t d[5], s[4];
   cuuint32_t b[5], es[5];
-  for (int i = 0; i < rank; ++i) { d[i] = dims[i]; b[i] = box[i]; es[i] = 1; }
+  for (int i = 0; i < rank; ++i) { d[i] = dims[i]; b[i] = box[i]; es[i] = elem_strides ? elem_strides[i] : 1; }
   for (int i = 0; i + 1 < rank; ++i) s[i] = strides_bytes[i];
   const CUtensorMapDataType ty = dt == DT_F16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16;
   CUresult r = encode_fn()(m, ty, (cuuint32_t)rank, const_cast<void*>(base), d, s, b, es,
@@ -253,14 +253,43 @@ void Net::build(const std::string& desc) {
   const bool f16 = dt != DT_F32;
   // 16-bit activations: channel pitch a multiple of 16 so every conv's K splits into TMA
   // chunks of 16/32/64 channels (one swizzle atom row of 32/64/128 B)
-  auto pitch = [&](int c) { return f16 ? rup(c, 16) : c; };
+  // Layout of a tensor with C channels, decided by its next channel-consuming layer (skipping
+  // activations, LRN, pooling, dropout, which keep the layout): a conv with G groups wants
+  // each group at a pitch of 16/32/64 (<= 64 channels) or a multiple of 64, i.e. one TMA row
+  // of 32/64/128 B per tap and chunk.  fp32 path: dense channels.
+  auto tap_pitch = [](int c) { return c <= 16 ? 16 : c <= 32 ? 32 : rup(c, 64); };
+  auto layout_for = [&](size_t from, Shape sh) {
+    sh.Cp = sh.C;
+    sh.gsz = sh.gpitch = 1 << 30;
+    if (!f16) return sh;
+    sh.Cp = rup(sh.C, 16);
+    for (size_t j = from; j < layers.size(); ++j) {
+      const LayerSpec& L = layers[j];
+      if (L.type == "Convolution" && L.group > 1 && sh.C % L.group == 0) {
+        const int cg = sh.C / L.group;
+        if (cg % 16 == 0) {
+          sh.gsz = cg;
+          sh.gpitch = tap_pitch(cg);
+          sh.Cp = L.group * sh.gpitch;
+        }
+        return sh;
+      }
+      if (L.type == "Convolution" || L.type == "LocallyConnected") {
+        sh.Cp = tap_pitch(sh.C);
+        return sh;
+      }
+      if (L.type == "InnerProduct" || L.type == "Softmax") return sh;
+    }
+    return sh;
+  };
   const std::vector<int>& d = layers[0].dims;
   Shape cur;
   if (d.size() == 1) { cur.C = d[0]; }
   else if (d.size() == 3) { cur.C = d[0]; cur.H = d[1]; cur.W = d[2]; }
   else throw Error(DJINN_E_SHAPE, "Input must have 1 or 3 dims");
   if (cur.C <= 0 || cur.H <= 0 || cur.W <= 0) throw Error(DJINN_E_SHAPE, "bad Input dims");
-  cur.Cp = pitch(cur.C);
+  cur = layout_for(1, cur);
+  if (cur.gsz < cur.C) throw Error(DJINN_E_UNSUPPORTED, "grouped first convolution on a 16-bit path");
   in_elems = (int64_t)cur.C * cur.H * cur.W;
 
   Op pk;
@@ -379,8 +408,11 @@ void Net::build(const std::string& desc) {
       g.KH = g.KW = L.kernel;
       g.stride = L.stride;
       g.pad = pad;
-      g.Cgp = (grp == 1) ? cur.Cp : Cg;
-      g.cin_goff = Cg;
+      if (f16 && grp > 1 && cur.gsz != Cg)
+        throw Error(DJINN_E_UNSUPPORTED, L.name + ": input channel layout does not match the grouping");
+      const bool grouped_layout = cur.gsz < cur.C;
+      g.Cgp = (grp == 1) ? cur.Cp : (grouped_layout ? cur.gpitch : Cg);
+      g.cin_goff = grouped_layout ? cur.gpitch : Cg;
       // First layer with few channels on the tensor-core path: repack the input so that K
       // is dense.  Strided kernels: space-to-depth by the stride (k x k / s  ->  ceil(k/s)^2
       // taps over s*s*C channels, stride 1).  Stride 1: unroll kx into channels (k x k -> k x 1).
@@ -392,7 +424,8 @@ void Net::build(const std::string& desc) {
           if (Hs - ks + 1 >= OH && Ws - ks + 1 >= OW) {
             pk.xform = o.xform = 1;
             pk.xf = o.xf = f;
-            pk.out.C = f * f * cur.C; pk.out.H = Hs; pk.out.W = Ws; pk.out.Cp = pitch(f * f * cur.C);
+            pk.out = Shape();
+            pk.out.C = f * f * cur.C; pk.out.H = Hs; pk.out.W = Ws; pk.out.Cp = tap_pitch(f * f * cur.C);
             g.H = Hs; g.W = Ws; g.Cp_in = g.Cgp = pk.out.Cp;
             g.KH = g.KW = ks;
             g.stride = 1;
@@ -400,21 +433,42 @@ void Net::build(const std::string& desc) {
         } else {
           pk.xform = o.xform = 2;
           pk.xf = o.xf = k;
-          pk.out.C = k * cur.C; pk.out.H = cur.H; pk.out.W = cur.W - k + 1; pk.out.Cp = pitch(k * cur.C);
+          pk.out = Shape();
+          pk.out.C = k * cur.C; pk.out.H = cur.H; pk.out.W = cur.W - k + 1; pk.out.Cp = tap_pitch(k * cur.C);
           g.H = cur.H; g.W = cur.W - k + 1; g.Cp_in = g.Cgp = pk.out.Cp;
           g.KH = k; g.KW = 1;
         }
         if (pk.xform) { o.in = pk.out; }
       }
       g.K = g.KH * g.KW * g.Cgp;
-      o.out.C = L.num_output; o.out.H = OH; o.out.W = OW; o.out.Cp = pitch(L.num_output);
+      o.out = Shape();
+      o.out.C = L.num_output; o.out.H = OH; o.out.W = OW;
+      o.out = layout_for(i + 1, o.out);
       g.out_pitch = o.out.Cp;
       g.cout_goff = Cog;
       g.write_cols = grp == 1 ? o.out.Cp : Cog;
       g.bias_zstride = Cog;
       o.ohw = lc ? 1 : OH * OW;
       g.zf = 1;
-      g.cw = g.Cgp % 64 == 0 ? 64 : (g.Cgp % 32 == 0 ? 32 : 16);
+      g.cw = g.Cgp >= 64 ? 64 : g.Cgp;
+      // M tile = a bx x by x bn block of output pixels (x fastest, product 128): the one with
+      // the least padding waste for this layer's OW x OH x batch.
+      const char* amode = getenv("DJINN_CONV_A");
+      g.a_tiled = (!lc && amode && strcmp(amode, "tiled") == 0) ? 1 : 0;
+      if (!lc) {
+        double best = 1e30;
+        for (int bx = 1; bx <= 128; bx *= 2)
+          for (int by = 1; bx * by <= 128; by *= 2) {
+            const int bn = 128 / (bx * by);
+            if (bx * g.stride > 256 || by * g.stride > 256) continue;
+            // padded pixels x (1 + 4/bx): a TMA box streams runs of bx contiguous pixels, short
+            // runs cost extra per row (B200 measurement)
+            const double cost = (double)rup(OW, bx) * rup(OH, by) * rup((int)max_rows, bn) * (1.0 + 4.0 / bx);
+            if (cost < best - 1e-9 || (cost < best + 1e-9 && bx > g.bx)) { best = cost; g.bx = bx; g.by = by; g.bn = bn; }
+          }
+      }
+      if (f16 && (g.Cgp % 16 || (g.Cgp > 64 && g.Cgp % 64) || (g.Cgp < 64 && g.Cgp != 16 && g.Cgp != 32)))
+        throw Error(DJINN_E_SHAPE, L.name + ": internal: input channel pitch not TMA-chunkable");
       // Caffe LRN right after (the activation of) this conv: fuse it into the epilogue when one
       // tile holds every channel of a pixel (all groups side by side in TMEM).
       if (f16 && !lc && i + 1 < layers.size() && layers[i + 1].type == "LRN" && layers[i + 1].lrn_size == 5) {
@@ -444,8 +498,10 @@ void Net::build(const std::string& desc) {
       g.a_pitch = g.K;
       g.zf = 1;
       g.cw = 64;
+      o.out = Shape();
       o.out.C = L.num_output; o.out.H = 1; o.out.W = 1;
-      o.out.Cp = last ? rup(L.num_output, 8) : pitch(L.num_output);
+      o.out = layout_for(i + 1, o.out);
+      if (last) o.out.Cp = rup(L.num_output, 8);
       g.out_pitch = o.out.Cp;
       g.write_cols = o.out.Cp;
       g.bias_zstride = 0;
@@ -453,6 +509,14 @@ void Net::build(const std::string& desc) {
       bcount = L.num_output;
     }
     if (last && g.mode != GM_DENSE) throw Error(DJINN_E_UNSUPPORTED, "the layer before Softmax must be InnerProduct");
+    g.out_pitch = o.out.Cp;
+    g.out_gsz = o.out.gsz;
+    g.out_gpitch = o.out.gpitch;
+    if (o.out.gsz < o.out.C) {  // grouped output layout: write real channels, pads zeroed per group
+      if (o.out.gsz % 16 || (g.mode == GM_CONV && g.Z > 1 && !g.epi_lrn && g.N % 16))
+        throw Error(DJINN_E_UNSUPPORTED, L.name + ": output channel groups must be multiples of 16");
+      g.write_cols = (g.mode == GM_CONV && g.Z > 1 && !g.epi_lrn) ? g.N : o.out.C;
+    }
     g.Kpad = f16 ? rup(g.K, 64) : g.K;
     g.out_f32 = last ? 1 : 0;
     o.out_buf = last ? 2 : 1 - curbuf;
@@ -582,7 +646,7 @@ void Net::load_weights(const float* w, size_t n, int mem) {
         for (int c = 0; c < C; ++c)
           for (int h = 0; h < H; ++h)
             for (int x = 0; x < W; ++x)
-              put(0, nn, ((int64_t)h * W + x) * Cp + c, w[off++]);
+              put(0, nn, ((int64_t)h * W + x) * Cp + o.in.pos(c), w[off++]);
       for (int nn = 0; nn < g.N; ++nn) bdst[nn] = (float)(w[off++] + (o.fold_half ? 0.5 * rowsum[nn] : 0.0));
     }
   }
@@ -643,7 +707,11 @@ Workspace* Net::workspace(cudaStream_t st) {
       // NHWC input [max_rows][H][W][Cp] viewed as a 4D tensor {C, W, H, N}
       uint64_t dims[4] = {(uint64_t)g.Cp_in, (uint64_t)g.W, (uint64_t)g.H, (uint64_t)max_rows};
       uint64_t strides[3] = {(uint64_t)g.Cp_in * 2, (uint64_t)g.W * g.Cp_in * 2, (uint64_t)g.H * g.W * g.Cp_in * 2};
-      if (g.mode == GM_CONV) {
+      if (g.mode == GM_CONV && g.a_tiled) {
+        uint32_t box[4] = {(uint32_t)g.cw, (uint32_t)(g.bx * g.stride), (uint32_t)(g.by * g.stride), (uint32_t)g.bn};
+        const uint32_t estr[4] = {1, (uint32_t)g.stride, (uint32_t)g.stride, 1};
+        encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 4, dims, strides, box, g.cw * 2, estr);
+      } else if (g.mode == GM_CONV) {
         // filter-window top-left positions: w = -pad + i*stride, i < OW (same for h)
         const int lower[2] = {-g.pad, -g.pad};
         const int upper[2] = {-g.pad + (g.OW - 1) * g.stride - (g.W - 1), -g.pad + (g.OH - 1) * g.stride - (g.H - 1)};
@@ -696,6 +764,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
         case OP_GEMM: {
           GemmGeom g = o.g;
           g.M = (int)(n * o.ohw);
+          g.Nimg = (int)n;
           const void* A = w->buf[o.in_buf];
           void* Y = w->buf[o.out_buf];
           const uint8_t* ar = (const uint8_t*)arena;
@@ -707,7 +776,8 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           break;
         }
         case OP_LRN:
-          e = launch_lrn(w->buf[o.in_buf], w->buf[o.out_buf], n * o.in.H * o.in.W, o.in.C, o.in.Cp, o.lrn_size,
+          e = launch_lrn(w->buf[o.in_buf], w->buf[o.out_buf], n * o.in.H * o.in.W, o.in.C, o.in.Cp, o.in.gsz,
+                         o.in.gpitch, o.lrn_size,
                          o.alpha, o.beta, o.lrn_k, dt, st);
           break;
         case OP_POOL:
@@ -745,7 +815,9 @@ std::string Net::plan_string() const {
     if (o.kind == OP_GEMM)
       s << " [" << modes[o.g.mode] << " N=" << o.g.N << " Z=" << o.g.Z << " K=" << o.g.K << " Kpad=" << o.g.Kpad
         << " act=" << o.g.act << " bn=" << o.bn << " cw=" << o.g.cw << " zf=" << o.g.zf << " KHxKW=" << o.g.KH << "x"
-        << o.g.KW << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << "]";
+        << o.g.KW << (o.g.mode == GM_CONV && o.g.a_tiled ? " block=" + std::to_string(o.g.bx) + "x" + std::to_string(o.g.by) + "x" +
+                                                  std::to_string(o.g.bn) : std::string())
+        << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << "]";
     if (o.kind == OP_PACK && o.xform) s << " [" << (o.xform == 1 ? "space-to-depth " : "kx-unroll ") << o.xf << "]";
     s << "\n";
   }

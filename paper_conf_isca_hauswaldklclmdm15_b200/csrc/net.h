@@ -45,7 +45,15 @@ struct LayerSpec {
 
 enum OpKind { OP_PACK, OP_GEMM, OP_LRN, OP_POOL, OP_SOFTMAX };
 
-struct Shape { int C = 0, H = 1, W = 1, Cp = 0; int64_t per_row() const { return (int64_t)H * W * Cp; } };
+// Per-row activation tensor: NHWC, channel pitch Cp.  Channels may be stored in groups of
+// gsz at a per-group pitch gpitch (logical channel c lives at (c / gsz) * gpitch + c % gsz),
+// so that a grouped convolution's per-group K is 16/32/64-aligned (one TMA row per tap).
+struct Shape {
+  int C = 0, H = 1, W = 1, Cp = 0;
+  int gsz = 1 << 30, gpitch = 1 << 30;
+  int64_t per_row() const { return (int64_t)H * W * Cp; }
+  int pos(int c) const { return (c / gsz) * gpitch + c % gsz; }
+};
 
 struct Op {
   OpKind kind;
@@ -122,7 +130,8 @@ struct Net {
 
 std::atomic<int64_t>& launch_counter();
 void encode_tmap(CUtensorMap* m, int dt, const void* base, int rank, const uint64_t* dims,
-                 const uint64_t* strides_bytes, const uint32_t* box, int swizzle_bytes = 128);
+                 const uint64_t* strides_bytes, const uint32_t* box, int swizzle_bytes = 128,
+                 const uint32_t* elem_strides = nullptr);
 void encode_im2col(CUtensorMap* m, int dt, const void* base, const uint64_t* dims, const uint64_t* strides_bytes,
                    const int* lower_wh, const int* upper_wh, int channels, int pixels, const uint32_t* elem_strides);
 

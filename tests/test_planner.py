@@ -1,0 +1,76 @@
+"""Host-side planner of libdjinn (djinn_describe: no device needed) -m "not gpu".
+
+Checks the library's own parse + shape inference against the oracle's independent one
+(parameter and layer counts), the plan decisions the kernels rely on, and the
+synchronous error paths of the description parser."""
+import pytest
+
+import paper_conf_isca_hauswaldklclmdm15_b200 as dj
+from oracle import OracleNet
+from oracle.calibrate import net_text
+
+APPS = ["imc", "dig", "face", "asr", "pos", "chk", "ner"]
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _built():
+    from paper_conf_isca_hauswaldklclmdm15_b200 import build
+    build.build()
+
+
+@pytest.mark.parametrize("prec", [dj.DJINN_FP32, dj.DJINN_BF16, dj.DJINN_FP16])
+@pytest.mark.parametrize("app", APPS)
+def test_counts_match_the_oracle(app, prec):
+    plan, in_e, out_e, n_params, n_layers = dj.djinn_describe(dj.net_description(app), prec, 64)
+    ref = OracleNet(net_text(app))
+    assert n_params == ref.n_params()
+    assert n_layers == ref.n_layers()
+    assert in_e == int(__import__("numpy").prod(ref.input_shape))
+    assert out_e == ref.out_dim
+
+
+def test_plan_first_layer_transforms_and_lrn_fusion():
+    imc = dj.djinn_describe(dj.net_description("imc"), dj.DJINN_BF16, 64)[0]
+    assert "space-to-depth 4" in imc
+    assert "conv1+norm1" in imc and "conv2+norm2" in imc and "lrn-epilogue" in imc
+    assert "48x57x57/p64" in imc                      # s2d: 4*4*3 channels at a 128-byte pitch
+    assert "96x27x27/p128" in imc                     # conv2 input: two groups of 48 at pitch 64
+    face = dj.djinn_describe(dj.net_description("face"), dj.DJINN_FP16, 64)[0]
+    assert "kx-unroll 11" in face and "KHxKW=11x1" in face
+    fp32 = dj.djinn_describe(dj.net_description("imc"), dj.DJINN_FP32, 64)[0]
+    assert "lrn norm1" in fp32 and "space-to-depth" not in fp32   # fp32 path: plain SIMT plan
+
+
+def test_asr_uses_centered_sigmoid_on_16bit_paths():
+    p16 = dj.djinn_describe(dj.net_description("asr"), dj.DJINN_BF16, 64)[0]
+    p32 = dj.djinn_describe(dj.net_description("asr"), dj.DJINN_FP32, 64)[0]
+    assert p16.count("act=5") == 6 and "act=5" not in p32
+
+
+@pytest.mark.parametrize("desc,code", [
+    ("layer { name: 'x' type: 'Input' ", dj.DJINN_E_PARSE),
+    ("layer { name: \"d\" type: \"Input\" top: \"d\" input_param { shape { dim: 4 } } }", dj.DJINN_E_UNSUPPORTED),
+    ("layer { type: \"Input\" input_param { shape { dim: 4 } } } layer { type: \"Swish\" } "
+     "layer { type: \"Softmax\" }", dj.DJINN_E_UNSUPPORTED),
+    ("layer { type: \"InnerProduct\" inner_product_param { num_output: 3 } } layer { type: \"Softmax\" }",
+     dj.DJINN_E_SHAPE),
+    ("layer { type: \"Input\" input_param { shape { dim: 3 dim: 5 dim: 5 } } } layer { type: \"Convolution\" "
+     "convolution_param { num_output: 4 kernel_size: 7 } } layer { type: \"InnerProduct\" "
+     "inner_product_param { num_output: 2 } } layer { type: \"Softmax\" }", dj.DJINN_E_SHAPE),
+    ("layer { type: \"Input\" input_param { shape { dim: 3 dim: 8 dim: 8 } } } layer { type: \"Convolution\" "
+     "convolution_param { num_output: 4 kernel_size: 3 group: 2 } } layer { type: \"InnerProduct\" "
+     "inner_product_param { num_output: 2 } } layer { type: \"Softmax\" }", dj.DJINN_E_SHAPE),
+])
+def test_description_errors(desc, code):
+    with pytest.raises(dj.DjinnError) as e:
+        dj.djinn_describe(desc, dj.DJINN_BF16, 16)
+    assert e.value.code == code
+
+
+def test_describe_argument_errors():
+    with pytest.raises(dj.DjinnError) as e:
+        dj.djinn_describe(dj.net_description("pos"), 9, 16)
+    assert e.value.code == dj.DJINN_E_INVAL
+    with pytest.raises(dj.DjinnError) as e:
+        dj.djinn_describe(dj.net_description("pos"), dj.DJINN_BF16, 0)
+    assert e.value.code == dj.DJINN_E_INVAL
