@@ -328,22 +328,34 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
   if (warp == TMA_WARP) {
     if (lane == 0) {
-      const int cw = g.cw, cbytes = BM * cw * 2, cpt = g.Cgp / cw;
+      // Division-free address generation: the (ky, kx, c) of each K chunk is advanced with
+      // counters (integer division on the single issuing thread throttled the TMA stream).
+      const int cw = g.cw, cbytes = BM * cw * 2;
+      const int chunks_per_kb = BK / cw;
       const int nchunks_k = g.K / cw;  // valid chunks along K
+      const int oy_per = g.OH * g.OW;
       int it = 0;
       for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
         const TileCoord tc = tile_coord(g, t, mt, nt);
         // conv: top-left input pixel of the filter window of the tile's first output pixel
         int wx = tc.x0 * g.stride - g.pad, wy = tc.y0 * g.stride - g.pad, img = tc.i0;
         if (g.mode == GM_CONV && !g.a_tiled) {
-          img = tc.m0 / (g.OH * g.OW);
-          const int rem = tc.m0 - img * g.OH * g.OW;
+          img = tc.m0 / oy_per;
+          const int rem = tc.m0 - img * oy_per;
           const int oy = rem / g.OW;
           wy = oy * g.stride - g.pad;
           wx = (rem - oy * g.OW) * g.stride - g.pad;
         }
         for (int zi = 0; zi < g.zf; ++zi) {
           const int z = tc.z0 * g.zf + zi;
+          int lcx = 0, lcy = 0;  // LC: input pixel of the location
+          if (g.mode == GM_LC) {
+            const int oy = z / g.OW;
+            lcy = oy * g.stride;
+            lcx = (z - oy * g.OW) * g.stride;
+          }
+          const int cbase = g.mode == GM_CONV ? z * g.cin_goff : 0;
+          int cc = 0, kx = 0, ky = 0, q = 0;  // chunk counters: channel offset, tap, chunk index
           for (int kb = 0; kb < num_kb; ++kb, ++it) {
             const int s = it % C::STAGES;
             const uint32_t ph = (it / C::STAGES) & 1;
@@ -354,24 +366,20 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             if (g.mode == GM_DENSE) {
               tma_2d(a_dst, &tmA, fb, kb * BK, tc.m0);
             } else {
-              for (int j = 0; j < BK / cw; ++j) {
-                const int q = kb * (BK / cw) + j;
-                int c, kx = 0, ky = 0;
-                if (q < nchunks_k) {
-                  const int tap = q / cpt;
-                  c = (q - tap * cpt) * cw + (g.mode == GM_CONV ? z * g.cin_goff : 0);
-                  ky = tap / g.KW;
-                  kx = tap - ky * g.KW;
-                } else {
-                  c = g.Cp_in;  // past the channel extent: TMA zero-fills the K tail
-                }
+              for (int j = 0; j < chunks_per_kb; ++j, ++q) {
+                // past the valid K: a channel coordinate beyond the extent -> TMA zero-fills
+                const int c = q < nchunks_k ? cbase + cc : g.Cp_in;
                 const uint32_t dst = a_dst + j * cbytes;
                 if (g.mode == GM_CONV) {
                   if (g.a_tiled) tma_4d(dst, &tmA, fb, c, wx + kx, wy + ky, img);
                   else tma_im2col_4d(dst, &tmA, fb, c, wx, wy, img, (uint16_t)kx, (uint16_t)ky);
                 } else {  // LC: rows are images at the fixed output location z
-                  const int oy = z / g.OW, ox = z - (z / g.OW) * g.OW;
-                  tma_4d(dst, &tmA, fb, c, ox * g.stride + kx, oy * g.stride + ky, tc.m0);
+                  tma_4d(dst, &tmA, fb, c, lcx + kx, lcy + ky, tc.m0);
+                }
+                cc += cw;
+                if (cc == g.Cgp) {
+                  cc = 0;
+                  if (++kx == g.KW) { kx = 0; ++ky; }
                 }
               }
             }
