@@ -16,7 +16,7 @@ from typing import Optional
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libdjinn.so")
+LIB_PATH = os.environ.get("DJINN_LIB") or os.path.join(_HERE, "libdjinn.so")
 NETS_DIR = os.path.join(_HERE, "nets")
 
 DJINN_OK, DJINN_E_INVAL, DJINN_E_PARSE, DJINN_E_SHAPE, DJINN_E_WEIGHTS = 0, -1, -2, -3, -4

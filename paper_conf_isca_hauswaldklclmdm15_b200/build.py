@@ -9,12 +9,14 @@ from concurrent.futures import ThreadPoolExecutor
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 ROOT = os.path.dirname(HERE)
-LIB = os.path.join(HERE, "libdjinn.so")
-OBJ = os.path.join(HERE, "build")
+VARIANT = os.environ.get("DJINN_BUILD_VARIANT", "")          # "stats": role-timing instrumentation
+LIB = os.path.join(HERE, "libdjinn%s.so" % ("_" + VARIANT if VARIANT else ""))
+OBJ = os.path.join(HERE, "build" + ("_" + VARIANT if VARIANT else ""))
 SOURCES = ["api.cu", "net.cu", "k_misc.cu", "k_simt.cu", "k_tc.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
-         "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "-I", os.path.join(ROOT, "include")]
+         "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "-I", os.path.join(ROOT, "include")] + \
+        (["-DDJINN_TC_STATS"] if VARIANT == "stats" else [])
 HEADERS = [os.path.join(CSRC, h) for h in os.listdir(CSRC) if h.endswith((".h", ".cuh"))] + \
           [os.path.join(ROOT, "include", "djinn.h")]
 

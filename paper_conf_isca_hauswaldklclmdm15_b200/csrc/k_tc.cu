@@ -32,6 +32,15 @@
 
 #include "kernels.h"
 
+#ifdef DJINN_TC_STATS
+#include <cstdio>
+#define STAT_T0() const unsigned long long _t0 = clock64()
+#define STAT_ADD(v) (v) += clock64() - _t0
+#else
+#define STAT_T0()
+#define STAT_ADD(v)
+#endif
+
 namespace djinn {
 namespace {
 
@@ -294,6 +303,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int num_kb = g.Kpad / BK;
+#ifdef DJINN_TC_STATS
+  unsigned long long st_prod_wait = 0, st_mma_full = 0, st_mma_tempty = 0, st_mma_issue = 0, st_epi_wait = 0,
+                     st_epi_work = 0;
+  const unsigned long long st_begin = clock64();
+#endif
   const int mt = num_m_tiles(g), nt = (g.N + BN - 1) / BN, zt = g.Z / g.zf;
   const int tiles = mt * nt * zt;
   const int slot_cols = g.zf * BN;
@@ -359,7 +373,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           for (int kb = 0; kb < num_kb; ++kb, ++it) {
             const int s = it % C::STAGES;
             const uint32_t ph = (it / C::STAGES) & 1;
-            mbar_wait(empty0 + 8 * s, ph ^ 1);
+            {
+              STAT_T0();
+              mbar_wait(empty0 + 8 * s, ph ^ 1);
+              STAT_ADD(st_prod_wait);
+            }
             const uint32_t fb = full0 + 8 * s;
             mbar_arrive_expect_tx(fb, C::A_BYTES + C::B_BYTES);
             const uint32_t a_dst = smem_u32(sA + s * C::A_BYTES);
@@ -397,15 +415,24 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++lt) {
         const int slot = nslots == 2 ? (lt & 1) : 0;
         const uint32_t use = nslots == 2 ? (uint32_t)(lt >> 1) : (uint32_t)lt;
-        mbar_wait(tempty0 + 8 * slot, (use & 1) ^ 1);
+        {
+          STAT_T0();
+          mbar_wait(tempty0 + 8 * slot, (use & 1) ^ 1);
+          STAT_ADD(st_mma_tempty);
+        }
         tc_fence_after();
         for (int zi = 0; zi < g.zf; ++zi) {
           const uint32_t d = tmem + (uint32_t)(slot * slot_cols + zi * BN);
           for (int kb = 0; kb < num_kb; ++kb, ++it) {
             const int s = it % C::STAGES;
             const uint32_t ph = (it / C::STAGES) & 1;
-            mbar_wait(full0 + 8 * s, ph);
+            {
+              STAT_T0();
+              mbar_wait(full0 + 8 * s, ph);
+              STAT_ADD(st_mma_full);
+            }
             tc_fence_after();
+            STAT_T0();
             const uint32_t a0 = smem_u32(sA + s * C::A_BYTES);
             const uint64_t bd = sdesc(smem_u32(sB + s * C::B_BYTES), 128);
 #pragma unroll
@@ -415,6 +442,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
               mma_f16(d, ad, bd + 2 * k, idesc, (kb | k) != 0);
             }
             mma_commit(empty0 + 8 * s);
+            STAT_ADD(st_mma_issue);
           }
         }
         mma_commit(tfull0 + 8 * slot);
@@ -441,8 +469,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         m = tc.m0 + r;
         mok = m < g.M;
       }
-      mbar_wait(tfull0 + 8 * slot, use & 1);
+      {
+        STAT_T0();
+        mbar_wait(tfull0 + 8 * slot, use & 1);
+        STAT_ADD(st_epi_wait);
+      }
       tc_fence_after();
+      STAT_T0();
       const uint32_t tbase = tmem + lane_base + (uint32_t)(slot * slot_cols);
       if (g.epi_lrn) {
         // Channels c = zi * N + n (N == BN when zf > 1) live in columns zi*BN + n.  The LRN
@@ -550,11 +583,19 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           }
         }
       }
+      STAT_ADD(st_epi_work);
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(tempty0 + 8 * slot);
     }
   }
+#ifdef DJINN_TC_STATS
+  if (blockIdx.x == 0 && (threadIdx.x == TMA_WARP * 32 || threadIdx.x == MMA_WARP * 32 || threadIdx.x == 0))
+    printf("[tc BN=%d mode=%d N=%d K=%d tiles=%d grid=%d] warp %d total %llu prod_wait %llu mma_full %llu "
+           "mma_tempty %llu mma_issue %llu epi_wait %llu epi_work %llu\n",
+           BN, g.mode, g.N, g.K, tiles, gridDim.x, warp, clock64() - st_begin, st_prod_wait, st_mma_full, st_mma_tempty,
+           st_mma_issue, st_epi_wait, st_epi_work);
+#endif
   tc_fence_before();
   __syncthreads();
   if (warp == MMA_WARP) {
