@@ -28,8 +28,6 @@ import sys
 import threading
 import time
 
-import numpy as np
-
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
@@ -40,7 +38,7 @@ BATCH_ROWS = {"imc": 1024, "face": 256, "asr": 8192, "pos": 4096, "chk": 4096, "
 ROWS_PER_QUERY = recipes.ROWS_PER_QUERY
 METRIC = "queries/sec per Tonic app at 1/2/4/8 B200; % tensor peak (GEMM) / % HBM BW"
 # oracle sample per app for the CPU baseline / reference arm (rows)
-CPU_SAMPLE = {"imc": 1, "face": 1, "asr": 64, "pos": 28, "chk": 28, "ner": 28, "dig": 10}
+CPU_SAMPLE = {"imc": 4, "face": 4, "asr": 256, "pos": 280, "chk": 280, "ner": 280, "dig": 100}
 
 
 def load_peaks():
@@ -59,29 +57,42 @@ def queries_per_step(world: int = 1) -> float:
 
 # ------------------------------------------------------------------ clocks sampler
 class ClockSampler:
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+    """nvidia-smi clocks / throttle reasons sampled every 50 ms in a background process; only
+    samples whose host timestamp falls inside [mark_start, mark_end] (the timed region) are
+    summarised (B200_PROFILING.md "clocks DURING the timed region")."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
 
     def __init__(self, device: int):
         self.device = device
         self.rows = []
         self.proc = None
+        self.t0 = self.t1 = None
 
     def __enter__(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
+            time.sleep(0.3)          # let the sampler start before the timed region
         except OSError:
             self.proc = None
         return self
 
     def _read(self):
         for line in self.proc.stdout:
-            self.rows.append([x.strip() for x in line.split(",")])
+            self.rows.append((time.time(), [x.strip() for x in line.split(",")]))
+
+    def mark_start(self):
+        self.t0 = time.time()
+
+    def mark_end(self):
+        self.t1 = time.time()
+        time.sleep(0.1)
 
     def __exit__(self, *a):
         if self.proc:
@@ -92,63 +103,84 @@ class ClockSampler:
                 self.proc.kill()
 
     def summary(self):
-        if not self.rows:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
-        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
-        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 5 + i and r[5 + i] == "Active"})
-        pw = [float(r[3]) for r in self.rows if r[3].replace(".", "").isdigit()]
+        rows = [r for t, r in self.rows if self.t0 is None or (self.t0 - 0.05 <= t <= (self.t1 or t) + 0.05)]
+        num = lambda x: x.replace(".", "", 1).isdigit()
+        sm = [float(r[0]) for r in rows if num(r[0])]
+        mx = [float(r[1]) for r in rows if len(r) > 1 and num(r[1])]
+        pw = [float(r[2]) for r in rows if len(r) > 2 and num(r[2])]
+        reasons = sorted({self.NAMES[i] for r in rows for i in range(4) if len(r) > 3 + i and r[3 + i] == "Active"})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows), "power_w_max": max(pw) if pw else None}
+                "reasons": reasons, "samples": len(rows), "power_w_max": max(pw) if pw else None}
 
 
 # ------------------------------------------------------------------ CPU oracle leg
-def run_oracle_sample(apps=APPS, threads=None):
-    """Time the fp64 oracle (as it stands) on CPU_SAMPLE rows of each app.
-    Returns (mixed-workload queries/s extrapolated from per-app s/row, detail)."""
-    from oracle import OracleNet
-    from oracle.calibrate import net_text
-    detail = {}
-    step_s = 0.0
-    for app in apps:
-        net = OracleNet(net_text(app))
-        W = recipes.gen_weights(app, "fp32")
-        n = CPU_SAMPLE[app]
-        x = recipes.gen_input_rows(app, 0, n, "fp32")
-        t0 = time.perf_counter()
-        net.forward(x, W)
-        dt = time.perf_counter() - t0
-        s_per_row = dt / n
-        detail[app] = {"rows": n, "seconds": dt, "queries_per_s": 1.0 / (s_per_row * ROWS_PER_QUERY[app])}
-        step_s += s_per_row * BATCH_ROWS[app]
-    return queries_per_step() / step_s, detail
+class OracleSample:
+    """The fp64 oracle (as it stands, untuned) on CPU_SAMPLE rows of each app.  Nets, weights
+    and inputs are prepared once; run() times only the oracle forward passes and returns the
+    mixed-workload queries/s extrapolated from the measured seconds per row of each app."""
+
+    def __init__(self, apps=APPS):
+        from oracle import OracleNet
+        from oracle.calibrate import net_text
+        self.apps = list(apps)
+        self.items = {}
+        for app in self.apps:
+            net = OracleNet(net_text(app))
+            W = recipes.gen_weights(app, "fp32")
+            x = recipes.gen_input_rows(app, 0, CPU_SAMPLE[app], "fp32")
+            self.items[app] = (net, W, x)
+
+    def run(self):
+        detail, step_s = {}, 0.0
+        for app in self.apps:
+            net, W, x = self.items[app]
+            n = x.shape[0]
+            t0 = time.perf_counter()
+            net.forward(x, W)
+            dt = time.perf_counter() - t0
+            s_per_row = dt / n
+            detail[app] = {"rows": n, "seconds": dt, "queries_per_s": 1.0 / (s_per_row * ROWS_PER_QUERY[app])}
+            step_s += s_per_row * BATCH_ROWS[app]
+        qps = sum(BATCH_ROWS[a] / ROWS_PER_QUERY[a] for a in self.apps) / step_s
+        return qps, detail
+
+
+def cpu_threads():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count()
+
+
+def sample_desc(apps=APPS):
+    return ("oracle forward on " + ", ".join(f"{a} {CPU_SAMPLE[a]} rows" for a in apps) +
+            "; mixed-step queries/s extrapolated from the measured seconds per row of each app")
 
 
 def reference_arm(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
-    cores = os.cpu_count()
+    ref = OracleSample()
     for _ in range(args.warmup):
-        run_oracle_sample()
-    vals = []
+        ref.run()
+    vals, per_app = [], {}
     t0 = time.perf_counter()
     for _ in range(args.steps):
-        v, detail = run_oracle_sample()
+        v, detail = ref.run()
         vals.append(v)
+        per_app = detail
     wall = time.perf_counter() - t0
     value = statistics.median(vals)
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * wall / max(1, args.steps),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": "tonic-mixed (Table 5 MIXED): one batch of every app per step",
-                       "batch_rows": BATCH_ROWS, "oracle_sample_rows": CPU_SAMPLE},
-            "cpu_baseline": {"value": value, "unit": "queries/s", "cores": cores, "kind": "oracle",
-                             "sample": "per step: " + ", ".join(f"{a} {CPU_SAMPLE[a]} rows" for a in APPS)
-                                       + "; extrapolated to the mixed step by measured seconds/row"},
+                       "batch_rows_per_gpu": BATCH_ROWS, "oracle_sample_rows": CPU_SAMPLE},
+            "cpu_baseline": {"value": value, "unit": "queries/s", "cores": cpu_threads(), "kind": "oracle",
+                             "sample": sample_desc()},
             "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
-            "per_app_queries_per_s": {a: d["queries_per_s"] for a, d in detail.items()}}
+            "per_app_queries_per_s": {a: d["queries_per_s"] for a, d in per_app.items()}}
     print(json.dumps(line), flush=True)
     return 0
 
@@ -157,7 +189,7 @@ def reference_arm(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=60)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="b200", choices=["b200", "reference"])
     ap.add_argument("--precision", default=os.environ.get("DJINN_BENCH_PRECISION", "bf16"),
@@ -175,6 +207,7 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_isca_hauswaldklclmdm15_b200 as dj
+    from paper_conf_isca_hauswaldklclmdm15_b200 import parallel
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -194,13 +227,10 @@ def main():
         w = recipes.flat_blob(recipes.gen_weights(app, grid)) if rank == 0 else None
         net = dj.DjinnNet(dj.net_description(app), w, grid, rows, local)
         if world > 1:
-            ptr, nbytes = net.arena()
-
-            class _Arena:
-                __cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (ptr, False), "version": 3}
-            dist.broadcast(torch.as_tensor(_Arena(), device="cuda"), src=0)
+            parallel.broadcast_buffer(parallel.arena_tensor(net), src=0)   # C1: one-time NCCL broadcast
         nets[app] = net
-        x = recipes.gen_input_rows(app, rank * rows, rows, grid)          # this rank's shard
+        r0, nrows = parallel.weak_shard(rows, rank)                         # this rank's own queries
+        x = recipes.gen_input_rows(app, r0, nrows, grid)
         inputs[app] = torch.from_numpy(x).cuda()
         outputs[app] = torch.empty(rows, net.out_elems, device="cuda")
         del w
@@ -223,12 +253,7 @@ def main():
             fn()
         e1.record(stream)
         barrier()
-        ms = e0.elapsed_time(e1)
-        if world > 1:
-            t = torch.tensor([ms], device="cuda")
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ms = t.item()
-        return ms
+        return parallel.max_over_ranks(e0.elapsed_time(e1), device="cuda")
 
     for _ in range(args.warmup):
         step()
@@ -237,7 +262,9 @@ def main():
         dj.djinn_profile(nets[app].handle, True)
     l0 = dj.djinn_kernel_launches()
     with ClockSampler(local) as clk:
+        clk.mark_start()
         ms = timed(step, args.steps)
+        clk.mark_end()
     launches = dj.djinn_kernel_launches() - l0
     ms_per_step = ms / args.steps
     qps = sum(BATCH_ROWS[a] / ROWS_PER_QUERY[a] for a in apps) * world / (ms_per_step / 1e3)
@@ -310,10 +337,8 @@ def main():
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        v, detail = run_oracle_sample(apps)
-        cpu = {"value": v, "unit": "queries/s", "cores": os.cpu_count(), "kind": "oracle",
-               "sample": "one oracle pass over " + ", ".join(f"{a} {CPU_SAMPLE[a]} rows" for a in apps)
-                         + "; mixed-step rate extrapolated from measured seconds/row",
+        v, detail = OracleSample(apps).run()
+        cpu = {"value": v, "unit": "queries/s", "cores": cpu_threads(), "kind": "oracle", "sample": sample_desc(apps),
                "per_app_queries_per_s": {a: d["queries_per_s"] for a, d in detail.items()}}
 
     if rank == 0:
