@@ -347,7 +347,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       const int cw = g.cw, cbytes = BM * cw * 2;
       const int chunks_per_kb = BK / cw;
       const int nchunks_k = g.K / cw;  // valid chunks along K
-      const int oy_per = g.OH * g.OW;
+      const int oy_per = g.OH * g.OWb;
       int it = 0;
       for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
         const TileCoord tc = tile_coord(g, t, mt, nt);
@@ -356,9 +356,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         if (g.mode == GM_CONV && !g.a_tiled) {
           img = tc.m0 / oy_per;
           const int rem = tc.m0 - img * oy_per;
-          const int oy = rem / g.OW;
+          const int oy = rem / g.OWb;
           wy = oy * g.stride - g.pad;
-          wx = (rem - oy * g.OW) * g.stride - g.pad;
+          wx = (rem - oy * g.OWb) * (g.xb > 1 ? g.xb : g.stride) - g.pad;
         }
         for (int zi = 0; zi < g.zf; ++zi) {
           const int z = tc.z0 * g.zf + zi;
@@ -539,6 +539,33 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           }
 #pragma unroll
           for (int j = 0; j < 16; ++j) cur[j] = nxt[j];
+        }
+      } else if (g.xb > 1) {
+        // x-blocked conv: row m = (img, oy, block), column c = dx * P + co with P = out_pitch;
+        // each 16-column chunk is channels [co0, co0+16) of output pixel block*xb + dx.
+        const int P = g.out_pitch, OWb = g.OWb;
+        const int img = m / (g.OH * OWb), rem = m - img * (g.OH * OWb);
+        const int oy = rem / OWb, ox0 = (rem - oy * OWb) * g.xb;
+        const int cols = BN / 2, cbeg = half * cols;
+        const int64_t rowpix = ((int64_t)img * g.OH + oy) * g.OW;
+#pragma unroll 1
+        for (int c = cbeg; c < cbeg + cols; c += 16) {
+          const int dx = c / P, co0 = c - dx * P;
+          float b[16];
+          load_bias16(b, bias, co0, g.Co);
+          uint32_t rr[16];
+          tmem_ld16(tbase + (uint32_t)c, rr);
+          tmem_wait_ld();
+          const int ox = ox0 + dx;
+          if (mok && ox < g.OW && c < g.N) {
+            float v[16];
+            bias_act16(v, rr, b, g.act);
+            if (co0 + 16 > g.Co) {
+#pragma unroll
+              for (int j = 0; j < 16; ++j) v[j] = co0 + j < g.Co ? v[j] : 0.f;
+            }
+            store16<BF16>(g, Y, (rowpix + ox) * P + co0, v, 2);
+          }
         }
       } else {
         // columns of each z-slice split between the two warps of a lane quarter

@@ -45,6 +45,9 @@ struct GemmGeom {
   // tensor-core path only
   int cw;             // A chunk width in elements (16 / 32 / 64): one TMA box per chunk
   int Nimg;           // conv: images in the batch
+  int xb, OWb;        // conv x-blocking: one GEMM row = xb adjacent output pixels (OWb blocks per
+                      // output row); columns are (dx, co) with co < out_pitch; 1 = off
+  int Co;             // real output channels (x-blocked conv: per dx)
   int a_tiled;        // conv: 0 = im2col-mode TMA over linear output pixels (default), 1 = tiled
                       //       4D boxes over bx x by x bn pixel blocks (DJINN_CONV_A=tiled)
   int bx, by, bn;     // conv: output-pixel block of one M tile (bx*by*bn == 128), x fastest

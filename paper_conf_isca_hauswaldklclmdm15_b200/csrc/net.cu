@@ -431,12 +431,29 @@ void Net::build(const std::string& desc) {
             g.stride = 1;
           }
         } else {
+          // kx-unroll, and x-block: each packed pixel holds U = k + XB - 1 horizontal taps so
+          // one GEMM row computes XB adjacent output pixels (N = XB * out pitch <= 256); the
+          // XB shifted copies of the kernel live in B.  Small-N layers then run full-rate MMAs
+          // (N <= 64 costs a 52-cycle floor per MMA on B200) and fetch XB x fewer A rows.
+          Shape os;
+          os.C = L.num_output; os.H = OH; os.W = OW;
+          os = layout_for(i + 1, os);
+          int XB = 1;
+          if (os.gsz >= os.C && os.Cp <= 64)
+            for (int xbc = 8; xbc >= 2; xbc /= 2)
+              if ((k + xbc - 1) * cur.C <= 64 && xbc * os.Cp <= 256) { XB = xbc; break; }
+          const int U = k + XB - 1, OWb = (OW + XB - 1) / XB;
           pk.xform = o.xform = 2;
-          pk.xf = o.xf = k;
+          pk.xf = o.xf = U;
           pk.out = Shape();
-          pk.out.C = k * cur.C; pk.out.H = cur.H; pk.out.W = cur.W - k + 1; pk.out.Cp = tap_pitch(k * cur.C);
-          g.H = cur.H; g.W = cur.W - k + 1; g.Cp_in = g.Cgp = pk.out.Cp;
+          pk.out.C = U * cur.C; pk.out.H = cur.H; pk.out.W = XB > 1 ? OWb * XB : OW; pk.out.Cp = tap_pitch(U * cur.C);
+          g.H = cur.H; g.W = pk.out.W; g.Cp_in = g.Cgp = pk.out.Cp;
           g.KH = k; g.KW = 1;
+          if (XB > 1) {
+            g.xb = XB;
+            g.OWb = OWb;
+            g.N = XB * os.Cp;
+          }
         }
         if (pk.xform) { o.in = pk.out; }
       }
@@ -448,7 +465,9 @@ void Net::build(const std::string& desc) {
       g.cout_goff = Cog;
       g.write_cols = grp == 1 ? o.out.Cp : Cog;
       g.bias_zstride = Cog;
-      o.ohw = lc ? 1 : OH * OW;
+      if (g.xb < 1) { g.xb = 1; g.OWb = OW; }
+      g.Co = Cog;
+      o.ohw = lc ? 1 : OH * g.OWb;
       g.zf = 1;
       g.cw = g.Cgp >= 64 ? 64 : g.Cgp;
       // M tile = a bx x by x bn block of output pixels (x fastest, product 128): the one with
@@ -622,12 +641,15 @@ void Net::load_weights(const float* w, size_t n, int mem) {
               if (o.xform == 1) {  // space-to-depth: tap (ky/f, kx/f), channel ((ky%f)*f + kx%f)*C0 + c
                 const int f = o.xf;
                 kk = (int64_t)((ky / f) * g.KW + kx / f) * g.Cgp + ((ky % f) * f + kx % f) * C0 + c;
-              } else if (o.xform == 2) {  // kx-unroll: tap ky, channel kx*C0 + c
+              } else if (o.xform == 2) {  // kx-unroll: tap ky, channel kx*C0 + c (+ x-block copies)
+                for (int dx = 1; dx < g.xb; ++dx)
+                  put(0, dx * g.out_pitch + co, (int64_t)ky * g.Cgp + (dx + kx) * C0 + c, w[off]);
                 kk = (int64_t)ky * g.Cgp + kx * C0 + c;
               } else {
                 kk = (int64_t)(ky * k + kx) * g.Cgp + c;
               }
-              put(co / g.N, co % g.N, kk, w[off++]);
+              if (g.xb > 1) put(0, co, kk, w[off++]);
+              else put(co / g.N, co % g.N, kk, w[off++]);
             }
       for (int co = 0; co < o.out.C; ++co) bdst[co] = w[off++];
     } else if (g.mode == GM_LC) {
@@ -713,9 +735,10 @@ Workspace* Net::workspace(cudaStream_t st) {
         encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 4, dims, strides, box, g.cw * 2, estr);
       } else if (g.mode == GM_CONV) {
         // filter-window top-left positions: w = -pad + i*stride, i < OW (same for h)
+        const int sx = g.xb > 1 ? g.xb : g.stride;
         const int lower[2] = {-g.pad, -g.pad};
-        const int upper[2] = {-g.pad + (g.OW - 1) * g.stride - (g.W - 1), -g.pad + (g.OH - 1) * g.stride - (g.H - 1)};
-        const uint32_t estr[4] = {1, (uint32_t)g.stride, (uint32_t)g.stride, 1};
+        const int upper[2] = {-g.pad + (g.OWb - 1) * sx - (g.W - 1), -g.pad + (g.OH - 1) * g.stride - (g.H - 1)};
+        const uint32_t estr[4] = {1, (uint32_t)sx, (uint32_t)g.stride, 1};
         encode_im2col(&w->tmA[i], dt, w->buf[o.in_buf], dims, strides, lower, upper, g.cw, 128, estr);
       } else {
         uint32_t box[4] = {(uint32_t)g.cw, 1, 1, 128};
@@ -815,7 +838,8 @@ std::string Net::plan_string() const {
     if (o.kind == OP_GEMM)
       s << " [" << modes[o.g.mode] << " N=" << o.g.N << " Z=" << o.g.Z << " K=" << o.g.K << " Kpad=" << o.g.Kpad
         << " act=" << o.g.act << " bn=" << o.bn << " cw=" << o.g.cw << " zf=" << o.g.zf << " KHxKW=" << o.g.KH << "x"
-        << o.g.KW << (o.g.mode == GM_CONV && o.g.a_tiled ? " block=" + std::to_string(o.g.bx) + "x" + std::to_string(o.g.by) + "x" +
+        << o.g.KW << (o.g.xb > 1 ? " xblock=" + std::to_string(o.g.xb) : std::string())
+        << (o.g.mode == GM_CONV && o.g.a_tiled ? " block=" + std::to_string(o.g.bx) + "x" + std::to_string(o.g.by) + "x" +
                                                   std::to_string(o.g.bn) : std::string())
         << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << "]";
     if (o.kind == OP_PACK && o.xform) s << " [" << (o.xform == 1 ? "space-to-depth " : "kx-unroll ") << o.xf << "]";
