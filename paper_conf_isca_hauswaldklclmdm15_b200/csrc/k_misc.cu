@@ -212,16 +212,22 @@ __global__ void pool_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t 
 // 16-bit storage: 8 channels (16 B) per thread, fp32 math.
 template <typename T>
 __global__ void pool16_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t rows, int Cp, int H, int W,
-                              int OH, int OW, int kern, int stride, int pad, int is_max) {
-  const int chunks = Cp / 8;
+                              int OH, int OW, int kern, int stride, int pad, int is_max, int out_xu) {
+  const int cchunks = Cp / 8, chunks = cchunks * out_xu;
   const int per_row = OH * OW * chunks;
   for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
     const T* xr = x + r * (int64_t)H * W * Cp;
     T* yr = y + r * (int64_t)per_row * 8;
     for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < per_row; i += gridDim.x * blockDim.x) {
-      const int ch = i % chunks;
+      const int chx = i % chunks;
       const int pix = i / chunks;
-      const int oy = pix / OW, ox = pix - (pix / OW) * OW;
+      const int oy = pix / OW;
+      const int slot = chx / cchunks, ch = chx - slot * cchunks;
+      const int ox = pix - oy * OW + slot;  // x-unrolled output: slot s holds pixel x + s
+      if (ox >= OW) {
+        *reinterpret_cast<uint4*>(yr + (int64_t)i * 8) = make_uint4(0, 0, 0, 0);
+        continue;
+      }
       int hs = oy * stride - pad, ws = ox * stride - pad;
       int he = min(hs + kern, H + pad), we = min(ws + kern, W + pad);
       const float area = (float)((he - hs) * (we - ws));
@@ -246,16 +252,16 @@ __global__ void pool16_kernel(const T* __restrict__ x, T* __restrict__ y, int64_
 }
 
 cudaError_t launch_pool(const void* x, void* y, int64_t rows, int C, int Cp, int H, int W, int OH,
-                        int OW, int kernel, int stride, int pad, int is_max, int dt, cudaStream_t st) {
+                        int OW, int kernel, int stride, int pad, int is_max, int out_xu, int dt, cudaStream_t st) {
   (void)C;
   const int T = 256;
   if (dt != DT_F32 && Cp % 8 == 0) {
-    const int per_row = OH * OW * (Cp / 8);
+    const int per_row = OH * OW * (Cp / 8) * out_xu;
     dim3 g(min(nblocks(per_row, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
     if (dt == DT_F16)
-      pool16_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
+      pool16_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
     else
-      pool16_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
+      pool16_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
     return cudaGetLastError();
   }
   const int64_t n = rows * (int64_t)OH * OW * Cp;

@@ -390,14 +390,22 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 const uint32_t dst = a_dst + j * cbytes;
                 if (g.mode == GM_CONV) {
                   if (g.a_tiled) tma_4d(dst, &tmA, fb, c, wx + kx, wy + ky, img);
-                  else tma_im2col_4d(dst, &tmA, fb, c, wx, wy, img, (uint16_t)kx, (uint16_t)ky);
+                  else tma_im2col_4d(dst, &tmA, fb, c, wx, wy, img, (uint16_t)(kx * g.kxs), (uint16_t)ky);
+                } else if (g.lcg > 1) {  // LC, lcg taps per row: 3D view {W*C, H, N}
+                  const int xe = q < nchunks_k ? (lcx + kx) * g.Cp_in : g.W * g.Cp_in;  // K tail: OOB
+                  tma_3d(dst, &tmA, fb, xe, lcy + ky, tc.m0);
                 } else {  // LC: rows are images at the fixed output location z
                   tma_4d(dst, &tmA, fb, c, lcx + kx, lcy + ky, tc.m0);
                 }
-                cc += cw;
-                if (cc == g.Cgp) {
-                  cc = 0;
-                  if (++kx == g.KW) { kx = 0; ++ky; }
+                if (g.lcg > 1) {
+                  kx += g.lcg;
+                  if (kx >= g.kwp) { kx = 0; ++ky; }
+                } else {
+                  cc += cw;
+                  if (cc == g.Cgp) {
+                    cc = 0;
+                    if (++kx == g.KW) { kx = 0; ++ky; }
+                  }
                 }
               }
             }

@@ -48,6 +48,8 @@ struct GemmGeom {
   int xb, OWb;        // conv x-blocking: one GEMM row = xb adjacent output pixels (OWb blocks per
                       // output row); columns are (dx, co) with co < out_pitch; 1 = off
   int Co;             // real output channels (x-blocked conv: per dx)
+  int lcg, kwp;       // LC: taps per TMA row (box {Cgp, lcg, 1, 128}) and KW padded to lcg
+  int kxs;            // conv: x offset between consecutive taps (x-unrolled input: xu), default 1
   int a_tiled;        // conv: 0 = im2col-mode TMA over linear output pixels (default), 1 = tiled
                       //       4D boxes over bx x by x bn pixel blocks (DJINN_CONV_A=tiled)
   int bx, by, bn;     // conv: output-pixel block of one M tile (bx*by*bn == 128), x fastest
@@ -87,8 +89,10 @@ cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, in
                        float alpha, float beta, float k, int dt, cudaStream_t st);
 
 // --- pooling (K5), NHWC, Caffe ceil geometry ------------------------------------------------
+// Output may be x-unrolled: pixel x stores pooled pixels x..x+out_xu-1 at pitch Cp each
+// (out pitch out_xu*Cp); slots past the right edge are zero.
 cudaError_t launch_pool(const void* x, void* y, int64_t rows, int C, int Cp, int H, int W, int OH,
-                        int OW, int kernel, int stride, int pad, int is_max, int dt, cudaStream_t st);
+                        int OW, int kernel, int stride, int pad, int is_max, int out_xu, int dt, cudaStream_t st);
 
 // --- softmax / argmax / logits copy (K6) ----------------------------------------------------
 // logits fp32 [rows][pitch]; mode 0: prob fp32 [rows][N]; 1: argmax int32 [rows]; 2: logits copy.

@@ -457,6 +457,35 @@ void Net::build(const std::string& desc) {
         }
         if (pk.xform) { o.in = pk.out; }
       }
+      g.kxs = 1;
+      // Small-N stride-1 conv fed by a pooling layer: the pool writes an x-unrolled layout
+      // (pixel x also carries x+1.. up to 64 channels) and the conv x-blocks XB output pixels
+      // per GEMM row (N = XB * out pitch): full-rate MMAs and XB x fewer TMA rows.
+      if (f16 && !lc && grp == 1 && ops.size() > 1 && ops.back().kind == OP_POOL && o.xform == 0 && L.stride == 1 &&
+          pad == 0 && cur.gsz >= cur.C && cur.xu == 1 && cur.Cp <= 32 && 64 % cur.Cp == 0) {
+        Shape os;
+        os.C = L.num_output; os.H = OH; os.W = OW;
+        os = layout_for(i + 1, os);
+        const int xu = 64 / cur.Cp;
+        int XB = 1;
+        for (int xbc = 8; xbc >= 2; xbc /= 2)
+          if (xbc * os.Cp <= 256 && os.gsz >= os.C && os.Cp <= 64) { XB = xbc; break; }
+        if (XB > 1) {
+          Op& pl = ops.back();
+          pl.out.P = pl.out.Cp;
+          pl.out.xu = xu;
+          pl.out.Cp = xu * pl.out.P;
+          cur = pl.out;
+          o.in = cur;
+          const int KWg = (XB + L.kernel - 1 + xu - 1) / xu;
+          g.Cp_in = g.Cgp = cur.Cp;
+          g.KW = KWg;
+          g.kxs = xu;
+          g.xb = XB;
+          g.OWb = (OW + XB - 1) / XB;
+          g.N = XB * os.Cp;
+        }
+      }
       g.K = g.KH * g.KW * g.Cgp;
       o.out = Shape();
       o.out.C = L.num_output; o.out.H = OH; o.out.W = OW;
@@ -470,6 +499,16 @@ void Net::build(const std::string& desc) {
       o.ohw = lc ? 1 : OH * g.OWb;
       g.zf = 1;
       g.cw = g.Cgp >= 64 ? 64 : g.Cgp;
+      g.lcg = 1;
+      g.kwp = g.KW;
+      if (f16 && lc && g.Cgp < 64 && 64 % g.Cgp == 0 && g.KW > 1) {
+        // LC A rows are images at one location: put lcg horizontally adjacent taps in one
+        // 128-byte TMA row (box {Cgp, lcg, 1, 128}); the padded taps carry zero weights.
+        g.lcg = 64 / g.Cgp;
+        g.kwp = rup(g.KW, g.lcg);
+        g.K = g.KH * g.kwp * g.Cgp;
+        g.cw = 64;
+      }
       // M tile = a bx x by x bn block of output pixels (x fastest, product 128): the one with
       // the least padding waste for this layer's OW x OH x batch.
       const char* amode = getenv("DJINN_CONV_A");
@@ -641,6 +680,13 @@ void Net::load_weights(const float* w, size_t n, int mem) {
               if (o.xform == 1) {  // space-to-depth: tap (ky/f, kx/f), channel ((ky%f)*f + kx%f)*C0 + c
                 const int f = o.xf;
                 kk = (int64_t)((ky / f) * g.KW + kx / f) * g.Cgp + ((ky % f) * f + kx % f) * C0 + c;
+              } else if (o.in.xu > 1) {  // x-unrolled input + x-block: tap group j, slot i
+                for (int dx = 0; dx < g.xb; ++dx) {
+                  const int e = dx + kx, jj = e / g.kxs, ii = e % g.kxs;
+                  const int64_t ki = (int64_t)(ky * g.KW + jj) * g.Cgp + ii * o.in.P + c;
+                  if (dx > 0) put(0, dx * g.out_pitch + co, ki, w[off]);
+                  else kk = ki;
+                }
               } else if (o.xform == 2) {  // kx-unroll: tap ky, channel kx*C0 + c (+ x-block copies)
                 for (int dx = 1; dx < g.xb; ++dx)
                   put(0, dx * g.out_pitch + co, (int64_t)ky * g.Cgp + (dx + kx) * C0 + c, w[off]);
@@ -659,7 +705,7 @@ void Net::load_weights(const float* w, size_t n, int mem) {
           for (int c = 0; c < C; ++c)
             for (int ky = 0; ky < k; ++ky)
               for (int kx = 0; kx < k; ++kx)
-                put(loc, co, (int64_t)(ky * k + kx) * g.Cgp + c, w[off++]);
+                put(loc, co, (int64_t)(ky * g.kwp + kx) * g.Cgp + c, w[off++]);
       for (int co = 0; co < g.N; ++co)
         for (int loc = 0; loc < g.Z; ++loc) bdst[(int64_t)loc * g.N + co] = w[off++];
     } else {
@@ -738,8 +784,17 @@ Workspace* Net::workspace(cudaStream_t st) {
         const int sx = g.xb > 1 ? g.xb : g.stride;
         const int lower[2] = {-g.pad, -g.pad};
         const int upper[2] = {-g.pad + (g.OWb - 1) * sx - (g.W - 1), -g.pad + (g.OH - 1) * g.stride - (g.H - 1)};
+        if ((g.KW - 1) * g.kxs > g.W - 1 - ((g.OWb - 1) * sx - g.pad))
+          throw Error(DJINN_E_SHAPE, o.name + ": internal: tap offsets exceed the im2col box");
         const uint32_t estr[4] = {1, (uint32_t)sx, (uint32_t)g.stride, 1};
         encode_im2col(&w->tmA[i], dt, w->buf[o.in_buf], dims, strides, lower, upper, g.cw, 128, estr);
+      } else if (g.lcg > 1) {
+        // LC with lcg taps per row: view each image row as one dense run {W*C, H, N}; a box
+        // {lcg*C, 1, 128} is then lcg adjacent pixels = one 128-byte swizzle row per image.
+        uint64_t d3[3] = {(uint64_t)g.W * g.Cp_in, (uint64_t)g.H, (uint64_t)max_rows};
+        uint64_t s3[2] = {(uint64_t)g.W * g.Cp_in * 2, (uint64_t)g.H * g.W * g.Cp_in * 2};
+        uint32_t box[3] = {(uint32_t)g.cw, 1, 128};
+        encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 3, d3, s3, box, g.cw * 2);
       } else {
         uint32_t box[4] = {(uint32_t)g.cw, 1, 1, 128};
         encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 4, dims, strides, box, g.cw * 2);
@@ -805,7 +860,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           break;
         case OP_POOL:
           e = launch_pool(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.H, o.in.W, o.out.H, o.out.W,
-                          o.kernel, o.stride, o.pad, o.is_max, dt, st);
+                          o.kernel, o.stride, o.pad, o.is_max, o.out.xu, dt, st);
           break;
         case OP_SOFTMAX:
           e = launch_softmax((const float*)w->buf[2], n, (int)out_elems, out_pitch, dst, mode, st);
@@ -839,6 +894,8 @@ std::string Net::plan_string() const {
       s << " [" << modes[o.g.mode] << " N=" << o.g.N << " Z=" << o.g.Z << " K=" << o.g.K << " Kpad=" << o.g.Kpad
         << " act=" << o.g.act << " bn=" << o.bn << " cw=" << o.g.cw << " zf=" << o.g.zf << " KHxKW=" << o.g.KH << "x"
         << o.g.KW << (o.g.xb > 1 ? " xblock=" + std::to_string(o.g.xb) : std::string())
+        << (o.g.kxs > 1 ? " x-unrolled-input=" + std::to_string(o.g.kxs) : std::string())
+        << (o.g.lcg > 1 ? " taps/row=" + std::to_string(o.g.lcg) : std::string())
         << (o.g.mode == GM_CONV && o.g.a_tiled ? " block=" + std::to_string(o.g.bx) + "x" + std::to_string(o.g.by) + "x" +
                                                   std::to_string(o.g.bn) : std::string())
         << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << "]";

@@ -51,6 +51,7 @@ enum OpKind { OP_PACK, OP_GEMM, OP_LRN, OP_POOL, OP_SOFTMAX };
 struct Shape {
   int C = 0, H = 1, W = 1, Cp = 0;
   int gsz = 1 << 30, gpitch = 1 << 30;
+  int xu = 1, P = 0;  // x-unrolled layout: pixel x stores pixels x..x+xu-1, each at pitch P (Cp = xu*P)
   int64_t per_row() const { return (int64_t)H * W * Cp; }
   int pos(int c) const { return (c / gsz) * gpitch + c % gsz; }
 };
