@@ -117,8 +117,64 @@ __global__ void pack_xform_kernel(const float* __restrict__ x, T* __restrict__ y
   }
 }
 
+// Compile-time specialisation of the first-layer transforms for the Tonic nets: every source
+// offset is a constant relative to the pixel's base address, so each output channel costs one
+// load and one convert (the generic kernel spent its time in index bookkeeping).
+template <typename T, int MODE, int C, int F, int CP>
+__global__ void pack_xform_fixed_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int H, int W,
+                                        int Ho, int Wo) {
+  const int per_row = Ho * Wo;
+  for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
+    const float* src = x + r * C * (int64_t)H * W;
+    for (int pix = blockIdx.x * blockDim.x + threadIdx.x; pix < per_row; pix += gridDim.x * blockDim.x) {
+      const int yo = pix / Wo, xo = pix - (pix / Wo) * Wo;
+      T* dst = y + (r * per_row + pix) * (int64_t)CP;
+      const int y0 = MODE == 1 ? yo * F : yo, x0 = MODE == 1 ? xo * F : xo;
+      const float* p0 = src + (int64_t)y0 * W + x0;
+#pragma unroll
+      for (int ch = 0; ch < CP; ch += 8) {
+        __align__(16) T v[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const int cc = ch + j;
+          float val = 0.f;
+          if (MODE == 1) {
+            const int d = cc / C, c = cc % C, dy = d / F, dx = d % F;
+            if (d < F * F && y0 + dy < H && x0 + dx < W) val = __ldg(p0 + ((int64_t)c * H + dy) * W + dx);
+          } else {
+            const int kx = cc / C, c = cc % C;
+            if (kx < F && x0 + kx < W) val = __ldg(p0 + (int64_t)c * H * W + kx);
+          }
+          v[j] = cvt<T>(val);
+        }
+        *reinterpret_cast<uint4*>(dst + ch) = *reinterpret_cast<const uint4*>(v);
+      }
+    }
+  }
+}
+
+template <typename T>
+static bool launch_pack_fixed(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f, int Ho,
+                              int Wo, int Cp, cudaStream_t st) {
+  dim3 g(min(nblocks(Ho * Wo, 128), 1024), (unsigned)(rows < 65535 ? rows : 65535));
+  if (mode == 2 && C == 3 && f == 18 && Cp == 64)
+    pack_xform_fixed_kernel<T, 2, 3, 18, 64><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
+  else if (mode == 2 && C == 1 && f == 12 && Cp == 16)
+    pack_xform_fixed_kernel<T, 2, 1, 12, 16><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
+  else if (mode == 1 && C == 3 && f == 4 && Cp == 64)
+    pack_xform_fixed_kernel<T, 1, 3, 4, 64><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
+  else
+    return false;
+  return true;
+}
+
 cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f,
                               int Ho, int Wo, int Cp, int dt, cudaStream_t st) {
+  if (dt != DT_F32 && mode != 0) {
+    const bool done = dt == DT_F16 ? launch_pack_fixed<__half>(x, y, rows, C, H, W, mode, f, Ho, Wo, Cp, st)
+                                   : launch_pack_fixed<__nv_bfloat16>(x, y, rows, C, H, W, mode, f, Ho, Wo, Cp, st);
+    if (done) return cudaGetLastError();
+  }
   const int T = 256;
   if (dt == DT_F32) {
     int64_t n = rows * (int64_t)H * W * Cp;
@@ -210,6 +266,49 @@ __global__ void pool_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t 
 }
 
 // 16-bit storage: 8 channels (16 B) per thread, fp32 math.
+// x-unrolled output (out_xu > 1): each pooled pixel is computed once and stored into slot s
+// of pixel x - s for every s; slots past the right edge are zero-filled by pixel x's thread.
+template <typename T>
+__global__ void pool16_xu_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t rows, int Cp, int H, int W,
+                                 int OH, int OW, int kern, int stride, int pad, int is_max, int out_xu) {
+  const int cchunks = Cp / 8;
+  const int per_row = OH * OW * cchunks, Cpo = out_xu * Cp;
+  for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
+    const T* xr = x + r * (int64_t)H * W * Cp;
+    T* yr = y + r * (int64_t)OH * OW * Cpo;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < per_row; i += gridDim.x * blockDim.x) {
+      const int ch = i % cchunks;
+      const int pix = i / cchunks;
+      const int oy = pix / OW, ox = pix - oy * OW;
+      int hs = oy * stride - pad, ws = ox * stride - pad;
+      int he = min(hs + kern, H + pad), we = min(ws + kern, W + pad);
+      const float area = (float)((he - hs) * (we - ws));
+      hs = max(hs, 0); ws = max(ws, 0); he = min(he, H); we = min(we, W);
+      const T* base = xr + ch * 8;
+      float acc[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) acc[j] = is_max ? -FLT_MAX : 0.f;
+      for (int h = hs; h < he; ++h)
+        for (int w = ws; w < we; ++w) {
+          const uint4 u = __ldg(reinterpret_cast<const uint4*>(base + (h * W + w) * Cp));
+          const T* v = reinterpret_cast<const T*>(&u);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) acc[j] = is_max ? fmaxf(acc[j], ld(v + j)) : acc[j] + ld(v + j);
+        }
+      __align__(16) T o[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) o[j] = cvt<T>(is_max ? acc[j] : acc[j] / area);
+      const uint4 ov = *reinterpret_cast<const uint4*>(o);
+      for (int sl = 0; sl < out_xu; ++sl) {
+        if (ox - sl >= 0)
+          *reinterpret_cast<uint4*>(yr + ((int64_t)oy * OW + ox - sl) * Cpo + sl * Cp + ch * 8) = ov;
+        if (sl > 0 && ox + sl >= OW)
+          *reinterpret_cast<uint4*>(yr + ((int64_t)oy * OW + ox) * Cpo + sl * Cp + ch * 8) = make_uint4(0, 0, 0, 0);
+      }
+    }
+  }
+}
+
 template <typename T>
 __global__ void pool16_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t rows, int Cp, int H, int W,
                               int OH, int OW, int kern, int stride, int pad, int is_max, int out_xu) {
@@ -255,6 +354,15 @@ cudaError_t launch_pool(const void* x, void* y, int64_t rows, int C, int Cp, int
                         int OW, int kernel, int stride, int pad, int is_max, int out_xu, int dt, cudaStream_t st) {
   (void)C;
   const int T = 256;
+  if (dt != DT_F32 && Cp % 8 == 0 && out_xu > 1) {
+    const int per_row = OH * OW * (Cp / 8);
+    dim3 g(min(nblocks(per_row, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
+    if (dt == DT_F16)
+      pool16_xu_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
+    else
+      pool16_xu_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
+    return cudaGetLastError();
+  }
   if (dt != DT_F32 && Cp % 8 == 0) {
     const int per_row = OH * OW * (Cp / 8) * out_xu;
     dim3 g(min(nblocks(per_row, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));

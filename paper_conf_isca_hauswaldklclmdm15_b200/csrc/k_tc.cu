@@ -362,11 +362,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         }
         for (int zi = 0; zi < g.zf; ++zi) {
           const int z = tc.z0 * g.zf + zi;
-          int lcx = 0, lcy = 0;  // LC: input pixel of the location
+          int lcx = 0, lcy = 0;  // LC: input pixel of the location (block)
           if (g.mode == GM_LC) {
-            const int oy = z / g.OW;
+            const int oy = z / g.OWb;
             lcy = oy * g.stride;
-            lcx = (z - oy * g.OW) * g.stride;
+            lcx = (z - oy * g.OWb) * g.xb * g.stride;
           }
           const int cbase = g.mode == GM_CONV ? z * g.cin_goff : 0;
           int cc = 0, kx = 0, ky = 0, q = 0;  // chunk counters: channel offset, tap, chunk index
@@ -549,18 +549,29 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           for (int j = 0; j < 16; ++j) cur[j] = nxt[j];
         }
       } else if (g.xb > 1) {
-        // x-blocked conv: row m = (img, oy, block), column c = dx * P + co with P = out_pitch;
-        // each 16-column chunk is channels [co0, co0+16) of output pixel block*xb + dx.
+        // x-blocked conv / LC: column c = dx * P + co with P = out_pitch; each 16-column chunk
+        // is channels [co0, co0+16) of output pixel block*xb + dx.  Conv: row m = (img, oy,
+        // block); LC: row m = image, the block is the tile's z.
         const int P = g.out_pitch, OWb = g.OWb;
-        const int img = m / (g.OH * OWb), rem = m - img * (g.OH * OWb);
-        const int oy = rem / OWb, ox0 = (rem - oy * OWb) * g.xb;
+        int img, oy, ox0;
+        if (g.mode == GM_LC) {
+          img = m;
+          oy = tc.z0 / OWb;
+          ox0 = (tc.z0 - oy * OWb) * g.xb;
+        } else {
+          img = m / (g.OH * OWb);
+          const int rem = m - img * (g.OH * OWb);
+          oy = rem / OWb;
+          ox0 = (rem - oy * OWb) * g.xb;
+        }
         const int cols = BN / 2, cbeg = half * cols;
         const int64_t rowpix = ((int64_t)img * g.OH + oy) * g.OW;
+        const float* bb = g.mode == GM_LC ? bias + (int64_t)tc.z0 * g.bias_zstride : bias;
 #pragma unroll 1
         for (int c = cbeg; c < cbeg + cols; c += 16) {
           const int dx = c / P, co0 = c - dx * P;
           float b[16];
-          load_bias16(b, bias, co0, g.Co);
+          load_bias16(b, g.mode == GM_LC ? bb + dx * g.Co : bb, co0, g.Co);
           uint32_t rr[16];
           tmem_ld16(tbase + (uint32_t)c, rr);
           tmem_wait_ld();

@@ -503,11 +503,26 @@ void Net::build(const std::string& desc) {
       g.kwp = g.KW;
       if (f16 && lc && g.Cgp < 64 && 64 % g.Cgp == 0 && g.KW > 1) {
         // LC A rows are images at one location: put lcg horizontally adjacent taps in one
-        // 128-byte TMA row (box {Cgp, lcg, 1, 128}); the padded taps carry zero weights.
+        // 128-byte TMA row; the padded taps carry zero weights.  x-block XB adjacent
+        // locations per GEMM (N = XB * out pitch, each location's filter bank on its own
+        // columns, shifted by dx*stride taps): the A row is shared by XB locations, so the
+        // N = 16 MMA floor and the A traffic are amortised XB times.
         g.lcg = 64 / g.Cgp;
-        g.kwp = rup(g.KW, g.lcg);
-        g.K = g.KH * g.kwp * g.Cgp;
         g.cw = 64;
+        const int P = o.out.Cp;
+        int XB = 1;
+        if (o.out.gsz >= o.out.C && P <= 64)
+          for (int xbc = 8; xbc >= 2; xbc /= 2)
+            if (xbc * P <= 256 && (xbc - 1) * g.stride + g.KW <= 32) { XB = xbc; break; }
+        g.kwp = rup((XB - 1) * g.stride + g.KW, g.lcg);
+        g.K = g.KH * g.kwp * g.Cgp;
+        if (XB > 1) {
+          g.xb = XB;
+          g.OWb = (OW + XB - 1) / XB;
+          g.Z = OH * g.OWb;
+          g.N = XB * P;
+          g.bias_zstride = XB * Cog;
+        }
       }
       // M tile = a bx x by x bn block of output pixels (x fastest, product 128): the one with
       // the least padding waste for this layer's OW x OH x batch.
@@ -700,14 +715,24 @@ void Net::load_weights(const float* w, size_t n, int mem) {
       for (int co = 0; co < o.out.C; ++co) bdst[co] = w[off++];
     } else if (g.mode == GM_LC) {
       const int k = g.KH;
-      for (int loc = 0; loc < g.Z; ++loc)
-        for (int co = 0; co < g.N; ++co)
+      const int OH = g.OH, OW = g.OW, Co = g.Co, XB = g.xb;
+      for (int loc = 0; loc < OH * OW; ++loc) {
+        const int oy = loc / OW, ox = loc % OW;
+        const int z = XB > 1 ? oy * g.OWb + ox / XB : loc, dx = XB > 1 ? ox % XB : 0;
+        for (int co = 0; co < Co; ++co)
           for (int c = 0; c < C; ++c)
             for (int ky = 0; ky < k; ++ky)
               for (int kx = 0; kx < k; ++kx)
-                put(loc, co, (int64_t)(ky * g.kwp + kx) * g.Cgp + c, w[off++]);
-      for (int co = 0; co < g.N; ++co)
-        for (int loc = 0; loc < g.Z; ++loc) bdst[(int64_t)loc * g.N + co] = w[off++];
+                put(z, dx * (XB > 1 ? g.out_pitch : 0) + co, (int64_t)(ky * g.kwp + dx * g.stride + kx) * g.Cgp + c,
+                    w[off++]);
+      }
+      // bias [Co][OH][OW] -> [z][dx][co] (one row of Co per location, locations padded to XB)
+      for (int co = 0; co < Co; ++co)
+        for (int loc = 0; loc < OH * OW; ++loc) {
+          const int oy = loc / OW, ox = loc % OW;
+          const int64_t slot = XB > 1 ? (int64_t)(oy * g.OWb + ox / XB) * XB + ox % XB : loc;
+          bdst[slot * Co + co] = w[off++];
+        }
     } else {
       // Caffe flattens (c, h, w); our rows are (h, w, c) with channel pitch Cp.
       for (int nn = 0; nn < g.N; ++nn)
@@ -784,7 +809,7 @@ Workspace* Net::workspace(cudaStream_t st) {
         const int sx = g.xb > 1 ? g.xb : g.stride;
         const int lower[2] = {-g.pad, -g.pad};
         const int upper[2] = {-g.pad + (g.OWb - 1) * sx - (g.W - 1), -g.pad + (g.OH - 1) * g.stride - (g.H - 1)};
-        if ((g.KW - 1) * g.kxs > g.W - 1 - ((g.OWb - 1) * sx - g.pad))
+        if (-g.pad + (g.OWb - 1) * sx + (g.KW - 1) * g.kxs > g.W - 1 + g.pad)
           throw Error(DJINN_E_SHAPE, o.name + ": internal: tap offsets exceed the im2col box");
         const uint32_t estr[4] = {1, (uint32_t)sx, (uint32_t)g.stride, 1};
         encode_im2col(&w->tmA[i], dt, w->buf[o.in_buf], dims, strides, lower, upper, g.cw, 128, estr);

@@ -36,7 +36,9 @@ def test_plan_first_layer_transforms_and_lrn_fusion():
     assert "48x57x57/p64" in imc                      # s2d: 4*4*3 channels at a 128-byte pitch
     assert "96x27x27/p128" in imc                     # conv2 input: two groups of 48 at pitch 64
     face = dj.djinn_describe(dj.net_description("face"), dj.DJINN_FP16, 64)[0]
-    assert "kx-unroll 11" in face and "KHxKW=11x1" in face
+    assert "kx-unroll 18" in face and "KHxKW=11x1" in face and "xblock=8" in face   # 8 outputs per GEMM row
+    assert "32x71x71/p64" in face and "x-unrolled-input=2" in face                  # M2 -> C3
+    assert "taps/row=4" in face                                                      # L4-L6
     fp32 = dj.djinn_describe(dj.net_description("imc"), dj.DJINN_FP32, 64)[0]
     assert "lrn norm1" in fp32 and "space-to-depth" not in fp32   # fp32 path: plain SIMT plan
 
