@@ -91,9 +91,10 @@ int djinn_load_net(const char* desc, size_t desc_len, const float* weights, size
       djinn::GemmGeom g = o.g;
       g.M = (int)(n.max_rows * o.ohw);
       o.bn = djinn::tc_pick_bn(g);
+      o.g.cg = djinn::tc_pick_cg(g, o.bn);
       uint64_t dims[3] = {(uint64_t)g.Kpad, (uint64_t)g.N, (uint64_t)g.Z};
       uint64_t strides[2] = {(uint64_t)g.Kpad * 2, (uint64_t)g.N * g.Kpad * 2};
-      uint32_t box[3] = {64, (uint32_t)o.bn, 1};
+      uint32_t box[3] = {64, (uint32_t)(o.bn / o.g.cg), 1};
       djinn::encode_tmap(&o.tmB, n.dt, (uint8_t*)n.arena + o.w_off, 3, dims, strides, box);
     }
     if (weights) n.load_weights(weights, n_floats, weights_mem);
@@ -250,6 +251,7 @@ int djinn_describe(const char* desc, size_t desc_len, int precision, int64_t max
         djinn::GemmGeom g = o.g;
         g.M = (int)(n.max_rows * o.ohw);
         o.bn = djinn::tc_pick_bn(g);
+        o.g.cg = djinn::tc_pick_cg(g, o.bn);
       }
     if (in_elems) *in_elems = n.in_elems;
     if (out_elems) *out_elems = n.out_elems;

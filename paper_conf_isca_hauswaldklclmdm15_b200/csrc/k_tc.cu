@@ -29,6 +29,7 @@
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "kernels.h"
 
@@ -47,10 +48,10 @@ namespace {
 constexpr int BM = 128, BK = 64;
 constexpr int EPI_WARPS = 8, TMA_WARP = 8, MMA_WARP = 9, NUM_THREADS = 320;
 
-template <int BN>
+template <int BN, int CG = 1>
 struct Cfg {
   static constexpr int A_BYTES = BM * BK * 2;
-  static constexpr int B_BYTES = BN * BK * 2;
+  static constexpr int B_BYTES = (BN / CG) * BK * 2;  // cta_group::2: each CTA holds half of B
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int STAGES = (200 * 1024) / STAGE_BYTES > 8 ? 8 : (200 * 1024) / STAGE_BYTES;
   static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 512;
@@ -111,6 +112,63 @@ __device__ __forceinline__ void tma_im2col_4d(uint32_t dst, const CUtensorMap* m
       "l"((uint64_t)map), "r"(bar), "r"(c), "r"(w), "r"(h), "r"(n), "h"(ox), "h"(oy)
       : "memory");
 }
+// ---- cta_group::2 (CTA pair) forms.  Both CTAs issue their own half of the operands; the
+// transaction bytes land on the LEADER's (rank 0) barrier: its shared::cluster address is the
+// local one with the peer bit (bit 24) cleared.
+constexpr uint32_t PEER_MASK = 0xFEFFFFFFu;
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tma_2d_2sm(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+      ::"r"(dst), "l"((uint64_t)map), "r"(bar & PEER_MASK), "r"(c0), "r"(c1) : "memory");
+}
+__device__ __forceinline__ void tma_3d_2sm(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1, int c2) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5}], [%2];"
+      ::"r"(dst), "l"((uint64_t)map), "r"(bar & PEER_MASK), "r"(c0), "r"(c1), "r"(c2) : "memory");
+}
+__device__ __forceinline__ void tma_4d_2sm(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1, int c2,
+                                           int c3) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], [%2];"
+      ::"r"(dst), "l"((uint64_t)map), "r"(bar & PEER_MASK), "r"(c0), "r"(c1), "r"(c2), "r"(c3) : "memory");
+}
+__device__ __forceinline__ void tma_im2col_4d_2sm(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c, int w,
+                                                  int h, int n, uint16_t ox, uint16_t oy) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.im2col.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};"
+      ::"r"(dst), "l"((uint64_t)map), "r"(bar & PEER_MASK), "r"(c), "r"(w), "r"(h), "r"(n), "h"(ox), "h"(oy)
+      : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_leader(uint32_t bar) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(bar & PEER_MASK) : "memory");
+}
+template <int CG>
+__device__ __forceinline__ void tma_a2(uint32_t dst, const CUtensorMap* m, uint32_t bar, int c0, int c1) {
+  if (CG == 2) tma_2d_2sm(dst, m, bar, c0, c1); else tma_2d(dst, m, bar, c0, c1);
+}
+template <int CG>
+__device__ __forceinline__ void tma_a3(uint32_t dst, const CUtensorMap* m, uint32_t bar, int c0, int c1, int c2) {
+  if (CG == 2) tma_3d_2sm(dst, m, bar, c0, c1, c2); else tma_3d(dst, m, bar, c0, c1, c2);
+}
+template <int CG>
+__device__ __forceinline__ void tma_a4(uint32_t dst, const CUtensorMap* m, uint32_t bar, int c0, int c1, int c2, int c3) {
+  if (CG == 2) tma_4d_2sm(dst, m, bar, c0, c1, c2, c3); else tma_4d(dst, m, bar, c0, c1, c2, c3);
+}
+template <int CG>
+__device__ __forceinline__ void tma_i2c(uint32_t dst, const CUtensorMap* m, uint32_t bar, int c, int w, int h, int n,
+                                        uint16_t ox, uint16_t oy) {
+  if (CG == 2) tma_im2col_4d_2sm(dst, m, bar, c, w, h, n, ox, oy); else tma_im2col_4d(dst, m, bar, c, w, h, n, ox, oy);
+}
+
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
@@ -125,10 +183,10 @@ __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, int row_bytes) {
 }
 
 // Instruction descriptor, kind::f16: D fp32, A/B fp16 (0) or bf16 (1), both K-major, M=128.
-template <int BN, bool BF16>
+template <int BN, bool BF16, int CG = 1>
 __device__ __forceinline__ uint32_t idesc_f16() {
   const uint32_t ab = BF16 ? 1u : 0u;
-  return (1u << 4) | (ab << 7) | (ab << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+  return (1u << 4) | (ab << 7) | (ab << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)((BM * CG) >> 4) << 24);
 }
 
 __device__ __forceinline__ void mma_f16(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
@@ -141,6 +199,21 @@ __device__ __forceinline__ void mma_f16(uint32_t d_tmem, uint64_t adesc, uint64_
 }
 __device__ __forceinline__ void mma_commit(uint32_t bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mma_f16_2sm(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                            uint32_t accum) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum)
+      : "memory");
+}
+// commit to the barrier at this smem offset in BOTH CTAs of the pair
+__device__ __forceinline__ void mma_commit_2sm(uint32_t bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(bar),
+      "h"((uint16_t)3)
+      : "memory");
 }
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
   asm volatile(
@@ -263,10 +336,10 @@ struct TileCoord {
   int m0, n0, z0;      // m0: first GEMM row (dense / LC); n0: column block; z0: z group
   int x0, y0, i0;      // conv: first output pixel (x, y) and image of the block
 };
-__device__ __forceinline__ TileCoord tile_coord(const GemmGeom& g, int t, int mt, int nt) {
+__device__ __forceinline__ TileCoord tile_coord(const GemmGeom& g, int t, int mt, int nt, int cg = 1) {
   TileCoord c;
   const int tm = t % mt;
-  c.m0 = tm * BM;
+  c.m0 = tm * BM * cg;
   t /= mt;
   c.n0 = (t % nt);
   c.z0 = t / nt;
@@ -279,18 +352,21 @@ __device__ __forceinline__ TileCoord tile_coord(const GemmGeom& g, int t, int mt
   }
   return c;
 }
-__device__ __forceinline__ int num_m_tiles(const GemmGeom& g) {
+__device__ __forceinline__ int num_m_tiles(const GemmGeom& g, int cg = 1) {
   if (g.mode == GM_CONV && g.a_tiled)
     return ((g.OW + g.bx - 1) / g.bx) * ((g.OH + g.by - 1) / g.by) * ((g.Nimg + g.bn - 1) / g.bn);
-  return (g.M + BM - 1) / BM;
+  return (g.M + BM * cg - 1) / (BM * cg);
 }
 
 // ---------------------------------------------------------------- the kernel
-template <int BN, bool BF16>
+template <int BN, bool BF16, int CG>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const GemmGeom g, const float* __restrict__ bias, void* __restrict__ Y) {
-  using C = Cfg<BN>;
+  using C = Cfg<BN, CG>;
+  // cta_group::2: a CTA pair computes a (2*128) x BN tile; rank 0 (leader) issues the MMAs.
+  const uint32_t rank = CG == 2 ? cluster_rank() : 0;
+  const int cid = blockIdx.x / CG, ncl = gridDim.x / CG;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
@@ -308,9 +384,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                      st_epi_work = 0;
   const unsigned long long st_begin = clock64();
 #endif
-  const int mt = num_m_tiles(g), nt = (g.N + BN - 1) / BN, zt = g.Z / g.zf;
+  const int mt = num_m_tiles(g, CG), nt = (g.N + BN - 1) / BN, zt = g.Z / g.zf;
   const int tiles = mt * nt * zt;
-  const int slot_cols = g.zf * BN;
+  int slot_cols = 32;  // TMEM columns per accumulator slot (power of two >= zf*BN)
+  while (slot_cols < g.zf * BN) slot_cols <<= 1;
   const int nslots = 2 * slot_cols <= 512 ? 2 : 1;
   int tcols = 32;
   while (tcols < nslots * slot_cols) tcols <<= 1;
@@ -322,7 +399,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     }
     for (int s = 0; s < 2; ++s) {
       mbar_init(tfull0 + 8 * s, 1);
-      mbar_init(tempty0 + 8 * s, EPI_WARPS);
+      mbar_init(tempty0 + 8 * s, EPI_WARPS * CG);  // leader's: both CTAs' epilogues arrive
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     fence_proxy_async();
@@ -330,13 +407,21 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmB) : "memory");
   }
   if (warp == MMA_WARP) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                 "r"((uint32_t)tcols)
-                 : "memory");
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    if (CG == 2) {
+      asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                   "r"((uint32_t)tcols)
+                   : "memory");
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+    } else {
+      asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                   "r"((uint32_t)tcols)
+                   : "memory");
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
   }
   tc_fence_before();
   __syncthreads();
+  if (CG == 2) cluster_sync();  // peer barriers initialised before any remote arrive / TMA tx
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
@@ -349,13 +434,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       const int nchunks_k = g.K / cw;  // valid chunks along K
       const int oy_per = g.OH * g.OWb;
       int it = 0;
-      for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
-        const TileCoord tc = tile_coord(g, t, mt, nt);
+      for (int t = cid; t < tiles; t += ncl) {
+        const TileCoord tc = tile_coord(g, t, mt, nt, CG);
+        const int my_m0 = tc.m0 + (int)rank * BM;  // this CTA's 128 rows of the pair tile
         // conv: top-left input pixel of the filter window of the tile's first output pixel
         int wx = tc.x0 * g.stride - g.pad, wy = tc.y0 * g.stride - g.pad, img = tc.i0;
         if (g.mode == GM_CONV && !g.a_tiled) {
-          img = tc.m0 / oy_per;
-          const int rem = tc.m0 - img * oy_per;
+          img = my_m0 / oy_per;
+          const int rem = my_m0 - img * oy_per;
           const int oy = rem / g.OWb;
           wy = oy * g.stride - g.pad;
           wx = (rem - oy * g.OWb) * (g.xb > 1 ? g.xb : g.stride) - g.pad;
@@ -379,23 +465,23 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
               STAT_ADD(st_prod_wait);
             }
             const uint32_t fb = full0 + 8 * s;
-            mbar_arrive_expect_tx(fb, C::A_BYTES + C::B_BYTES);
+            if (rank == 0) mbar_arrive_expect_tx(fb, CG * (C::A_BYTES + C::B_BYTES));
             const uint32_t a_dst = smem_u32(sA + s * C::A_BYTES);
             if (g.mode == GM_DENSE) {
-              tma_2d(a_dst, &tmA, fb, kb * BK, tc.m0);
+              tma_a2<CG>(a_dst, &tmA, fb, kb * BK, my_m0);
             } else {
               for (int j = 0; j < chunks_per_kb; ++j, ++q) {
                 // past the valid K: a channel coordinate beyond the extent -> TMA zero-fills
                 const int c = q < nchunks_k ? cbase + cc : g.Cp_in;
                 const uint32_t dst = a_dst + j * cbytes;
                 if (g.mode == GM_CONV) {
-                  if (g.a_tiled) tma_4d(dst, &tmA, fb, c, wx + kx, wy + ky, img);
-                  else tma_im2col_4d(dst, &tmA, fb, c, wx, wy, img, (uint16_t)(kx * g.kxs), (uint16_t)ky);
+                  if (g.a_tiled) tma_a4<CG>(dst, &tmA, fb, c, wx + kx, wy + ky, img);
+                  else tma_i2c<CG>(dst, &tmA, fb, c, wx, wy, img, (uint16_t)(kx * g.kxs), (uint16_t)ky);
                 } else if (g.lcg > 1) {  // LC, lcg taps per row: 3D view {W*C, H, N}
                   const int xe = q < nchunks_k ? (lcx + kx) * g.Cp_in : g.W * g.Cp_in;  // K tail: OOB
-                  tma_3d(dst, &tmA, fb, xe, lcy + ky, tc.m0);
+                  tma_a3<CG>(dst, &tmA, fb, xe, lcy + ky, my_m0);
                 } else {  // LC: rows are images at the fixed output location z
-                  tma_4d(dst, &tmA, fb, c, lcx + kx, lcy + ky, tc.m0);
+                  tma_a4<CG>(dst, &tmA, fb, c, lcx + kx, lcy + ky, my_m0);
                 }
                 if (g.lcg > 1) {
                   kx += g.lcg;
@@ -409,18 +495,29 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 }
               }
             }
-            tma_3d(smem_u32(sB + s * C::B_BYTES), &tmB, fb, kb * BK, tc.n0 * BN, z);
+            tma_a3<CG>(smem_u32(sB + s * C::B_BYTES), &tmB, fb, kb * BK, tc.n0 * BN + (int)rank * (BN / CG), z);
           }
         }
       }
     }
     __syncwarp();
   } else if (warp == MMA_WARP) {
-    if (lane == 0) {
-      const uint32_t idesc = idesc_f16<BN, BF16>();
+    if (lane == 0 && rank == 0) {
+      const uint32_t idesc = idesc_f16<BN, BF16, CG>();
       const int cw = g.mode == GM_DENSE ? 64 : g.cw, cbytes = BM * cw * 2;
+      // Everything that does not change per k-block is hoisted: the single issuing thread's
+      // instruction latency (not the tensor core) bounded N <= 128 MMAs at ~77+ cycles each.
+      // A descriptor of stage s, step k = (desc of the stage base) + adelta[k] (16-byte units).
+      uint32_t adelta[BK / 16];
+#pragma unroll
+      for (int k = 0; k < BK / 16; ++k) {
+        const int e = k * 16;
+        adelta[k] = (uint32_t)(((e / cw) * cbytes + (e % cw) * 2) >> 4);
+      }
+      const uint64_t a_hi = sdesc(0, cw * 2), b_hi = sdesc(0, 128);
+      const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
       int it = 0, lt = 0;
-      for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++lt) {
+      for (int t = cid; t < tiles; t += ncl, ++lt) {
         const int slot = nslots == 2 ? (lt & 1) : 0;
         const uint32_t use = nslots == 2 ? (uint32_t)(lt >> 1) : (uint32_t)lt;
         {
@@ -441,19 +538,20 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             }
             tc_fence_after();
             STAT_T0();
-            const uint32_t a0 = smem_u32(sA + s * C::A_BYTES);
-            const uint64_t bd = sdesc(smem_u32(sB + s * C::B_BYTES), 128);
+            const uint64_t ad = a_hi | (uint64_t)(((sA0 + s * C::A_BYTES) & 0x3FFFFu) >> 4);
+            const uint64_t bd = b_hi | (uint64_t)(((sB0 + s * C::B_BYTES) & 0x3FFFFu) >> 4);
 #pragma unroll
             for (int k = 0; k < BK / 16; ++k) {
-              const int e = k * 16;  // element offset of this K step inside the stage
-              const uint64_t ad = sdesc(a0 + (e / cw) * cbytes + (e % cw) * 2, cw * 2);
-              mma_f16(d, ad, bd + 2 * k, idesc, (kb | k) != 0);
+              if (CG == 2) mma_f16_2sm(d, ad + adelta[k], bd + 2 * k, idesc, (kb | k) != 0);
+              else mma_f16(d, ad + adelta[k], bd + 2 * k, idesc, (kb | k) != 0);
             }
-            mma_commit(empty0 + 8 * s);
+            if (CG == 2) mma_commit_2sm(empty0 + 8 * s);
+            else mma_commit(empty0 + 8 * s);
             STAT_ADD(st_mma_issue);
           }
         }
-        mma_commit(tfull0 + 8 * slot);
+        if (CG == 2) mma_commit_2sm(tfull0 + 8 * slot);
+        else mma_commit(tfull0 + 8 * slot);
       }
     }
     __syncwarp();
@@ -462,8 +560,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const int quarter = warp & 3, half = warp >> 2;
     int lt = 0;
     const uint32_t lane_base = (uint32_t)(quarter * 32) << 16;
-    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++lt) {
-      const TileCoord tc = tile_coord(g, t, mt, nt);
+    for (int t = cid; t < tiles; t += ncl, ++lt) {
+      TileCoord tc = tile_coord(g, t, mt, nt, CG);
+      tc.m0 += (int)rank * BM;  // this CTA's rows of the pair tile
       const int slot = nslots == 2 ? (lt & 1) : 0;
       const uint32_t use = nslots == 2 ? (uint32_t)(lt >> 1) : (uint32_t)lt;
       const int r = quarter * 32 + lane;
@@ -632,7 +731,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       STAT_ADD(st_epi_work);
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(tempty0 + 8 * slot);
+      if (lane == 0) {
+        if (CG == 2) mbar_arrive_leader(tempty0 + 8 * slot);
+        else mbar_arrive(tempty0 + 8 * slot);
+      }
     }
   }
 #ifdef DJINN_TC_STATS
@@ -644,20 +746,24 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 #endif
   tc_fence_before();
   __syncthreads();
+  if (CG == 2) cluster_sync();  // no remote arrive / commit may target a finished peer
   if (warp == MMA_WARP) {
     tc_fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"((uint32_t)tcols) : "memory");
+    if (CG == 2)
+      asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"((uint32_t)tcols) : "memory");
+    else
+      asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"((uint32_t)tcols) : "memory");
   }
 }
 
 int g_num_sms = 0;
 
-template <int BN, bool BF16>
+template <int BN, bool BF16, int CG>
 cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtensorMap* tmB, const float* bias, void* Y,
                         cudaStream_t st) {
-  using C = Cfg<BN>;
+  using C = Cfg<BN, CG>;
   static bool attr_set = false;  // benign race: idempotent attribute set
-  auto kern = tc_gemm_kernel<BN, BF16>;
+  auto kern = tc_gemm_kernel<BN, BF16, CG>;
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
     if (e != cudaSuccess) return e;
@@ -665,23 +771,46 @@ cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtenso
   }
   const int64_t mtiles = (g.mode == GM_CONV && g.a_tiled)
                              ? (int64_t)((g.OW + g.bx - 1) / g.bx) * ((g.OH + g.by - 1) / g.by) *
-                                                  ((g.Nimg + g.bn - 1) / g.bn)
-                                            : (g.M + BM - 1) / BM;
+                                   ((g.Nimg + g.bn - 1) / g.bn)
+                             : (g.M + BM * CG - 1) / (BM * CG);
   const int64_t tiles = mtiles * ((g.N + BN - 1) / BN) * (g.Z / g.zf);
-  const int grid = (int)(tiles < tc_num_sms() ? tiles : tc_num_sms());
-  kern<<<grid, NUM_THREADS, C::SMEM, st>>>(*tmA, *tmB, g, bias, Y);
-  return cudaGetLastError();
+  const int max_cl = tc_num_sms() / CG;
+  const int clusters = (int)(tiles < max_cl ? tiles : max_cl);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(clusters * CG);
+  cfg.blockDim = dim3(NUM_THREADS);
+  cfg.dynamicSmemBytes = C::SMEM;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = CG;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, *tmA, *tmB, g, bias, Y);
 }
 
 template <bool BF16>
 cudaError_t launch_bn(const GemmGeom& g, int bn, const CUtensorMap* tmA, const CUtensorMap* tmB, const float* bias,
                       void* Y, cudaStream_t st) {
+  if (g.cg == 2) {
+    switch (bn) {
+      case 96: return launch_inst<96, BF16, 2>(g, tmA, tmB, bias, Y, st);
+      case 128: return launch_inst<128, BF16, 2>(g, tmA, tmB, bias, Y, st);
+      case 192: return launch_inst<192, BF16, 2>(g, tmA, tmB, bias, Y, st);
+      case 256: return launch_inst<256, BF16, 2>(g, tmA, tmB, bias, Y, st);
+      default: return cudaErrorInvalidValue;
+    }
+  }
   switch (bn) {
-    case 16: return launch_inst<16, BF16>(g, tmA, tmB, bias, Y, st);
-    case 32: return launch_inst<32, BF16>(g, tmA, tmB, bias, Y, st);
-    case 64: return launch_inst<64, BF16>(g, tmA, tmB, bias, Y, st);
-    case 128: return launch_inst<128, BF16>(g, tmA, tmB, bias, Y, st);
-    case 256: return launch_inst<256, BF16>(g, tmA, tmB, bias, Y, st);
+    case 16: return launch_inst<16, BF16, 1>(g, tmA, tmB, bias, Y, st);
+    case 32: return launch_inst<32, BF16, 1>(g, tmA, tmB, bias, Y, st);
+    case 64: return launch_inst<64, BF16, 1>(g, tmA, tmB, bias, Y, st);
+    case 96: return launch_inst<96, BF16, 1>(g, tmA, tmB, bias, Y, st);
+    case 128: return launch_inst<128, BF16, 1>(g, tmA, tmB, bias, Y, st);
+    case 192: return launch_inst<192, BF16, 1>(g, tmA, tmB, bias, Y, st);
+    case 256: return launch_inst<256, BF16, 1>(g, tmA, tmB, bias, Y, st);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -699,13 +828,24 @@ int tc_num_sms() {
   return g_num_sms;
 }
 
+int tc_pick_cg(const GemmGeom& g, int bn) {
+  const char* e = getenv("DJINN_CTA_PAIR");
+  if (e && e[0] == '0') return 1;
+  if (bn < 96 || (g.mode == GM_CONV && g.a_tiled)) return 1;
+  return 2;
+}
+
 int tc_pick_bn(const GemmGeom& g) {
   const int n = g.N;
   if (n <= 16) return 16;
   if (n <= 32) return 32;
   if (n <= 64) return 64;
+  if (n <= 96) return 96;
   if (n <= 128) return 128;
-  return 256;
+  if (n <= 192) return 192;
+  // wider N: the tile (192 or 256) with the least padding, ties to the larger
+  // 192 only when it needs no more tiles than 256 (e.g. N = 384); otherwise bigger tiles win
+  return (n + 191) / 192 <= (n + 255) / 256 ? 192 : 256;
 }
 
 cudaError_t launch_tc_gemm(const GemmGeom& g, int bn, int dt, const CUtensorMap* tmA, const CUtensorMap* tmB,

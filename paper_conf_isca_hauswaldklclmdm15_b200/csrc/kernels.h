@@ -50,6 +50,7 @@ struct GemmGeom {
   int Co;             // real output channels (x-blocked conv: per dx)
   int lcg, kwp;       // LC: taps per TMA row (box {Cgp, lcg, 1, 128}) and KW padded to lcg
   int kxs;            // conv: x offset between consecutive taps (x-unrolled input: xu), default 1
+  int cg;             // 1: one CTA per 128-row tile; 2: cta_group::2 CTA pair per 256-row tile (B split)
   int a_tiled;        // conv: 0 = im2col-mode TMA over linear output pixels (default), 1 = tiled
                       //       4D boxes over bx x by x bn pixel blocks (DJINN_CONV_A=tiled)
   int bx, by, bn;     // conv: output-pixel block of one M tile (bx*by*bn == 128), x fastest
@@ -79,6 +80,7 @@ cudaError_t launch_simt_gemm(const GemmGeom& g, const float* A, const float* B, 
 //      dense-> 2D tiled map over [rows][a_pitch], box {64, 128}.
 // Swizzle of A boxes: cw*2 bytes (32B / 64B / 128B).
 int tc_pick_bn(const GemmGeom& g);
+int tc_pick_cg(const GemmGeom& g, int bn);  // 2 when a CTA pair (cta_group::2) pays off
 int tc_num_sms();
 cudaError_t launch_tc_gemm(const GemmGeom& g, int bn, int dt, const CUtensorMap* tmA,
                            const CUtensorMap* tmB, const float* bias, void* Y, cudaStream_t st);

@@ -917,7 +917,7 @@ std::string Net::plan_string() const {
       << o.out_buf;
     if (o.kind == OP_GEMM)
       s << " [" << modes[o.g.mode] << " N=" << o.g.N << " Z=" << o.g.Z << " K=" << o.g.K << " Kpad=" << o.g.Kpad
-        << " act=" << o.g.act << " bn=" << o.bn << " cw=" << o.g.cw << " zf=" << o.g.zf << " KHxKW=" << o.g.KH << "x"
+        << " act=" << o.g.act << " bn=" << o.bn << " cg=" << o.g.cg << " cw=" << o.g.cw << " zf=" << o.g.zf << " KHxKW=" << o.g.KH << "x"
         << o.g.KW << (o.g.xb > 1 ? " xblock=" + std::to_string(o.g.xb) : std::string())
         << (o.g.kxs > 1 ? " x-unrolled-input=" + std::to_string(o.g.kxs) : std::string())
         << (o.g.lcg > 1 ? " taps/row=" + std::to_string(o.g.lcg) : std::string())
