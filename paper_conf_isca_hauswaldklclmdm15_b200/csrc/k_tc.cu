@@ -46,7 +46,7 @@ namespace djinn {
 namespace {
 
 constexpr int BM = 128, BK = 64;
-constexpr int EPI_WARPS = 8, TMA_WARP = 8, MMA_WARP = 9, NUM_THREADS = 320;
+constexpr int EPI_WARPS = 8, TMA_WARP = 8, MMA_WARP = 9, TMAB_WARP = 10, NUM_THREADS = 352;
 
 template <int BN, int CG = 1>
 struct Cfg {
@@ -393,6 +393,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   while (tcols < nslots * slot_cols) tcols <<= 1;
 
   if (warp == TMA_WARP && lane == 0) {
+    // (barriers are initialised before the __syncthreads below; the B producer, warp 10,
+    // starts after it)
     for (int s = 0; s < C::STAGES; ++s) {
       mbar_init(full0 + 8 * s, 1);
       mbar_init(empty0 + 8 * s, 1);
@@ -495,7 +497,25 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 }
               }
             }
-            tma_a3<CG>(smem_u32(sB + s * C::B_BYTES), &tmB, fb, kb * BK, tc.n0 * BN + (int)rank * (BN / CG), z);
+          }
+        }
+      }
+    }
+    __syncwarp();
+  } else if (warp == TMAB_WARP) {
+    // B (weights) producer: a second issuing thread so the A and B TMA streams overlap (one
+    // thread issuing both serialised on TMA-instruction latency).  The expect-tx of the stage
+    // (both operands) is armed by the A producer; tx may complete before it is armed.
+    if (lane == 0) {
+      int it = 0;
+      for (int t = cid; t < tiles; t += ncl) {
+        const TileCoord tc = tile_coord(g, t, mt, nt, CG);
+        for (int zi = 0; zi < g.zf; ++zi) {
+          const int z = tc.z0 * g.zf + zi;
+          for (int kb = 0; kb < num_kb; ++kb, ++it) {
+            const int s = it % C::STAGES;
+            mbar_wait(empty0 + 8 * s, ((it / C::STAGES) & 1) ^ 1);
+            tma_a3<CG>(smem_u32(sB + s * C::B_BYTES), &tmB, full0 + 8 * s, kb * BK, tc.n0 * BN + (int)rank * (BN / CG), z);
           }
         }
       }
@@ -555,7 +575,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       }
     }
     __syncwarp();
-  } else {
+  } else if (warp < EPI_WARPS) {
     // ---- epilogue (warps 0-7): TMEM -> registers -> bias + act (+ LRN) -> global ----
     const int quarter = warp & 3, half = warp >> 2;
     int lt = 0;
