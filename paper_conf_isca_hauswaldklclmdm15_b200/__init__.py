@@ -28,7 +28,7 @@ PRECISION = {"fp32": DJINN_FP32, "bf16": DJINN_BF16, "fp16": DJINN_FP16}
 EXPORTS = ["djinn_load_net", "djinn_forward", "djinn_sync", "djinn_free", "djinn_net_info",
            "djinn_weight_arena", "djinn_plan_info", "djinn_profile", "djinn_profile_read", "djinn_op_info",
            "djinn_describe", "djinn_last_error", "djinn_kernel_launches"]
-OP_KINDS = ["pack", "gemm", "lrn", "pool", "softmax"]
+OP_KINDS = ["pack", "gemm", "lrn", "pool", "softmax", "lrn+pool"]
 
 
 class DjinnError(RuntimeError):

@@ -16,7 +16,7 @@ SOURCES = ["api.cu", "net.cu", "k_misc.cu", "k_simt.cu", "k_tc.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "-I", os.path.join(ROOT, "include")] + \
-        (["-DDJINN_TC_STATS"] if VARIANT == "stats" else [])
+        (["-DDJINN_TC_STATS"] if VARIANT == "stats" else []) + os.environ.get("DJINN_EXTRA_FLAGS", "").split()
 HEADERS = [os.path.join(CSRC, h) for h in os.listdir(CSRC) if h.endswith((".h", ".cuh"))] + \
           [os.path.join(ROOT, "include", "djinn.h")]
 

@@ -236,6 +236,88 @@ cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, in
 }
 
 // ------------------------------------------------------------------------------------------
+// K4+K5 fused: y = maxpool(LRN(x)).  One thread per (output pixel, 8-channel chunk of the output
+// layout); for every pixel of the pooling window it loads the 8 channels plus the neighbouring
+// chunks (the LRN window needs c-2 .. c+2), evaluates Caffe's LRN in fp32 and keeps the max.
+// The conv before it stores its ReLU output in fp16, so LRN's input keeps
+// 11 mantissa bits on the bf16 path too.
+template <typename TO>
+__global__ void lrn_pool_kernel(const __half* __restrict__ x, TO* __restrict__ y, int64_t rows, int C, int Cpi, int H,
+                                int W, int OH, int OW, int kern, int stride, int pad, int gsz, int gpitch, int Cpo,
+                                float an, float nbeta, float k) {
+  const int chunks = Cpo / 8;
+  const int per_row = OH * OW * chunks;
+  for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
+    const __half* xr = x + r * (int64_t)H * W * Cpi;
+    TO* yr = y + r * (int64_t)OH * OW * Cpo;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < per_row; i += gridDim.x * blockDim.x) {
+      const int p8 = i % chunks, pix = i / chunks;
+      const int pos = p8 * 8, grp = pos / gpitch, within = pos - grp * gpitch;
+      const int c0 = grp * gsz + within;  // logical channel of this output chunk
+      __align__(16) TO o[8];
+      if (within >= gsz || c0 >= C) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) o[j] = cvt<TO>(0.f);
+        *reinterpret_cast<uint4*>(yr + (int64_t)pix * Cpo + pos) = *reinterpret_cast<const uint4*>(o);
+        continue;
+      }
+      const int oy = pix / OW, ox = pix - (pix / OW) * OW;
+      int hs = oy * stride - pad, ws = ox * stride - pad;
+      int he = min(hs + kern, H + pad), we = min(ws + kern, W + pad);
+      hs = max(hs, 0); ws = max(ws, 0); he = min(he, H); we = min(we, W);
+      float acc[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) acc[j] = -FLT_MAX;
+      for (int h = hs; h < he; ++h)
+        for (int w = ws; w < we; ++w) {
+          const __half* px = xr + ((int64_t)h * W + w) * Cpi + c0;
+          float v[24];
+          const uint4 uc = __ldg(reinterpret_cast<const uint4*>(px));
+          const uint4 up = c0 >= 8 ? __ldg(reinterpret_cast<const uint4*>(px - 8)) : make_uint4(0, 0, 0, 0);
+          const uint4 un = c0 + 8 < C ? __ldg(reinterpret_cast<const uint4*>(px + 8)) : make_uint4(0, 0, 0, 0);
+          const __half* hp = reinterpret_cast<const __half*>(&up);
+          const __half* hc = reinterpret_cast<const __half*>(&uc);
+          const __half* hn = reinterpret_cast<const __half*>(&un);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            v[j] = __half2float(hp[j]);
+            v[8 + j] = __half2float(hc[j]);
+            v[16 + j] = __half2float(hn[j]);
+          }
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            const float s5 = (v[6 + j] * v[6 + j] + v[7 + j] * v[7 + j]) + (v[8 + j] * v[8 + j] + v[9 + j] * v[9 + j]) +
+                             v[10 + j] * v[10 + j];
+            const float l = v[8 + j] * exp2f(nbeta * __log2f(fmaf(an, s5, k)));
+            acc[j] = fmaxf(acc[j], l);
+          }
+        }
+#pragma unroll
+      for (int j = 0; j < 8; ++j) o[j] = cvt<TO>(acc[j]);
+      *reinterpret_cast<uint4*>(yr + (int64_t)pix * Cpo + pos) = *reinterpret_cast<const uint4*>(o);
+    }
+  }
+}
+
+cudaError_t launch_lrn_pool(const void* x, void* y, int64_t rows, int C, int Cpi, int H, int W, int OH, int OW,
+                            int kernel, int stride, int pad, int out_gsz, int out_gpitch, int Cpo, int size,
+                            float alpha, float beta, float k, int dt, cudaStream_t st) {
+  if (size != 5 || C % 8 || Cpi % 8 || Cpo % 8) return cudaErrorInvalidValue;
+  if (out_gsz > C) { out_gsz = C; out_gpitch = Cpo; }
+  if (out_gsz % 8 || out_gpitch % 8) return cudaErrorInvalidValue;
+  const int per_row = OH * OW * (Cpo / 8);
+  dim3 g(min(nblocks(per_row, 256), 1024), (unsigned)(rows < 65535 ? rows : 65535));
+  const float an = alpha / size;
+  if (dt == DT_F16)
+    lrn_pool_kernel<__half><<<g, 256, 0, st>>>((const __half*)x, (__half*)y, rows, C, Cpi, H, W, OH, OW, kernel, stride,
+                                               pad, out_gsz, out_gpitch, Cpo, an, -beta, k);
+  else
+    lrn_pool_kernel<__nv_bfloat16><<<g, 256, 0, st>>>((const __half*)x, (__nv_bfloat16*)y, rows, C, Cpi, H, W, OH, OW,
+                                                      kernel, stride, pad, out_gsz, out_gpitch, Cpo, an, -beta, k);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------
 // K5: Caffe pooling (MAX / AVE), ceil geometry; window clipped to the image, AVE divisor is
 // the window area clipped to H+pad but not to the image.
 template <typename T>

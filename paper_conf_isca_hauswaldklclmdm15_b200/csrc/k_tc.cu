@@ -48,6 +48,7 @@ namespace {
 constexpr int BM = 128, BK = 64;
 constexpr int EPI_WARPS = 8, TMA_WARP = 8, MMA_WARP = 9, TMAB_WARP = 10, NUM_THREADS = 352;
 
+constexpr int KTAB_MAX = 256;  // im2col producer: per-K-chunk (channel, kx, ky) table entries
 template <int BN, int CG = 1>
 struct Cfg {
   static constexpr int A_BYTES = BM * BK * 2;
@@ -116,6 +117,11 @@ __device__ __forceinline__ void tma_im2col_4d(uint32_t dst, const CUtensorMap* m
 // transaction bytes land on the LEADER's (rank 0) barrier: its shared::cluster address is the
 // local one with the peer bit (bit 24) cleared.
 constexpr uint32_t PEER_MASK = 0xFEFFFFFFu;
+__device__ __forceinline__ bool elect_one() {
+  uint32_t p;
+  asm volatile("{\n\t.reg .pred P;\n\telect.sync _|P, 0xffffffff;\n\tselp.u32 %0, 1, 0, P;\n\t}" : "=r"(p));
+  return p != 0;
+}
 __device__ __forceinline__ uint32_t cluster_rank() {
   uint32_t r;
   asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
@@ -148,8 +154,15 @@ __device__ __forceinline__ void tma_im2col_4d_2sm(uint32_t dst, const CUtensorMa
       ::"r"(dst), "l"((uint64_t)map), "r"(bar & PEER_MASK), "r"(c), "r"(w), "r"(h), "r"(n), "h"(ox), "h"(oy)
       : "memory");
 }
+// Relaxed arrives for the TMEM-empty handshake: TMEM reuse is ordered by tcgen05.wait::ld +
+// tcgen05.fence::before_thread_sync, and no generic memory needs to be published, so the
+// .release form (MEMBAR.ALL.CTA + ERRBAR: the epilogue waited for its global stores to drain,
+// ~24% of stall samples) is not needed.
 __device__ __forceinline__ void mbar_arrive_leader(uint32_t bar) {
-  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(bar & PEER_MASK) : "memory");
+  asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(bar & PEER_MASK) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_relaxed(uint32_t bar) {
+  asm volatile("mbarrier.arrive.relaxed.cta.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
 template <int CG>
 __device__ __forceinline__ void tma_a2(uint32_t dst, const CUtensorMap* m, uint32_t bar, int c0, int c1) {
@@ -295,8 +308,29 @@ __device__ __forceinline__ uint32_t pack2(float a, float b) {
   }
 }
 
+// Diagnostic builds only (tools/): DJINN_DBG_NOSTORE drops the epilogue's
+// global stores, DJINN_DBG_NOEPI skips the epilogue work (TMEM slots are released at once).
+#ifdef DJINN_DBG_NOEPI
+constexpr bool kDbgNoEpi = true;
+#else
+constexpr bool kDbgNoEpi = false;
+#endif
+#ifdef DJINN_DBG_NOB
+constexpr bool kDbgNoB = true;  // DJINN_DBG_NOB: the B operand is not loaded
+#else
+constexpr bool kDbgNoB = false;
+#endif
+#ifdef DJINN_DBG_NOMMA
+constexpr bool kDbgNoMma = true;  // DJINN_DBG_NOMMA: operands stream, no MMA is issued
+#else
+constexpr bool kDbgNoMma = false;
+#endif
+
 template <bool BF16>
 __device__ __forceinline__ void store16(const GemmGeom& g, void* Y, int64_t off, const float (&v)[16], int nvalid8) {
+#ifdef DJINN_DBG_NOSTORE
+  if (v[0] != 12345.f) return;
+#endif
   if (g.out_f32) {
     float* yp = reinterpret_cast<float*>(Y) + off;
 #pragma unroll
@@ -305,6 +339,14 @@ __device__ __forceinline__ void store16(const GemmGeom& g, void* Y, int64_t off,
         reinterpret_cast<float4*>(yp + 8 * h)[0] = make_float4(v[8 * h], v[8 * h + 1], v[8 * h + 2], v[8 * h + 3]);
         reinterpret_cast<float4*>(yp + 8 * h)[1] = make_float4(v[8 * h + 4], v[8 * h + 5], v[8 * h + 6], v[8 * h + 7]);
       }
+  } else if (BF16 && g.out_half) {
+    uint16_t* yp = reinterpret_cast<uint16_t*>(Y) + off;
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+      if (h < nvalid8)
+        *reinterpret_cast<uint4*>(yp + 8 * h) =
+            make_uint4(pack2<false>(v[8 * h], v[8 * h + 1]), pack2<false>(v[8 * h + 2], v[8 * h + 3]),
+                       pack2<false>(v[8 * h + 4], v[8 * h + 5]), pack2<false>(v[8 * h + 6], v[8 * h + 7]));
   } else {
     uint16_t* yp = reinterpret_cast<uint16_t*>(Y) + off;
 #pragma unroll
@@ -352,6 +394,13 @@ __device__ __forceinline__ TileCoord tile_coord(const GemmGeom& g, int t, int mt
   }
   return c;
 }
+// Broadcast lane 0's copy: the values are warp-uniform already; this tells ptxas so.
+__device__ __forceinline__ int warp_uniform(int v) { return __shfl_sync(0xffffffffu, v, 0); }
+__device__ __forceinline__ TileCoord warp_uniform(TileCoord c) {
+  c.m0 = warp_uniform(c.m0); c.n0 = warp_uniform(c.n0); c.z0 = warp_uniform(c.z0);
+  c.x0 = warp_uniform(c.x0); c.y0 = warp_uniform(c.y0); c.i0 = warp_uniform(c.i0);
+  return c;
+}
 __device__ __forceinline__ int num_m_tiles(const GemmGeom& g, int cg = 1) {
   if (g.mode == GM_CONV && g.a_tiled)
     return ((g.OW + g.bx - 1) / g.bx) * ((g.OH + g.by - 1) / g.by) * ((g.Nimg + g.bn - 1) / g.bn);
@@ -374,13 +423,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   uint64_t* bars = reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
   // bars: full[STAGES], empty[STAGES], tfull[2], tempty[2]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * C::STAGES + 4);
+  __shared__ uint32_t ktab[KTAB_MAX];
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + C::STAGES);
   const uint32_t tfull0 = smem_u32(bars + 2 * C::STAGES), tempty0 = smem_u32(bars + 2 * C::STAGES + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int num_kb = g.Kpad / BK;
 #ifdef DJINN_TC_STATS
-  unsigned long long st_prod_wait = 0, st_mma_full = 0, st_mma_tempty = 0, st_mma_issue = 0, st_epi_wait = 0,
+  unsigned long long st_prod_wait = 0, st_prod_issue = 0, st_mma_full = 0, st_mma_tempty = 0, st_mma_issue = 0, st_epi_wait = 0,
                      st_epi_work = 0;
   const unsigned long long st_begin = clock64();
 #endif
@@ -428,105 +478,188 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   const uint32_t tmem = *tmem_slot;
 
   if (warp == TMA_WARP) {
-    if (lane == 0) {
-      // Division-free address generation: the (ky, kx, c) of each K chunk is advanced with
-      // counters (integer division on the single issuing thread throttled the TMA stream).
-      const int cw = g.cw, cbytes = BM * cw * 2;
-      const int chunks_per_kb = BK / cw;
-      const int nchunks_k = g.K / cw;  // valid chunks along K
-      const int oy_per = g.OH * g.OWb;
-      int it = 0;
-      for (int t = cid; t < tiles; t += ncl) {
-        const TileCoord tc = tile_coord(g, t, mt, nt, CG);
-        const int my_m0 = tc.m0 + (int)rank * BM;  // this CTA's 128 rows of the pair tile
-        // conv: top-left input pixel of the filter window of the tile's first output pixel
-        int wx = tc.x0 * g.stride - g.pad, wy = tc.y0 * g.stride - g.pad, img = tc.i0;
-        if (g.mode == GM_CONV && !g.a_tiled) {
-          img = my_m0 / oy_per;
-          const int rem = my_m0 - img * oy_per;
-          const int oy = rem / g.OWb;
-          wy = oy * g.stride - g.pad;
-          wx = (rem - oy * g.OWb) * (g.xb > 1 ? g.xb : g.stride) - g.pad;
+    // A producer.  The whole warp runs the loop (warp-uniform values stay in uniform
+    // registers), one elected lane issues; (ky, kx, c) of each K chunk advance by counters
+    // (no division).  The single-lane version spent ~900 cycles of dependent instructions
+    // per stage, which capped the operand stream at ~20 B/cycle/SM.
+    const int cw = g.cw, cbytes = BM * cw * 2;
+    const int chunks_per_kb = BK / cw;
+    const int nchunks_k = g.K / cw;  // valid chunks along K
+    const int oy_per = g.OH * g.OWb;
+    const int mode = g.mode, a_tiled = g.a_tiled, lcg = g.lcg, kwp = g.kwp, KW = g.KW, Cgp = g.Cgp, kxs = g.kxs;
+    const int Cp_in = g.Cp_in, zf = g.zf;
+    const uint32_t sA0 = smem_u32(sA);
+    const bool leader = elect_one();
+    int s = 0;
+    uint32_t ph = 0;
+    const int nq = num_kb * chunks_per_kb;
+    if (mode == GM_CONV && !a_tiled && nq <= KTAB_MAX) {
+      // im2col fast path: the (channel, kx, ky) of every K chunk comes from a table built
+      // once, so a stage costs a handful of instructions (the issuing warp's instruction
+      // latency, not the TMA unit, had bounded the operand stream: DESIGN.md sec 5).
+      const int cpt = Cgp / cw;  // chunks per tap
+      for (int qq = lane; qq < nq; qq += 32) {
+        uint32_t e = 0xFFFFu;  // past the valid K: channel = Cp_in (TMA zero-fills)
+        if (qq < nchunks_k) {
+          const int tap = qq / cpt, kx = tap % KW, ky = tap / KW;
+          e = (uint32_t)((qq - tap * cpt) * cw) | ((uint32_t)(kx * kxs) << 16) | ((uint32_t)ky << 24);
         }
-        for (int zi = 0; zi < g.zf; ++zi) {
-          const int z = tc.z0 * g.zf + zi;
-          int lcx = 0, lcy = 0;  // LC: input pixel of the location (block)
-          if (g.mode == GM_LC) {
-            const int oy = z / g.OWb;
-            lcy = oy * g.stride;
-            lcx = (z - oy * g.OWb) * g.xb * g.stride;
-          }
-          const int cbase = g.mode == GM_CONV ? z * g.cin_goff : 0;
-          int cc = 0, kx = 0, ky = 0, q = 0;  // chunk counters: channel offset, tap, chunk index
-          for (int kb = 0; kb < num_kb; ++kb, ++it) {
-            const int s = it % C::STAGES;
-            const uint32_t ph = (it / C::STAGES) & 1;
+        ktab[qq] = e;
+      }
+      __syncwarp();
+      const uint32_t tx_bytes = CG * (C::A_BYTES + (kDbgNoB ? 0 : C::B_BYTES));
+      const int sx = g.xb > 1 ? g.xb : g.stride, OWb = g.OWb, st = g.stride, pd = g.pad, cin_goff = g.cin_goff;
+      for (int t = cid; t < tiles; t += ncl) {
+        const TileCoord tc = warp_uniform(tile_coord(g, t, mt, nt, CG));
+        const int my_m0 = tc.m0 + (int)rank * BM;
+        const int img = warp_uniform(my_m0 / oy_per);
+        const int rem = my_m0 - img * oy_per;
+        const int oy = rem / OWb;
+        const int wy = warp_uniform(oy * st - pd), wx = warp_uniform((rem - oy * OWb) * sx - pd);
+        for (int zi = 0; zi < zf; ++zi) {
+          const int cbase = (tc.z0 * zf + zi) * cin_goff;
+          int q = 0;
+          for (int kb = 0; kb < num_kb; ++kb) {
             {
               STAT_T0();
               mbar_wait(empty0 + 8 * s, ph ^ 1);
               STAT_ADD(st_prod_wait);
             }
+            STAT_T0();
             const uint32_t fb = full0 + 8 * s;
-            if (rank == 0) mbar_arrive_expect_tx(fb, CG * (C::A_BYTES + C::B_BYTES));
-            const uint32_t a_dst = smem_u32(sA + s * C::A_BYTES);
-            if (g.mode == GM_DENSE) {
-              tma_a2<CG>(a_dst, &tmA, fb, kb * BK, my_m0);
-            } else {
-              for (int j = 0; j < chunks_per_kb; ++j, ++q) {
-                // past the valid K: a channel coordinate beyond the extent -> TMA zero-fills
-                const int c = q < nchunks_k ? cbase + cc : g.Cp_in;
-                const uint32_t dst = a_dst + j * cbytes;
-                if (g.mode == GM_CONV) {
-                  if (g.a_tiled) tma_a4<CG>(dst, &tmA, fb, c, wx + kx, wy + ky, img);
-                  else tma_i2c<CG>(dst, &tmA, fb, c, wx, wy, img, (uint16_t)(kx * g.kxs), (uint16_t)ky);
-                } else if (g.lcg > 1) {  // LC, lcg taps per row: 3D view {W*C, H, N}
-                  const int xe = q < nchunks_k ? (lcx + kx) * g.Cp_in : g.W * g.Cp_in;  // K tail: OOB
-                  tma_a3<CG>(dst, &tmA, fb, xe, lcy + ky, my_m0);
-                } else {  // LC: rows are images at the fixed output location z
-                  tma_a4<CG>(dst, &tmA, fb, c, lcx + kx, lcy + ky, my_m0);
-                }
-                if (g.lcg > 1) {
-                  kx += g.lcg;
-                  if (kx >= g.kwp) { kx = 0; ++ky; }
-                } else {
-                  cc += cw;
-                  if (cc == g.Cgp) {
-                    cc = 0;
-                    if (++kx == g.KW) { kx = 0; ++ky; }
+            const uint32_t a_dst = sA0 + (uint32_t)s * C::A_BYTES;
+            if (leader) {
+              if (rank == 0) mbar_arrive_expect_tx(fb, tx_bytes);
+              for (int j = 0; j < chunks_per_kb; ++j) {
+                const uint32_t e = ktab[q + j];
+                const int cr = (int)(e & 0xFFFFu);
+                const int c = cr == 0xFFFF ? Cp_in : cbase + cr;
+                tma_i2c<CG>(a_dst + j * cbytes, &tmA, fb, c, wx, wy, img, (uint16_t)((e >> 16) & 0xFF), (uint16_t)(e >> 24));
+              }
+            }
+            __syncwarp();
+            STAT_ADD(st_prod_issue);
+            q += chunks_per_kb;
+            if (++s == C::STAGES) { s = 0; ph ^= 1; }
+          }
+        }
+      }
+    } else
+    for (int t = cid; t < tiles; t += ncl) {
+      const TileCoord tc = warp_uniform(tile_coord(g, t, mt, nt, CG));
+      const int my_m0 = tc.m0 + (int)rank * BM;  // this CTA's 128 rows of the pair tile
+      // conv: top-left input pixel of the filter window of the tile's first output pixel
+      int wx = tc.x0 * g.stride - g.pad, wy = tc.y0 * g.stride - g.pad, img = tc.i0;
+      if (mode == GM_CONV && !a_tiled) {
+        img = my_m0 / oy_per;
+        const int rem = my_m0 - img * oy_per;
+        const int oy = rem / g.OWb;
+        wy = oy * g.stride - g.pad;
+        wx = (rem - oy * g.OWb) * (g.xb > 1 ? g.xb : g.stride) - g.pad;
+      }
+      // every lane holds the same values; saying so lets ptxas use plain R2UR for the TMA
+      // operands instead of an ELECT/R2UR.BROADCAST waterfall per issue
+      wx = warp_uniform(wx);
+      wy = warp_uniform(wy);
+      img = warp_uniform(img);
+      for (int zi = 0; zi < zf; ++zi) {
+        const int z = tc.z0 * zf + zi;
+        int lcx = 0, lcy = 0;  // LC: input pixel of the location (block)
+        if (mode == GM_LC) {
+          const int oy = z / g.OWb;
+          lcy = warp_uniform(oy * g.stride);
+          lcx = warp_uniform((z - oy * g.OWb) * g.xb * g.stride);
+        }
+        const int cbase = mode == GM_CONV ? z * g.cin_goff : 0;
+        int cc = 0, kx = 0, ky = 0, q = 0;  // chunk counters: channel offset, tap, chunk index
+        for (int kb = 0; kb < num_kb; ++kb) {
+          {
+            STAT_T0();
+            mbar_wait(empty0 + 8 * s, ph ^ 1);
+            STAT_ADD(st_prod_wait);
+          }
+          STAT_T0();
+          const uint32_t fb = full0 + 8 * s;
+          if (leader && rank == 0) mbar_arrive_expect_tx(fb, CG * (C::A_BYTES + (kDbgNoB ? 0 : C::B_BYTES)));
+          const uint32_t a_dst = sA0 + (uint32_t)s * C::A_BYTES;
+          if (mode == GM_DENSE) {
+            if (leader) tma_a2<CG>(a_dst, &tmA, fb, kb * BK, my_m0);
+          } else {
+            for (int j = 0; j < chunks_per_kb; ++j, ++q) {
+              // past the valid K: a channel coordinate beyond the extent -> TMA zero-fills
+              const int c = q < nchunks_k ? cbase + cc : Cp_in;
+              const uint32_t dst = a_dst + j * cbytes;
+              if (mode == GM_CONV) {
+                if (a_tiled) {
+                  if (leader) tma_a4<CG>(dst, &tmA, fb, c, wx + kx, wy + ky, img);
+                } else if (leader) {
+#ifdef DJINN_DBG_WALK
+                  if (g.K == 576 && g.OW == 55) {  // diagnostic: tools/tma_bench2.cu's walk (conv1)
+                    const int m0 = my_m0, per_img = g.OW * g.OH, im = m0 / per_img, rem = m0 - im * per_img;
+                    const int oy = rem / g.OW, ox = rem - oy * g.OW;
+                    tma_i2c<CG>(dst, &tmA, fb, 0, ox, oy, im, (uint16_t)(kb % 3), (uint16_t)(kb / 3));
+                  } else {
+                    tma_i2c<CG>(dst, &tmA, fb, c, wx, wy, img, (uint16_t)(kx * kxs), (uint16_t)ky);
                   }
+#else
+                  tma_i2c<CG>(dst, &tmA, fb, c, wx, wy, img, (uint16_t)(kx * kxs), (uint16_t)ky);
+#endif
+                }
+              } else if (lcg > 1) {  // LC, lcg taps per row: 3D view {W*C, H, N}
+                const int xe = q < nchunks_k ? (lcx + kx) * Cp_in : g.W * Cp_in;  // K tail: OOB
+                if (leader) tma_a3<CG>(dst, &tmA, fb, xe, lcy + ky, my_m0);
+              } else {  // LC: rows are images at the fixed output location z
+                if (leader) tma_a4<CG>(dst, &tmA, fb, c, lcx + kx, lcy + ky, my_m0);
+              }
+              if (lcg > 1) {
+                kx += lcg;
+                if (kx >= kwp) { kx = 0; ++ky; }
+              } else {
+                cc += cw;
+                if (cc == Cgp) {
+                  cc = 0;
+                  if (++kx == KW) { kx = 0; ++ky; }
                 }
               }
             }
           }
+          __syncwarp();
+          STAT_ADD(st_prod_issue);
+          if (++s == C::STAGES) { s = 0; ph ^= 1; }
         }
       }
     }
-    __syncwarp();
   } else if (warp == TMAB_WARP) {
-    // B (weights) producer: a second issuing thread so the A and B TMA streams overlap (one
-    // thread issuing both serialised on TMA-instruction latency).  The expect-tx of the stage
-    // (both operands) is armed by the A producer; tx may complete before it is armed.
-    if (lane == 0) {
-      int it = 0;
+    // B (weights) producer: a second issuing warp so the A and B TMA streams overlap.  The
+    // expect-tx of the stage (both operands) is armed by the A producer; tx may complete
+    // before it is armed.
+    if (!kDbgNoB) {
+      const bool leader = elect_one();
+      const uint32_t sB0 = smem_u32(sB);
+      const int bn_off = (int)rank * (BN / CG);
+      int s = 0;
+      uint32_t ph = 0;
       for (int t = cid; t < tiles; t += ncl) {
-        const TileCoord tc = tile_coord(g, t, mt, nt, CG);
+        const TileCoord tc = warp_uniform(tile_coord(g, t, mt, nt, CG));
         for (int zi = 0; zi < g.zf; ++zi) {
           const int z = tc.z0 * g.zf + zi;
-          for (int kb = 0; kb < num_kb; ++kb, ++it) {
-            const int s = it % C::STAGES;
-            mbar_wait(empty0 + 8 * s, ((it / C::STAGES) & 1) ^ 1);
-            tma_a3<CG>(smem_u32(sB + s * C::B_BYTES), &tmB, full0 + 8 * s, kb * BK, tc.n0 * BN + (int)rank * (BN / CG), z);
+          for (int kb = 0; kb < num_kb; ++kb) {
+            mbar_wait(empty0 + 8 * s, ph ^ 1);
+            if (leader) tma_a3<CG>(sB0 + (uint32_t)s * C::B_BYTES, &tmB, full0 + 8 * s, kb * BK, tc.n0 * BN + bn_off, z);
+            __syncwarp();
+            if (++s == C::STAGES) { s = 0; ph ^= 1; }
           }
         }
       }
     }
-    __syncwarp();
   } else if (warp == MMA_WARP) {
-    if (lane == 0 && rank == 0) {
+    // The whole warp runs the issue loop (warp-uniform control flow lets the compiler keep
+    // descriptors and counters in uniform registers); one elected lane issues.  A single-lane
+    // loop compiled to ~20 dependent instructions per MMA (ELECT/R2UR.BROADCAST waterfalls),
+    // ~100 cycles -- twice the tensor core's time for an N = 96 MMA.
+    if (rank == 0) {
       const uint32_t idesc = idesc_f16<BN, BF16, CG>();
       const int cw = g.mode == GM_DENSE ? 64 : g.cw, cbytes = BM * cw * 2;
-      // Everything that does not change per k-block is hoisted: the single issuing thread's
-      // instruction latency (not the tensor core) bounded N <= 128 MMAs at ~77+ cycles each.
       // A descriptor of stage s, step k = (desc of the stage base) + adelta[k] (16-byte units).
       uint32_t adelta[BK / 16];
 #pragma unroll
@@ -535,8 +668,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         adelta[k] = (uint32_t)(((e / cw) * cbytes + (e % cw) * 2) >> 4);
       }
       const uint64_t a_hi = sdesc(0, cw * 2), b_hi = sdesc(0, 128);
-      const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
-      int it = 0, lt = 0;
+      const uint32_t sA0 = (smem_u32(sA) & 0x3FFFFu) >> 4, sB0 = (smem_u32(sB) & 0x3FFFFu) >> 4;
+      int s = 0, lt = 0;
+      uint32_t ph = 0;
       for (int t = cid; t < tiles; t += ncl, ++lt) {
         const int slot = nslots == 2 ? (lt & 1) : 0;
         const uint32_t use = nslots == 2 ? (uint32_t)(lt >> 1) : (uint32_t)lt;
@@ -548,9 +682,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         tc_fence_after();
         for (int zi = 0; zi < g.zf; ++zi) {
           const uint32_t d = tmem + (uint32_t)(slot * slot_cols + zi * BN);
-          for (int kb = 0; kb < num_kb; ++kb, ++it) {
-            const int s = it % C::STAGES;
-            const uint32_t ph = (it / C::STAGES) & 1;
+          for (int kb = 0; kb < num_kb; ++kb) {
             {
               STAT_T0();
               mbar_wait(full0 + 8 * s, ph);
@@ -558,23 +690,30 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             }
             tc_fence_after();
             STAT_T0();
-            const uint64_t ad = a_hi | (uint64_t)(((sA0 + s * C::A_BYTES) & 0x3FFFFu) >> 4);
-            const uint64_t bd = b_hi | (uint64_t)(((sB0 + s * C::B_BYTES) & 0x3FFFFu) >> 4);
+            if (elect_one()) {
+              const uint64_t ad = a_hi | (uint64_t)(sA0 + (uint32_t)s * (C::A_BYTES >> 4));
+              const uint64_t bd = b_hi | (uint64_t)(sB0 + (uint32_t)s * (C::B_BYTES >> 4));
 #pragma unroll
-            for (int k = 0; k < BK / 16; ++k) {
-              if (CG == 2) mma_f16_2sm(d, ad + adelta[k], bd + 2 * k, idesc, (kb | k) != 0);
-              else mma_f16(d, ad + adelta[k], bd + 2 * k, idesc, (kb | k) != 0);
+              for (int k = 0; k < (kDbgNoMma ? 0 : BK / 16); ++k) {
+                if (CG == 2) mma_f16_2sm(d, ad + adelta[k], bd + 2 * k, idesc, (kb | k) != 0);
+                else mma_f16(d, ad + adelta[k], bd + 2 * k, idesc, (kb | k) != 0);
+              }
+              if (kDbgNoMma && CG == 1) mbar_arrive(empty0 + 8 * s);  // diagnostic: plain arrive
+              else if (CG == 2) mma_commit_2sm(empty0 + 8 * s);
+              else mma_commit(empty0 + 8 * s);
             }
-            if (CG == 2) mma_commit_2sm(empty0 + 8 * s);
-            else mma_commit(empty0 + 8 * s);
+            __syncwarp();
             STAT_ADD(st_mma_issue);
+            if (++s == C::STAGES) { s = 0; ph ^= 1; }
           }
         }
-        if (CG == 2) mma_commit_2sm(tfull0 + 8 * slot);
-        else mma_commit(tfull0 + 8 * slot);
+        if (elect_one()) {
+          if (CG == 2) mma_commit_2sm(tfull0 + 8 * slot);
+          else mma_commit(tfull0 + 8 * slot);
+        }
+        __syncwarp();
       }
     }
-    __syncwarp();
   } else if (warp < EPI_WARPS) {
     // ---- epilogue (warps 0-7): TMEM -> registers -> bias + act (+ LRN) -> global ----
     const int quarter = warp & 3, half = warp >> 2;
@@ -597,14 +736,18 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         mok = m < g.M;
       }
       {
+        // one lane per warp polls the barrier (256 polling threads slowed the whole SM's
+        // TMA stream ~3x); the warp then reconverges
         STAT_T0();
-        mbar_wait(tfull0 + 8 * slot, use & 1);
+        if (lane == 0) mbar_wait(tfull0 + 8 * slot, use & 1);
+        __syncwarp();
         STAT_ADD(st_epi_wait);
       }
       tc_fence_after();
       STAT_T0();
       const uint32_t tbase = tmem + lane_base + (uint32_t)(slot * slot_cols);
-      if (g.epi_lrn) {
+      if (kDbgNoEpi) {
+      } else if (g.epi_lrn) {
         // Channels c = zi * N + n (N == BN when zf > 1) live in columns zi*BN + n.  The LRN
         // window is clipped to [0, Ctot); values beyond are zero, so zero-padding is exact.
         // Warp half h processes 16-channel chunks [ib, ie) with a one-chunk halo each side.
@@ -753,15 +896,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       __syncwarp();
       if (lane == 0) {
         if (CG == 2) mbar_arrive_leader(tempty0 + 8 * slot);
-        else mbar_arrive(tempty0 + 8 * slot);
+        else mbar_arrive_relaxed(tempty0 + 8 * slot);
       }
     }
   }
 #ifdef DJINN_TC_STATS
   if (blockIdx.x == 0 && (threadIdx.x == TMA_WARP * 32 || threadIdx.x == MMA_WARP * 32 || threadIdx.x == 0))
-    printf("[tc BN=%d mode=%d N=%d K=%d tiles=%d grid=%d] warp %d total %llu prod_wait %llu mma_full %llu "
+    printf("[tc BN=%d mode=%d N=%d K=%d tiles=%d grid=%d] warp %d total %llu prod_wait %llu prod_issue %llu mma_full %llu "
            "mma_tempty %llu mma_issue %llu epi_wait %llu epi_work %llu\n",
-           BN, g.mode, g.N, g.K, tiles, gridDim.x, warp, clock64() - st_begin, st_prod_wait, st_mma_full, st_mma_tempty,
+           BN, g.mode, g.N, g.K, tiles, gridDim.x, warp, clock64() - st_begin, st_prod_wait, st_prod_issue, st_mma_full, st_mma_tempty,
            st_mma_issue, st_epi_wait, st_epi_work);
 #endif
   tc_fence_before();

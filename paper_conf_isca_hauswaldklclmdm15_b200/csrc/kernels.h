@@ -51,6 +51,7 @@ struct GemmGeom {
   int lcg, kwp;       // LC: taps per TMA row (box {Cgp, lcg, 1, 128}) and KW padded to lcg
   int kxs;            // conv: x offset between consecutive taps (x-unrolled input: xu), default 1
   int cg;             // 1: one CTA per 128-row tile; 2: cta_group::2 CTA pair per 256-row tile (B split)
+  int out_half;       // 16-bit output stored as fp16 whatever the path type (an LRN-only consumer)
   int a_tiled;        // conv: 0 = im2col-mode TMA over linear output pixels (default), 1 = tiled
                       //       4D boxes over bx x by x bn pixel blocks (DJINN_CONV_A=tiled)
   int bx, by, bn;     // conv: output-pixel block of one M tile (bx*by*bn == 128), x fastest
@@ -89,6 +90,13 @@ cudaError_t launch_tc_gemm(const GemmGeom& g, int bn, int dt, const CUtensorMap*
 // Channel c of a pixel is stored at (c/gsz)*gpitch + c%gsz (grouped layouts); pads -> 0.
 cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, int gsz, int gpitch, int size,
                        float alpha, float beta, float k, int dt, cudaStream_t st);
+
+// --- LRN + max pooling fused (K4+K5): fp16 NHWC input (pitch Cpi, C channels, pads zero),
+// Caffe LRN across channels in fp32, Caffe MAX pooling of the LRN output (kernel 1 = no pool),
+// output in type dt with a grouped channel layout (gsz, gpitch, pitch Cpo; pads written as 0).
+cudaError_t launch_lrn_pool(const void* x, void* y, int64_t rows, int C, int Cpi, int H, int W, int OH, int OW,
+                            int kernel, int stride, int pad, int out_gsz, int out_gpitch, int Cpo, int size,
+                            float alpha, float beta, float k, int dt, cudaStream_t st);
 
 // --- pooling (K5), NHWC, Caffe ceil geometry ------------------------------------------------
 // Output may be x-unrolled: pixel x stores pooled pixels x..x+out_xu-1 at pitch Cp each

@@ -364,6 +364,7 @@ void Net::build(const std::string& desc) {
       continue;
     }
     // ---- weighted layers: Convolution / LocallyConnected / InnerProduct ----
+    bool lrn_pool_next = false;
     int act = ACT_NONE;
     size_t j = i + 1;
     if (j < layers.size() && act_of(layers[j].type) >= 0) {
@@ -544,7 +545,19 @@ void Net::build(const std::string& desc) {
         throw Error(DJINN_E_SHAPE, L.name + ": internal: input channel pitch not TMA-chunkable");
       // Caffe LRN right after (the activation of) this conv: fuse it into the epilogue when one
       // tile holds every channel of a pixel (all groups side by side in TMEM).
-      if (f16 && !lc && i + 1 < layers.size() && layers[i + 1].type == "LRN" && layers[i + 1].lrn_size == 5) {
+      const char* lrn_sep = getenv("DJINN_LRN_POOL");
+      if (f16 && !lc && i + 1 < layers.size() && layers[i + 1].type == "LRN" && layers[i + 1].lrn_size == 5 &&
+          lrn_sep && lrn_sep[0] == '1' && L.num_output % 8 == 0) {
+        // Alternative (DJINN_LRN_POOL=1): the conv's epilogue stays bias + ReLU and stores fp16
+        // (only LRN reads it), and LRN + the MAX pooling after it run as one separate kernel.
+        // Measured slower than the epilogue fusion below.
+        lrn_pool_next = true;
+        g.out_half = 1;
+        o.out.Cp = rup(o.out.C, 16);
+        o.out.gsz = o.out.gpitch = 1 << 30;
+        g.out_pitch = o.out.Cp;
+        g.write_cols = grp == 1 ? o.out.Cp : Cog;
+      } else if (f16 && !lc && i + 1 < layers.size() && layers[i + 1].type == "LRN" && layers[i + 1].lrn_size == 5) {
         const int bn = tc_pick_bn(g);
         if (Cog <= 256 && (grp == 1 || bn == Cog) && grp * bn <= 256) {
           const LayerSpec& R = layers[i + 1];
@@ -608,6 +621,42 @@ void Net::build(const std::string& desc) {
     n_params += wcount + bcount;
     cur = o.out;
     ops.push_back(o);
+    if (lrn_pool_next) {
+      const LayerSpec& R = layers[i + 1];
+      Op lp;
+      lp.kind = OP_LRNPOOL;
+      lp.name = R.name;
+      lp.in = cur;
+      lp.lrn_size = R.lrn_size;
+      lp.alpha = R.alpha;
+      lp.beta = R.beta;
+      lp.lrn_k = R.lrn_k;
+      lp.kernel = 1; lp.stride = 1; lp.pad = 0; lp.is_max = 1;
+      Shape os = cur;
+      ++i;
+      ++n_layers;
+      if (i + 1 < layers.size() && layers[i + 1].type == "Pooling" && layers[i + 1].pool_max) {
+        const LayerSpec& Pl = layers[i + 1];
+        auto pout = [&](int in) {
+          int out = (int)((in + 2 * Pl.pad - Pl.kernel + Pl.stride - 1) / Pl.stride) + 1;
+          if (in + 2 * Pl.pad - Pl.kernel < 0) out = 1;
+          if (Pl.pad > 0 && (out - 1) * Pl.stride >= in + Pl.pad) --out;
+          return out;
+        };
+        os.H = pout(cur.H);
+        os.W = pout(cur.W);
+        lp.kernel = Pl.kernel; lp.stride = Pl.stride; lp.pad = Pl.pad;
+        lp.name += "+" + Pl.name;
+        ++i;
+        ++n_layers;
+      }
+      os = layout_for(i + 1, os);
+      lp.out = os;
+      lp.in_buf = o.out_buf;
+      lp.out_buf = curbuf = 1 - o.out_buf;
+      cur = os;
+      ops.push_back(lp);
+    }
   }
   out_elems = cur.C;
   arena_bytes = rupz(arena_off, 1024);
@@ -643,6 +692,7 @@ void Net::build(const std::string& desc) {
         break;
       }
       case OP_LRN: o.bytes_row = 2 * in_e * es; break;
+      case OP_LRNPOOL: o.bytes_row = in_e * es + out_e * es; break;
       case OP_POOL: o.bytes_row = in_e * es + out_e * es; break;
       case OP_SOFTMAX: o.bytes_row = 2.0 * in_e * 4; break;
     }
@@ -887,6 +937,11 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           e = launch_pool(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.H, o.in.W, o.out.H, o.out.W,
                           o.kernel, o.stride, o.pad, o.is_max, o.out.xu, dt, st);
           break;
+        case OP_LRNPOOL:
+          e = launch_lrn_pool(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.H, o.in.W, o.out.H, o.out.W,
+                              o.kernel, o.stride, o.pad, o.out.gsz, o.out.gpitch, o.out.Cp, o.lrn_size, o.alpha,
+                              o.beta, o.lrn_k, dt, st);
+          break;
         case OP_SOFTMAX:
           e = launch_softmax((const float*)w->buf[2], n, (int)out_elems, out_pitch, dst, mode, st);
           break;
@@ -907,7 +962,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
 
 std::string Net::plan_string() const {
   std::ostringstream s;
-  static const char* kinds[] = {"pack", "gemm", "lrn", "pool", "softmax"};
+  static const char* kinds[] = {"pack", "gemm", "lrn", "pool", "softmax", "lrn+pool"};
   static const char* modes[] = {"dense", "conv", "local"};
   s << "net " << name << " precision " << (dt == DT_F32 ? "fp32" : dt == DT_BF16 ? "bf16" : "fp16") << " max_rows "
     << max_rows << " arena " << arena_bytes << " B params " << n_params << "\n";
@@ -923,7 +978,7 @@ std::string Net::plan_string() const {
         << (o.g.lcg > 1 ? " taps/row=" + std::to_string(o.g.lcg) : std::string())
         << (o.g.mode == GM_CONV && o.g.a_tiled ? " block=" + std::to_string(o.g.bx) + "x" + std::to_string(o.g.by) + "x" +
                                                   std::to_string(o.g.bn) : std::string())
-        << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << "]";
+        << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << (o.g.out_half ? " fp16-out" : "") << "]";
     if (o.kind == OP_PACK && o.xform) s << " [" << (o.xform == 1 ? "space-to-depth " : "kx-unroll ") << o.xf << "]";
     s << "\n";
   }

@@ -43,7 +43,7 @@ struct LayerSpec {
   std::vector<int> dims;
 };
 
-enum OpKind { OP_PACK, OP_GEMM, OP_LRN, OP_POOL, OP_SOFTMAX };
+enum OpKind { OP_PACK, OP_GEMM, OP_LRN, OP_POOL, OP_SOFTMAX, OP_LRNPOOL };
 
 // Per-row activation tensor: NHWC, channel pitch Cp.  Channels may be stored in groups of
 // gsz at a per-group pitch gpitch (logical channel c lives at (c / gsz) * gpitch + c % gsz),

@@ -1,3 +1,4 @@
+import os
 """Host-side planner of libdjinn (djinn_describe: no device needed) -m "not gpu".
 
 Checks the library's own parse + shape inference against the oracle's independent one
@@ -39,6 +40,12 @@ def test_plan_first_layer_transforms_and_lrn_fusion():
     assert "kx-unroll 18" in face and "KHxKW=11x1" in face and "xblock=8" in face   # 8 outputs per GEMM row
     assert "32x71x71/p64" in face and "x-unrolled-input=2" in face                  # M2 -> C3
     assert "taps/row=4" in face                                                      # L4-L6
+    os.environ["DJINN_LRN_POOL"] = "1"                       # alternative: separate LRN+pool kernel
+    try:
+        sep = dj.djinn_describe(dj.net_description("imc"), dj.DJINN_BF16, 64)[0]
+    finally:
+        del os.environ["DJINN_LRN_POOL"]
+    assert "lrn+pool norm1+pool1" in sep and "lrn+pool norm2+pool2" in sep and "fp16-out" in sep
     fp32 = dj.djinn_describe(dj.net_description("imc"), dj.DJINN_FP32, 64)[0]
     assert "lrn norm1" in fp32 and "space-to-depth" not in fp32   # fp32 path: plain SIMT plan
 
