@@ -432,6 +432,117 @@ __global__ void pool16_kernel(const T* __restrict__ x, T* __restrict__ y, int64_
   }
 }
 
+// K5 MAX pooling with a channel-layout change: one thread per (output pixel, 8-channel chunk of
+// the OUTPUT layout); input and output layouts may differ (plain / grouped / x-unrolled), so the
+// pool's producer writes its natural pitch and the pool writes the consumer's layout.  Block =
+// (chunks of one output pixel) x (PIX consecutive output pixels of one image); the channel
+// mapping is computed once per block; the max runs on packed 16-bit pairs (exact).
+__device__ __forceinline__ uint4 max8(uint4 a, uint4 b, __half) {
+  uint4 r;
+  const __half2* x = reinterpret_cast<const __half2*>(&a);
+  const __half2* y = reinterpret_cast<const __half2*>(&b);
+  __half2* z = reinterpret_cast<__half2*>(&r);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) z[j] = __hmax2(x[j], y[j]);
+  return r;
+}
+__device__ __forceinline__ uint4 max8(uint4 a, uint4 b, __nv_bfloat16) {
+  uint4 r;
+  const __nv_bfloat162* x = reinterpret_cast<const __nv_bfloat162*>(&a);
+  const __nv_bfloat162* y = reinterpret_cast<const __nv_bfloat162*>(&b);
+  __nv_bfloat162* z = reinterpret_cast<__nv_bfloat162*>(&r);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) z[j] = __hmax2(x[j], y[j]);
+  return r;
+}
+
+template <typename T, int K>
+__global__ void pool_max_remap_kernel(const T* __restrict__ x, T* __restrict__ y, int C, int Cpi, int gsz_i,
+                                      int gpitch_i, int H, int W, int OH, int OW, int kern, int stride, int pad,
+                                      int Cpo, int gsz_o, int gpitch_o, int xu) {
+  __shared__ int in_off[64];  // per output chunk: input channel offset, -1 = zero chunk
+  const int P = Cpo / xu, chunks = P / 8;
+  if (threadIdx.y == 0 && threadIdx.x < chunks) {
+    const int pos = threadIdx.x * 8, grp = pos / gpitch_o, within = pos - grp * gpitch_o, c0 = grp * gsz_o + within;
+    in_off[threadIdx.x] = (within < gsz_o && c0 < C) ? (c0 / gsz_i) * gpitch_i + c0 % gsz_i : -1;
+  }
+  __syncthreads();
+  const int pix = blockIdx.x * blockDim.y + threadIdx.y;
+  if (pix >= OH * OW) return;
+  const int oy = pix / OW, ox = pix - oy * OW;
+  const int64_t r = blockIdx.y;
+  const int off = in_off[threadIdx.x];
+  T* yo = y + ((r * OH + oy) * OW + ox) * (int64_t)Cpo + threadIdx.x * 8;
+  uint4 ov = make_uint4(0, 0, 0, 0);
+  if (off >= 0) {
+    const T* base = x + r * (int64_t)H * W * Cpi + off;
+    int hs = oy * stride - pad, ws = ox * stride - pad;
+    int he = min(hs + kern, H + pad), we = min(ws + kern, W + pad);
+    hs = max(hs, 0); ws = max(ws, 0); he = min(he, H); we = min(we, W);
+    if (K > 0) {
+      // all K*K loads issued together; taps outside the clipped window re-read a tap inside
+      // it (a duplicate cannot change a max)
+      uint4 v[K > 0 ? K * K : 1];
+#pragma unroll
+      for (int a = 0; a < K; ++a)
+#pragma unroll
+        for (int b = 0; b < K; ++b) {
+          const int h = min(hs + a, he - 1), w = min(ws + b, we - 1);
+          v[a * K + b] = __ldg(reinterpret_cast<const uint4*>(base + ((int64_t)h * W + w) * Cpi));
+        }
+      ov = v[0];
+#pragma unroll
+      for (int j = 1; j < K * K; ++j) ov = max8(ov, v[j], T());
+    } else {
+      ov = __ldg(reinterpret_cast<const uint4*>(base + ((int64_t)hs * W + ws) * Cpi));
+      for (int h = hs; h < he; ++h)
+        for (int w = ws; w < we; ++w)
+          ov = max8(ov, __ldg(reinterpret_cast<const uint4*>(base + ((int64_t)h * W + w) * Cpi)), T());
+    }
+  }
+  *reinterpret_cast<uint4*>(yo) = ov;
+  for (int sl = 1; sl < xu; ++sl) {
+    if (ox - sl >= 0) *reinterpret_cast<uint4*>(yo - (int64_t)sl * Cpo + sl * P) = ov;  // pixel ox-sl, slot sl
+    if (ox + sl >= OW) *reinterpret_cast<uint4*>(yo + sl * P) = make_uint4(0, 0, 0, 0);  // past the row end
+  }
+}
+
+cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int Cpi, int gsz_i, int gpitch_i, int H,
+                              int W, int OH, int OW, int kernel, int stride, int pad, int Cpo, int gsz_o, int gpitch_o,
+                              int xu, int dt, cudaStream_t st) {
+  if (xu < 1 || Cpo % xu) return cudaErrorInvalidValue;
+  // plain layouts: one group spanning every position (channel c at c; pads read as zeros)
+  const bool gi = gsz_i < C, go = gsz_o < C;
+  if (!gi) gsz_i = gpitch_i = 1 << 30;
+  if (!go) gsz_o = gpitch_o = 1 << 30;
+  if (xu > 1 && go) return cudaErrorInvalidValue;
+  if (dt == DT_F32 || Cpi % 8 || Cpo % 8 || (gi && (gsz_i % 8 || gpitch_i % 8)) || (go && (gsz_o % 8 || gpitch_o % 8)) ||
+      kernel > stride + 1)
+    return cudaErrorInvalidValue;
+  const int chunks = Cpo / xu / 8;
+  if (chunks > 64) return cudaErrorInvalidValue;
+  const int pix = 256 / chunks;
+  for (int64_t r0 = 0; r0 < rows; r0 += 65535) {  // grid.z <= 65535 images per launch
+    const int64_t nr = rows - r0 < 65535 ? rows - r0 : 65535;
+    dim3 blk(chunks, pix), g((OH * OW + pix - 1) / pix, (unsigned)nr);
+    const size_t xo = (size_t)r0 * H * W * Cpi, yo = (size_t)r0 * OH * OW * Cpo;
+#define DJ_POOL_LAUNCH(T, KK)                                                                                   \
+  pool_max_remap_kernel<T, KK><<<g, blk, 0, st>>>((const T*)x + xo, (T*)y + yo, C, Cpi, gsz_i, gpitch_i, H, W, OH, OW, \
+                                                  kernel, stride, pad, Cpo, gsz_o, gpitch_o, xu)
+    if (dt == DT_F16) {
+      if (kernel == 3) DJ_POOL_LAUNCH(__half, 3);
+      else if (kernel == 2) DJ_POOL_LAUNCH(__half, 2);
+      else DJ_POOL_LAUNCH(__half, 0);
+    } else {
+      if (kernel == 3) DJ_POOL_LAUNCH(__nv_bfloat16, 3);
+      else if (kernel == 2) DJ_POOL_LAUNCH(__nv_bfloat16, 2);
+      else DJ_POOL_LAUNCH(__nv_bfloat16, 0);
+    }
+#undef DJ_POOL_LAUNCH
+  }
+  return cudaGetLastError();
+}
+
 cudaError_t launch_pool(const void* x, void* y, int64_t rows, int C, int Cp, int H, int W, int OH,
                         int OW, int kernel, int stride, int pad, int is_max, int out_xu, int dt, cudaStream_t st) {
   (void)C;

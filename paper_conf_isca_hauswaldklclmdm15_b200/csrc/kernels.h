@@ -91,6 +91,12 @@ cudaError_t launch_tc_gemm(const GemmGeom& g, int bn, int dt, const CUtensorMap*
 cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, int gsz, int gpitch, int size,
                        float alpha, float beta, float k, int dt, cudaStream_t st);
 
+// --- MAX pooling with a channel-layout change (plain/grouped in, plain/grouped/x-unrolled out), 16-bit,
+// kernel <= stride + 1.
+cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int Cpi, int gsz_i, int gpitch_i, int H,
+                              int W, int OH, int OW, int kernel, int stride, int pad, int Cpo, int gsz_o, int gpitch_o,
+                              int xu, int dt, cudaStream_t st);
+
 // --- LRN + max pooling fused (K4+K5): fp16 NHWC input (pitch Cpi, C channels, pads zero),
 // Caffe LRN across channels in fp32, Caffe MAX pooling of the LRN output (kernel 1 = no pool),
 // output in type dt with a grouped channel layout (gsz, gpitch, pitch Cpo; pads written as 0).

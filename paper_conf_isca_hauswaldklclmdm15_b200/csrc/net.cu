@@ -265,6 +265,9 @@ void Net::build(const std::string& desc) {
     sh.Cp = rup(sh.C, 16);
     for (size_t j = from; j < layers.size(); ++j) {
       const LayerSpec& L = layers[j];
+      // a MAX pool the column kernel handles re-lays the channels itself: its producer
+      // writes the plain pitch (no grouped-layout padding read back by the pool)
+      if (L.type == "Pooling" && L.pool_max && L.kernel <= L.stride + 1) return sh;
       if (L.type == "Convolution" && L.group > 1 && sh.C % L.group == 0) {
         const int cg = sh.C / L.group;
         if (cg % 16 == 0) {
@@ -350,9 +353,12 @@ void Net::build(const std::string& desc) {
         if (L.pad > 0 && (out - 1) * L.stride >= in + L.pad) --out;
         return out;
       };
-      o.out = cur;
+      o.out = Shape();
+      o.out.C = cur.C;
       o.out.H = pout(cur.H);
       o.out.W = pout(cur.W);
+      o.out = layout_for(i + 1, o.out);
+      if (!(f16 && L.pool_max && L.kernel <= L.stride + 1)) o.out = Shape{cur.C, o.out.H, o.out.W, cur.Cp, cur.gsz, cur.gpitch, 1, 0};
       o.kernel = L.kernel;
       o.stride = L.stride;
       o.pad = L.pad;
@@ -463,7 +469,8 @@ void Net::build(const std::string& desc) {
       // (pixel x also carries x+1.. up to 64 channels) and the conv x-blocks XB output pixels
       // per GEMM row (N = XB * out pitch): full-rate MMAs and XB x fewer TMA rows.
       if (f16 && !lc && grp == 1 && ops.size() > 1 && ops.back().kind == OP_POOL && o.xform == 0 && L.stride == 1 &&
-          pad == 0 && cur.gsz >= cur.C && cur.xu == 1 && cur.Cp <= 32 && 64 % cur.Cp == 0) {
+          pad == 0 && cur.gsz >= cur.C && cur.xu == 1 && cur.Cp <= 32 && 64 % cur.Cp == 0 &&
+          ops.back().in.Cp == cur.Cp && ops.back().in.gsz >= cur.C) {
         Shape os;
         os.C = L.num_output; os.H = OH; os.W = OW;
         os = layout_for(i + 1, os);
@@ -934,8 +941,13 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
                          o.alpha, o.beta, o.lrn_k, dt, st);
           break;
         case OP_POOL:
-          e = launch_pool(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.H, o.in.W, o.out.H, o.out.W,
-                          o.kernel, o.stride, o.pad, o.is_max, o.out.xu, dt, st);
+          if (dt != DT_F32 && o.is_max && o.kernel <= o.stride + 1)
+            e = launch_pool_remap(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.gsz, o.in.gpitch,
+                                  o.in.H, o.in.W, o.out.H, o.out.W, o.kernel, o.stride, o.pad, o.out.Cp, o.out.gsz,
+                                  o.out.gpitch, o.out.xu, dt, st);
+          else
+            e = launch_pool(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.H, o.in.W, o.out.H, o.out.W,
+                            o.kernel, o.stride, o.pad, o.is_max, o.out.xu, dt, st);
           break;
         case OP_LRNPOOL:
           e = launch_lrn_pool(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.H, o.in.W, o.out.H, o.out.W,

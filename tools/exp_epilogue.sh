@@ -1,4 +1,4 @@
-# Diagnostic: per-op times of IMC under the diagnostic builds.
+# Diagnostic: per-op times of IMC / FACE (tools/op_times.py); DJINN_LIB selects a variant build.
 L=$PWD/paper_conf_isca_hauswaldklclmdm15_b200
-for v in libdjinn libdjinn_nomma; do DJINN_LIB=$L/$v.so timeout 120 python tools/op_times.py imc bf16 1024 10 | grep -E "conv|fc|total"; done
-DJINN_LIB=$L/libdjinn_stats.so timeout 300 python tools/run_app.py imc bf16 1024 1 2>&1 | grep "\[tc" | head -6
+timeout 120 python tools/op_times.py imc bf16 1024 10 | grep -E "pool|total"
+timeout 120 python tools/op_times.py face bf16 256 10 | grep -E "pool|M2|total"
