@@ -30,7 +30,7 @@ static inline int nblocks(int64_t n, int t) { return (int)((n + t - 1) / t); }
 // convolution a dense, 16-element-aligned K (DESIGN.md sec 5 "first layer").
 template <typename T>
 __global__ void pack16_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int C, int H, int W,
-                              int mode, int f, int Ho, int Wo, int Cp) {
+                              int mode, int f, int xs, int Ho, int Wo, int Cp) {
   const int chunks = Cp / 8;
   const int per_row = Ho * Wo * chunks;  // 32-bit index math inside a row
   for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
@@ -57,7 +57,7 @@ __global__ void pack16_kernel(const float* __restrict__ x, T* __restrict__ y, in
         } else {
           const int kx = cc / C;
           c = cc - kx * C;
-          xx = xo + kx;
+          xx = xo * xs + kx;
           ok = kx < f && xx < W;
         }
         v[j] = cvt<T>(ok ? __ldg(src + (c * H + yy) * W + xx) : 0.f);
@@ -86,7 +86,7 @@ __global__ void pack32_kernel(const float* __restrict__ x, float* __restrict__ y
 // tracked with incremental counters (no integer division per element).
 template <typename T>
 __global__ void pack_xform_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int C, int H, int W,
-                                  int mode, int f, int Ho, int Wo, int Cp) {
+                                  int mode, int f, int xs, int Ho, int Wo, int Cp) {
   const int per_row = Ho * Wo;
   for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
     const float* src = x + r * C * (int64_t)H * W;
@@ -99,7 +99,7 @@ __global__ void pack_xform_kernel(const float* __restrict__ x, T* __restrict__ y
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
           const int yy = mode == 1 ? yo * f + a : yo;
-          const int xx = mode == 1 ? xo * f + b : xo + a;
+          const int xx = mode == 1 ? xo * f + b : xo * xs + a;
           const bool ok = a < f && yy < H && xx < W;
           v[j] = cvt<T>(ok ? __ldg(src + ((int64_t)c * H + yy) * W + xx) : 0.f);
           if (++c == C) {
@@ -120,7 +120,7 @@ __global__ void pack_xform_kernel(const float* __restrict__ x, T* __restrict__ y
 // Compile-time specialisation of the first-layer transforms for the Tonic nets: every source
 // offset is a constant relative to the pixel's base address, so each output channel costs one
 // load and one convert (the generic kernel spent its time in index bookkeeping).
-template <typename T, int MODE, int C, int F, int CP>
+template <typename T, int MODE, int C, int F, int CP, int XS>
 __global__ void pack_xform_fixed_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int H, int W,
                                         int Ho, int Wo) {
   const int per_row = Ho * Wo;
@@ -129,7 +129,7 @@ __global__ void pack_xform_fixed_kernel(const float* __restrict__ x, T* __restri
     for (int pix = blockIdx.x * blockDim.x + threadIdx.x; pix < per_row; pix += gridDim.x * blockDim.x) {
       const int yo = pix / Wo, xo = pix - (pix / Wo) * Wo;
       T* dst = y + (r * per_row + pix) * (int64_t)CP;
-      const int y0 = MODE == 1 ? yo * F : yo, x0 = MODE == 1 ? xo * F : xo;
+      const int y0 = MODE == 1 ? yo * F : yo, x0 = MODE == 1 ? xo * F : xo * XS;
       const float* p0 = src + (int64_t)y0 * W + x0;
 #pragma unroll
       for (int ch = 0; ch < CP; ch += 8) {
@@ -154,25 +154,25 @@ __global__ void pack_xform_fixed_kernel(const float* __restrict__ x, T* __restri
 }
 
 template <typename T>
-static bool launch_pack_fixed(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f, int Ho,
+static bool launch_pack_fixed(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f, int xs, int Ho,
                               int Wo, int Cp, cudaStream_t st) {
   dim3 g(min(nblocks(Ho * Wo, 128), 1024), (unsigned)(rows < 65535 ? rows : 65535));
-  if (mode == 2 && C == 3 && f == 18 && Cp == 64)
-    pack_xform_fixed_kernel<T, 2, 3, 18, 64><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
-  else if (mode == 2 && C == 1 && f == 12 && Cp == 16)
-    pack_xform_fixed_kernel<T, 2, 1, 12, 16><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
+  if (mode == 2 && C == 3 && f == 18 && xs == 8 && Cp == 64)
+    pack_xform_fixed_kernel<T, 2, 3, 18, 64, 8><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
+  else if (mode == 2 && C == 1 && f == 12 && xs == 8 && Cp == 16)
+    pack_xform_fixed_kernel<T, 2, 1, 12, 16, 8><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
   else if (mode == 1 && C == 3 && f == 4 && Cp == 64)
-    pack_xform_fixed_kernel<T, 1, 3, 4, 64><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
+    pack_xform_fixed_kernel<T, 1, 3, 4, 64, 1><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
   else
     return false;
   return true;
 }
 
-cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f,
+cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f, int xs,
                               int Ho, int Wo, int Cp, int dt, cudaStream_t st) {
   if (dt != DT_F32 && mode != 0) {
-    const bool done = dt == DT_F16 ? launch_pack_fixed<__half>(x, y, rows, C, H, W, mode, f, Ho, Wo, Cp, st)
-                                   : launch_pack_fixed<__nv_bfloat16>(x, y, rows, C, H, W, mode, f, Ho, Wo, Cp, st);
+    const bool done = dt == DT_F16 ? launch_pack_fixed<__half>(x, y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp, st)
+                                   : launch_pack_fixed<__nv_bfloat16>(x, y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp, st);
     if (done) return cudaGetLastError();
   }
   const int T = 256;
@@ -182,16 +182,16 @@ cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int 
   } else if (mode != 0) {
     dim3 g(min(nblocks(Ho * Wo, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
     if (dt == DT_F16)
-      pack_xform_kernel<__half><<<g, T, 0, st>>>(x, (__half*)y, rows, C, H, W, mode, f, Ho, Wo, Cp);
+      pack_xform_kernel<__half><<<g, T, 0, st>>>(x, (__half*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
     else
-      pack_xform_kernel<__nv_bfloat16><<<g, T, 0, st>>>(x, (__nv_bfloat16*)y, rows, C, H, W, mode, f, Ho, Wo, Cp);
+      pack_xform_kernel<__nv_bfloat16><<<g, T, 0, st>>>(x, (__nv_bfloat16*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
   } else {
     const int per_row = Ho * Wo * (Cp / 8);
     dim3 g(min(nblocks(per_row, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
     if (dt == DT_F16)
-      pack16_kernel<__half><<<g, T, 0, st>>>(x, (__half*)y, rows, C, H, W, mode, f, Ho, Wo, Cp);
+      pack16_kernel<__half><<<g, T, 0, st>>>(x, (__half*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
     else
-      pack16_kernel<__nv_bfloat16><<<g, T, 0, st>>>(x, (__nv_bfloat16*)y, rows, C, H, W, mode, f, Ho, Wo, Cp);
+      pack16_kernel<__nv_bfloat16><<<g, T, 0, st>>>(x, (__nv_bfloat16*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
   }
   return cudaGetLastError();
 }

@@ -508,7 +508,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       }
       __syncwarp();
       const uint32_t tx_bytes = CG * (C::A_BYTES + (kDbgNoB ? 0 : C::B_BYTES));
-      const int sx = g.xb > 1 ? g.xb : g.stride, OWb = g.OWb, st = g.stride, pd = g.pad, cin_goff = g.cin_goff;
+      const int sx = g.xstep, OWb = g.OWb, st = g.stride, pd = g.pad, cin_goff = g.cin_goff;
       for (int t = cid; t < tiles; t += ncl) {
         const TileCoord tc = warp_uniform(tile_coord(g, t, mt, nt, CG));
         const int my_m0 = tc.m0 + (int)rank * BM;
@@ -555,7 +555,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         const int rem = my_m0 - img * oy_per;
         const int oy = rem / g.OWb;
         wy = oy * g.stride - g.pad;
-        wx = (rem - oy * g.OWb) * (g.xb > 1 ? g.xb : g.stride) - g.pad;
+        wx = (rem - oy * g.OWb) * g.xstep - g.pad;
       }
       // every lane holds the same values; saying so lets ptxas use plain R2UR for the TMA
       // operands instead of an ELECT/R2UR.BROADCAST waterfall per issue

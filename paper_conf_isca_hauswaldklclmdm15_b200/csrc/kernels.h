@@ -50,6 +50,8 @@ struct GemmGeom {
   int Co;             // real output channels (x-blocked conv: per dx)
   int lcg, kwp;       // LC: taps per TMA row (box {Cgp, lcg, 1, 128}) and KW padded to lcg
   int kxs;            // conv: x offset between consecutive taps (x-unrolled input: xu), default 1
+  int xstep;          // conv: input-x offset between consecutive GEMM-row pixels (blocks):
+                      //   stride, or xb when x-blocked, or 1 over a block-packed first layer
   int cg;             // 1: one CTA per 128-row tile; 2: cta_group::2 CTA pair per 256-row tile (B split)
   int out_half;       // 16-bit output stored as fp16 whatever the path type (an LRN-only consumer)
   int a_tiled;        // conv: 0 = im2col-mode TMA over linear output pixels (default), 1 = tiled
@@ -63,9 +65,11 @@ struct GemmGeom {
 
 // --- pack (K0): fp32 NCHW rows -> NHWC with channel pitch Cp, type dt -------------------
 // mode 0: y[r][h][w][c] = x[r][c][h][w];  mode 1 (space-to-depth by f):
-// y[r][ty][tx][(dy*f+dx)*C + c] = x[r][c][f*ty+dy][f*tx+dx];  mode 2 (kx-unroll of width f):
-// y[r][h][w][kx*C + c] = x[r][c][h][w+kx].  Out-of-range sources and pad channels are 0.
-cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f,
+// y[r][ty][tx][(dy*f+dx)*C + c] = x[r][c][f*ty+dy][f*tx+dx];  mode 2 (kx-unroll of width f,
+// packed pixels xs input pixels apart -- xs = the conv's x-block, so only the pixels the
+// GEMM rows start at are written): y[r][h][j][kx*C + c] = x[r][c][h][j*xs+kx].
+// Out-of-range sources and pad channels are 0.
+cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f, int xs,
                               int Ho, int Wo, int Cp, int dt, cudaStream_t st);
 
 // --- SIMT fp32 implicit GEMM (K7; exact fp32 FFMA accumulation) --------------------------

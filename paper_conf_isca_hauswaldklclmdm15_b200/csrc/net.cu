@@ -452,14 +452,16 @@ void Net::build(const std::string& desc) {
           const int U = k + XB - 1, OWb = (OW + XB - 1) / XB;
           pk.xform = o.xform = 2;
           pk.xf = o.xf = U;
+          pk.xs = o.xs = XB;
           pk.out = Shape();
-          pk.out.C = U * cur.C; pk.out.H = cur.H; pk.out.W = XB > 1 ? OWb * XB : OW; pk.out.Cp = tap_pitch(U * cur.C);
+          pk.out.C = U * cur.C; pk.out.H = cur.H; pk.out.W = OWb; pk.out.Cp = tap_pitch(U * cur.C);
           g.H = cur.H; g.W = pk.out.W; g.Cp_in = g.Cgp = pk.out.Cp;
           g.KH = k; g.KW = 1;
           if (XB > 1) {
             g.xb = XB;
             g.OWb = OWb;
             g.N = XB * os.Cp;
+            g.xstep = 1;  // packed pixel j already starts at input x = j * XB
           }
         }
         if (pk.xform) { o.in = pk.out; }
@@ -503,6 +505,7 @@ void Net::build(const std::string& desc) {
       g.write_cols = grp == 1 ? o.out.Cp : Cog;
       g.bias_zstride = Cog;
       if (g.xb < 1) { g.xb = 1; g.OWb = OW; }
+      if (g.xstep < 1) g.xstep = g.xb > 1 ? g.xb : g.stride;
       g.Co = Cog;
       o.ohw = lc ? 1 : OH * g.OWb;
       g.zf = 1;
@@ -863,7 +866,7 @@ Workspace* Net::workspace(cudaStream_t st) {
         encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 4, dims, strides, box, g.cw * 2, estr);
       } else if (g.mode == GM_CONV) {
         // filter-window top-left positions: w = -pad + i*stride, i < OW (same for h)
-        const int sx = g.xb > 1 ? g.xb : g.stride;
+        const int sx = g.xstep;
         const int lower[2] = {-g.pad, -g.pad};
         const int upper[2] = {-g.pad + (g.OWb - 1) * sx - (g.W - 1), -g.pad + (g.OH - 1) * g.stride - (g.H - 1)};
         if (-g.pad + (g.OWb - 1) * sx + (g.KW - 1) * g.kxs > g.W - 1 + g.pad)
@@ -918,7 +921,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
       if (profile) ck(cudaEventRecord(prof_events[pbase + i], st), "profile event");
       switch (o.kind) {
         case OP_PACK:
-          e = launch_pack_input(src, w->buf[0], n, o.in.C, o.in.H, o.in.W, o.xform, o.xf, o.out.H, o.out.W, o.out.Cp,
+          e = launch_pack_input(src, w->buf[0], n, o.in.C, o.in.H, o.in.W, o.xform, o.xf, o.xs, o.out.H, o.out.W, o.out.Cp,
                                 dt, st);
           break;
         case OP_GEMM: {
@@ -991,7 +994,7 @@ std::string Net::plan_string() const {
         << (o.g.mode == GM_CONV && o.g.a_tiled ? " block=" + std::to_string(o.g.bx) + "x" + std::to_string(o.g.by) + "x" +
                                                   std::to_string(o.g.bn) : std::string())
         << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << (o.g.out_half ? " fp16-out" : "") << "]";
-    if (o.kind == OP_PACK && o.xform) s << " [" << (o.xform == 1 ? "space-to-depth " : "kx-unroll ") << o.xf << "]";
+    if (o.kind == OP_PACK && o.xform) s << " [" << (o.xform == 1 ? "space-to-depth " : "kx-unroll ") << o.xf << (o.xs > 1 ? " step " + std::to_string(o.xs) : std::string()) << "]";
     s << "\n";
   }
   return s.str();

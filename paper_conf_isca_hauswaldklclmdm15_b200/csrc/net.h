@@ -70,7 +70,7 @@ struct Op {
   bool fold_half = false;       // bias += 1/2 * rowsum(W): the producer stores sigma - 1/2
   // first-layer input transform (PACK op and the conv it feeds): 0 none, 1 space-to-depth
   // by xf (= conv stride), 2 kx-unroll of a stride-1 kernel of width xf
-  int xform = 0, xf = 1;
+  int xform = 0, xf = 1, xs = 1;  // xs: kx-unroll x step (packed pixel j starts at input x = j*xs)
   Shape orig_in;                // the layer's input before the transform
   int orig_k = 0;               // original kernel size
   // lrn
