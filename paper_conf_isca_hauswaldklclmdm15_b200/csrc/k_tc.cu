@@ -438,7 +438,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   const int tiles = mt * nt * zt;
   int slot_cols = 32;  // TMEM columns per accumulator slot (power of two >= zf*BN)
   while (slot_cols < g.zf * BN) slot_cols <<= 1;
-  const int nslots = 2 * slot_cols <= 512 ? 2 : 1;
+  const int nslots = 2;  // launch_inst guarantees zf * BN <= 256 (two accumulator slots)
   int tcols = 32;
   while (tcols < nslots * slot_cols) tcols <<= 1;
 
@@ -451,7 +451,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     }
     for (int s = 0; s < 2; ++s) {
       mbar_init(tfull0 + 8 * s, 1);
-      mbar_init(tempty0 + 8 * s, EPI_WARPS * CG);  // leader's: both CTAs' epilogues arrive
+      mbar_init(tempty0 + 8 * s, (EPI_WARPS / 2) * CG);  // one warpgroup per slot; leader's: both CTAs'
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     fence_proxy_async();
@@ -716,15 +716,20 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     }
   } else if (warp < EPI_WARPS) {
     // ---- epilogue (warps 0-7): TMEM -> registers -> bias + act (+ LRN) -> global ----
-    const int quarter = warp & 3, half = warp >> 2;
-    int lt = 0;
+    // The two warpgroups alternate tiles: warpgroup h drains TMEM slot h (local tiles lt with
+    // lt % 2 == h), so every thread owns one whole output row (pixel) of its tile: the LRN
+    // channel window slides through registers with no halo recomputation, and each warpgroup
+    // has two MMA tile-times for its tile.
+    const int quarter = warp & 3, wg = warp >> 2;
     const uint32_t lane_base = (uint32_t)(quarter * 32) << 16;
+    const int r = quarter * 32 + lane;
+    int lt = 0;
     for (int t = cid; t < tiles; t += ncl, ++lt) {
+      if ((lt & 1) != wg) continue;
       TileCoord tc = tile_coord(g, t, mt, nt, CG);
       tc.m0 += (int)rank * BM;  // this CTA's rows of the pair tile
-      const int slot = nslots == 2 ? (lt & 1) : 0;
-      const uint32_t use = nslots == 2 ? (uint32_t)(lt >> 1) : (uint32_t)lt;
-      const int r = quarter * 32 + lane;
+      const int slot = lt & 1;
+      const uint32_t use = (uint32_t)(lt >> 1);
       int m;       // output pixel (conv) / GEMM row (dense, LC)
       bool mok;
       if (g.mode == GM_CONV && g.a_tiled) {
@@ -748,41 +753,46 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       const uint32_t tbase = tmem + lane_base + (uint32_t)(slot * slot_cols);
       if (kDbgNoEpi) {
       } else if (g.epi_lrn) {
-        // Channels c = zi * N + n (N == BN when zf > 1) live in columns zi*BN + n.  The LRN
-        // window is clipped to [0, Ctot); values beyond are zero, so zero-padding is exact.
-        // Warp half h processes 16-channel chunks [ib, ie) with a one-chunk halo each side.
+        // Caffe LRN across the pixel's Ctot = zf * N channels (channel zi * N + n lives in
+        // column zi * BN + n).  The window [c-2, c+2] is clipped to [0, Ctot): values beyond
+        // are zero, so zero-padding is exact.  Chunk i+2 is in flight from TMEM while chunk i
+        // is normalised.
         const int N = g.N, Ctot = g.zf * N;
-        const int nch = (Ctot + 15) / 16, per = (nch + 1) / 2;
-        const int ib = half * per, ie = min(nch, ib + per);
+        const int nch = (Ctot + 15) / 16;
         const int64_t obase = (int64_t)m * g.out_pitch;
         const float ka = g.lrn_alpha_over_n, kk = g.lrn_k, nb = -g.lrn_beta;
-        float cur[16], nxt[16];
-        float pm2 = 0.f, pm1 = 0.f;
-        auto load_chunk = [&](int i, float (&v)[16]) {
+        int zi_n = 0, n_n = 0;  // (z slice, column) of the next chunk to load: no division
+        auto issue = [&](uint32_t (&rr)[16]) {
+          tmem_ld16(tbase + (uint32_t)(zi_n * BN + n_n), rr);
+        };
+        auto advance = [&]() {
+          n_n += 16;
+          if (n_n >= N) { n_n = 0; ++zi_n; }
+        };
+        auto convert = [&](int i, const uint32_t (&rr)[16], float (&v)[16]) {
           const int c0 = i * 16;
-          const int zi = c0 / N, n0 = c0 - zi * N;
           float b[16];
           load_bias16(b, bias, c0, Ctot);
-          uint32_t rr[16];
-          tmem_ld16(tbase + (uint32_t)(zi * BN + n0), rr);
-          tmem_wait_ld();
           bias_act16(v, rr, b, g.act);
           if (c0 + 16 > Ctot) {
 #pragma unroll
             for (int j = 0; j < 16; ++j) v[j] = c0 + j < Ctot ? v[j] : 0.f;
           }
         };
-        if (ib < ie) {
-          if (ib > 0) {
-            load_chunk(ib - 1, cur);
-            pm2 = cur[14] * cur[14];
-            pm1 = cur[15] * cur[15];
-          }
-          load_chunk(ib, cur);
-        }
-        for (int i = ib; i < ie; ++i) {
+        float cur[16], nxt[16];
+        uint32_t rr[16];
+        issue(rr);
+        advance();
+        tmem_wait_ld();
+        convert(0, rr, cur);
+        if (nch > 1) { issue(rr); advance(); }
+        float pm2 = 0.f, pm1 = 0.f;
+#pragma unroll 1
+        for (int i = 0; i < nch; ++i) {
           if (i + 1 < nch) {
-            load_chunk(i + 1, nxt);
+            tmem_wait_ld();
+            convert(i + 1, rr, nxt);
+            if (i + 2 < nch) { issue(rr); advance(); }
           } else {
 #pragma unroll
             for (int j = 0; j < 16; ++j) nxt[j] = 0.f;
@@ -826,12 +836,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           oy = rem / OWb;
           ox0 = (rem - oy * OWb) * g.xb;
         }
-        const int cols = BN / 2, cbeg = half * cols;
         const int64_t rowpix = ((int64_t)img * g.OH + oy) * g.OW;
         const float* bb = g.mode == GM_LC ? bias + (int64_t)tc.z0 * g.bias_zstride : bias;
+        int dx = 0, co0 = 0;
 #pragma unroll 1
-        for (int c = cbeg; c < cbeg + cols; c += 16) {
-          const int dx = c / P, co0 = c - dx * P;
+        for (int c = 0; c < BN; c += 16) {
           float b[16];
           load_bias16(b, g.mode == GM_LC ? bb + dx * g.Co : bb, co0, g.Co);
           uint32_t rr[16];
@@ -847,21 +856,19 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             }
             store16<BF16>(g, Y, (rowpix + ox) * P + co0, v, 2);
           }
+          co0 += 16;
+          if (co0 >= P) { co0 = 0; ++dx; }
         }
       } else {
-        // columns of each z-slice split between the two warps of a lane quarter
-        const int cols = BN >= 32 ? BN / 2 : BN;
-        const int cbeg = BN >= 32 ? half * cols : 0;
-        const bool active = BN >= 32 || half == 0;
-        for (int zi = 0; zi < g.zf && active; ++zi) {
+        for (int zi = 0; zi < g.zf; ++zi) {
           const int z = tc.z0 * g.zf + zi;
           const int64_t pix = (g.mode == GM_LC) ? (int64_t)m * g.OH * g.OW + z : (int64_t)m;
           const int goff = (g.mode == GM_CONV) ? z * g.cout_goff : 0;
           const float* bz = bias + (int64_t)z * g.bias_zstride;
           const int nb0 = tc.n0 * BN;
 #pragma unroll 1
-          for (int c = cbeg; c < cbeg + cols; c += 32) {
-            const bool two = c + 16 < cbeg + cols;
+          for (int c = 0; c < BN; c += 32) {
+            const bool two = c + 16 < BN;
             float b0[16], b1[16];
             load_bias16(b0, bz, nb0 + c, g.N);  // bias loads in flight during the TMEM load
             if (two) load_bias16(b1, bz, nb0 + c + 16, g.N);
@@ -937,6 +944,7 @@ cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtenso
                                    ((g.Nimg + g.bn - 1) / g.bn)
                              : (g.M + BM * CG - 1) / (BM * CG);
   const int64_t tiles = mtiles * ((g.N + BN - 1) / BN) * (g.Z / g.zf);
+  if (g.zf * BN > 256) return cudaErrorInvalidValue;  // two TMEM accumulator slots needed
   const int max_cl = tc_num_sms() / CG;
   const int clusters = (int)(tiles < max_cl ? tiles : max_cl);
   cudaLaunchConfig_t cfg = {};
