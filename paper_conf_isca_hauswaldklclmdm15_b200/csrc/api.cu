@@ -86,12 +86,10 @@ int djinn_load_net(const char* desc, size_t desc_len, const float* weights, size
       return fail(DJINN_E_NOMEM, "weight arena allocation (" + std::to_string(n.arena_bytes) + " B)");
     }
     // per-layer tile choice and B tensor maps over the arena
+    n.choose_tiles();
     for (djinn::Op& o : n.ops) {
       if (o.kind != djinn::OP_GEMM || n.dt == djinn::DT_F32) continue;
-      djinn::GemmGeom g = o.g;
-      g.M = (int)(n.max_rows * o.ohw);
-      o.bn = djinn::tc_pick_bn(g);
-      o.g.cg = djinn::tc_pick_cg(g, o.bn);
+      const djinn::GemmGeom& g = o.g;
       uint64_t dims[3] = {(uint64_t)g.Kpad, (uint64_t)g.N, (uint64_t)g.Z};
       uint64_t strides[2] = {(uint64_t)g.Kpad * 2, (uint64_t)g.N * g.Kpad * 2};
       uint32_t box[3] = {64, (uint32_t)(o.bn / o.g.cg), 1};
@@ -246,13 +244,7 @@ int djinn_describe(const char* desc, size_t desc_len, int precision, int64_t max
     n.dt = precision == DJINN_FP32 ? djinn::DT_F32 : precision == DJINN_BF16 ? djinn::DT_BF16 : djinn::DT_F16;
     n.max_rows = max_rows;
     n.build(std::string(desc, desc_len));
-    for (djinn::Op& o : n.ops)
-      if (o.kind == djinn::OP_GEMM && n.dt != djinn::DT_F32) {
-        djinn::GemmGeom g = o.g;
-        g.M = (int)(n.max_rows * o.ohw);
-        o.bn = djinn::tc_pick_bn(g);
-        o.g.cg = djinn::tc_pick_cg(g, o.bn);
-      }
+    n.choose_tiles();
     if (in_elems) *in_elems = n.in_elems;
     if (out_elems) *out_elems = n.out_elems;
     if (n_params) *n_params = n.n_params;

@@ -459,7 +459,7 @@ __device__ __forceinline__ uint4 max8(uint4 a, uint4 b, __nv_bfloat16) {
 template <typename T, int K>
 __global__ void pool_max_remap_kernel(const T* __restrict__ x, T* __restrict__ y, int C, int Cpi, int gsz_i,
                                       int gpitch_i, int H, int W, int OH, int OW, int kern, int stride, int pad,
-                                      int Cpo, int gsz_o, int gpitch_o, int xu) {
+                                      int Cpo, int gsz_o, int gpitch_o, int xu, int obd) {
   __shared__ int in_off[64];  // per output chunk: input channel offset, -1 = zero chunk
   const int P = Cpo / xu, chunks = P / 8;
   if (threadIdx.y == 0 && threadIdx.x < chunks) {
@@ -472,7 +472,7 @@ __global__ void pool_max_remap_kernel(const T* __restrict__ x, T* __restrict__ y
   const int oy = pix / OW, ox = pix - oy * OW;
   const int64_t r = blockIdx.y;
   const int off = in_off[threadIdx.x];
-  T* yo = y + ((r * OH + oy) * OW + ox) * (int64_t)Cpo + threadIdx.x * 8;
+  T* yo = y + ((r * (OH + 2 * obd) + oy + obd) * (OW + 2 * obd) + ox + obd) * (int64_t)Cpo + threadIdx.x * 8;
   uint4 ov = make_uint4(0, 0, 0, 0);
   if (off >= 0) {
     const T* base = x + r * (int64_t)H * W * Cpi + off;
@@ -509,8 +509,8 @@ __global__ void pool_max_remap_kernel(const T* __restrict__ x, T* __restrict__ y
 
 cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int Cpi, int gsz_i, int gpitch_i, int H,
                               int W, int OH, int OW, int kernel, int stride, int pad, int Cpo, int gsz_o, int gpitch_o,
-                              int xu, int dt, cudaStream_t st) {
-  if (xu < 1 || Cpo % xu) return cudaErrorInvalidValue;
+                              int xu, int obd, int dt, cudaStream_t st) {
+  if (xu < 1 || Cpo % xu || obd < 0 || (obd > 0 && xu > 1)) return cudaErrorInvalidValue;
   // plain layouts: one group spanning every position (channel c at c; pads read as zeros)
   const bool gi = gsz_i < C, go = gsz_o < C;
   if (!gi) gsz_i = gpitch_i = 1 << 30;
@@ -525,10 +525,10 @@ cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int C
   for (int64_t r0 = 0; r0 < rows; r0 += 65535) {  // grid.z <= 65535 images per launch
     const int64_t nr = rows - r0 < 65535 ? rows - r0 : 65535;
     dim3 blk(chunks, pix), g((OH * OW + pix - 1) / pix, (unsigned)nr);
-    const size_t xo = (size_t)r0 * H * W * Cpi, yo = (size_t)r0 * OH * OW * Cpo;
+    const size_t xo = (size_t)r0 * H * W * Cpi, yo = (size_t)r0 * (OH + 2 * obd) * (OW + 2 * obd) * Cpo;
 #define DJ_POOL_LAUNCH(T, KK)                                                                                   \
   pool_max_remap_kernel<T, KK><<<g, blk, 0, st>>>((const T*)x + xo, (T*)y + yo, C, Cpi, gsz_i, gpitch_i, H, W, OH, OW, \
-                                                  kernel, stride, pad, Cpo, gsz_o, gpitch_o, xu)
+                                                  kernel, stride, pad, Cpo, gsz_o, gpitch_o, xu, obd)
     if (dt == DT_F16) {
       if (kernel == 3) DJ_POOL_LAUNCH(__half, 3);
       else if (kernel == 2) DJ_POOL_LAUNCH(__half, 2);

@@ -46,7 +46,10 @@ namespace djinn {
 namespace {
 
 constexpr int BM = 128, BK = 64;
-constexpr int EPI_WARPS = 8, TMA_WARP = 8, MMA_WARP = 9, TMAB_WARP = 10, NUM_THREADS = 352;
+// Warp roles: 0-7 epilogue, 8-11 TMA loaders, 12 TMEM allocator + MMA issuer.  A warp issues one
+// TMA box per ~375 cycles however large the box (tools/tma_bench3.cu: the rate scales with the
+// number of issuing warps, not with bytes), so stages are dealt round-robin to four loaders.
+constexpr int EPI_WARPS = 8, LOAD_WARP0 = 8, NLOAD = 4, MMA_WARP = 12, NUM_THREADS = 32 * 13;
 
 constexpr int KTAB_MAX = 256;  // im2col producer: per-K-chunk (channel, kx, ky) table entries
 template <int BN, int CG = 1>
@@ -80,6 +83,22 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
         : "r"(bar), "r"(parity)
         : "memory");
     if (++iters > (1u << 28)) __trap();  // a lost arrival must fault, never hang the GPU
+  } while (!done);
+}
+// Waiting threads suspend in the barrier until its phase completes (or the hint expires):
+// spinning producers / epilogue pollers had been taking issue slots from the epilogue warps
+// sharing their SM sub-partition (ncu: branch_resolving + no_inst stalls at the poll loops).
+__device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
+  uint32_t done, iters = 0;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(bar), "r"(parity), "r"(0x989680u)
+        : "memory");
+    if (++iters > (1u << 24)) __trap();  // a lost arrival must fault, never hang the GPU
   } while (!done);
 }
 __device__ __forceinline__ void tma_2d(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1) {
@@ -365,6 +384,10 @@ template <bool BF16>
 __device__ __forceinline__ void store_chunk(const GemmGeom& g, void* Y, int64_t pixbase, int cglob,
                                             const float (&v)[16], int nvalid8) {
   const int gsz = g.out_gsz;
+  if (gsz == g.out_gpitch) {  // plain layout (or groups stored back to back): no division
+    store16<BF16>(g, Y, pixbase + cglob, v, nvalid8);
+    return;
+  }
   const int grp = cglob / gsz, cin = cglob - grp * gsz;
   const int64_t gbase = pixbase + (int64_t)grp * g.out_gpitch;
   store16<BF16>(g, Y, gbase + cin, v, nvalid8);
@@ -408,7 +431,7 @@ __device__ __forceinline__ int num_m_tiles(const GemmGeom& g, int cg = 1) {
 }
 
 // ---------------------------------------------------------------- the kernel
-template <int BN, bool BF16, int CG>
+template <int BN, bool BF16, int CG, bool SLAB>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const GemmGeom g, const float* __restrict__ bias, void* __restrict__ Y) {
@@ -418,14 +441,21 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   const int cid = blockIdx.x / CG, ncl = gridDim.x / CG;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // non-slab: [A ring][B ring][bars];  slab: [B ring][2 slabs][bars]
+  const int NST = SLAB ? g.stages : C::STAGES;  // ring stages
+  const uint32_t slab_chunk = SLAB ? (uint32_t)(g.slab_parts * g.slab_rows * 128) : 0u;  // one 64-channel chunk
+  const uint32_t slab_bytes = SLAB ? (uint32_t)(g.zf * (g.Cgp / 64)) * slab_chunk : 0u;
   uint8_t* sA = smem;
-  uint8_t* sB = smem + C::STAGES * C::A_BYTES;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
-  // bars: full[STAGES], empty[STAGES], tfull[2], tempty[2]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * C::STAGES + 4);
+  uint8_t* sB = SLAB ? smem : smem + C::STAGES * C::A_BYTES;
+  uint8_t* sSlab = smem + ((NST * C::B_BYTES + 1023) & ~1023);
+  uint64_t* bars = SLAB ? reinterpret_cast<uint64_t*>(sSlab + 2 * slab_bytes)
+                        : reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
+  // bars: full[NST], empty[NST], tfull[2], tempty[2], sfull[2], sempty[2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * NST + 8);
   __shared__ uint32_t ktab[KTAB_MAX];
-  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + C::STAGES);
-  const uint32_t tfull0 = smem_u32(bars + 2 * C::STAGES), tempty0 = smem_u32(bars + 2 * C::STAGES + 2);
+  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + NST);
+  const uint32_t tfull0 = smem_u32(bars + 2 * NST), tempty0 = smem_u32(bars + 2 * NST + 2);
+  const uint32_t sfull0 = smem_u32(bars + 2 * NST + 4), sempty0 = smem_u32(bars + 2 * NST + 6);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int num_kb = g.Kpad / BK;
@@ -442,16 +472,17 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   int tcols = 32;
   while (tcols < nslots * slot_cols) tcols <<= 1;
 
-  if (warp == TMA_WARP && lane == 0) {
-    // (barriers are initialised before the __syncthreads below; the B producer, warp 10,
-    // starts after it)
-    for (int s = 0; s < C::STAGES; ++s) {
+  if (warp == LOAD_WARP0 && lane == 0) {
+    // (barriers are initialised before the __syncthreads below; every other role starts after it)
+    for (int s = 0; s < NST; ++s) {
       mbar_init(full0 + 8 * s, 1);
       mbar_init(empty0 + 8 * s, 1);
     }
     for (int s = 0; s < 2; ++s) {
       mbar_init(tfull0 + 8 * s, 1);
       mbar_init(tempty0 + 8 * s, (EPI_WARPS / 2) * CG);  // one warpgroup per slot; leader's: both CTAs'
+      mbar_init(sfull0 + 8 * s, 1);
+      mbar_init(sempty0 + 8 * s, 1);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     fence_proxy_async();
@@ -477,37 +508,99 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
-  if (warp == TMA_WARP) {
-    // A producer.  The whole warp runs the loop (warp-uniform values stay in uniform
-    // registers), one elected lane issues; (ky, kx, c) of each K chunk advance by counters
-    // (no division).  The single-lane version spent ~900 cycles of dependent instructions
-    // per stage, which capped the operand stream at ~20 B/cycle/SM.
+  if (warp >= LOAD_WARP0 && warp < LOAD_WARP0 + NLOAD) {
+    // TMA loaders.  Each loader warp runs the whole loop (warp-uniform values stay in uniform
+    // registers, (ky, kx, c) of each K chunk advance by counters: no division) and one elected
+    // lane issues the stages it owns: stage q belongs to loader q % NLOAD, which loads its A
+    // chunk(s) and B box and arms its barrier; in slab mode loader 0 loads the per-tile slabs
+    // and the (B-only) stages go round-robin to loaders 1..NLOAD-1.
+    const int li = warp - LOAD_WARP0;
     const int cw = g.cw, cbytes = BM * cw * 2;
     const int chunks_per_kb = BK / cw;
     const int nchunks_k = g.K / cw;  // valid chunks along K
     const int oy_per = g.OH * g.OWb;
     const int mode = g.mode, a_tiled = g.a_tiled, lcg = g.lcg, kwp = g.kwp, KW = g.KW, Cgp = g.Cgp, kxs = g.kxs;
     const int Cp_in = g.Cp_in, zf = g.zf;
-    const uint32_t sA0 = smem_u32(sA);
+    const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
+    const int bn_off = (int)rank * (BN / CG);
     const bool leader = elect_one();
-    int s = 0;
+    const uint32_t tx_bytes = SLAB ? CG * C::B_BYTES : CG * (C::A_BYTES + (kDbgNoB ? 0 : C::B_BYTES));
+    const int nown = SLAB ? NLOAD - 1 : NLOAD, myq = SLAB ? li - 1 : li;  // stage owner index
+    int s = 0, qo = 0;  // ring slot; owner of the current stage (q % nown)
     uint32_t ph = 0;
+    auto load_b = [&](uint32_t fb, int kb, int n0, int z) {
+      if (!kDbgNoB) tma_a3<CG>(sB0 + (uint32_t)s * C::B_BYTES, &tmB, fb, kb * BK, n0 * BN + bn_off, z);
+    };
+    auto next_stage = [&]() {
+      if (++s == NST) { s = 0; ph ^= 1; }
+      if (++qo == nown) qo = 0;
+    };
     const int nq = num_kb * chunks_per_kb;
-    if (mode == GM_CONV && !a_tiled && nq <= KTAB_MAX) {
+    if (SLAB && li == 0) {
+      // one slab per tile: zf groups x (Cgp / 64) channel chunks x slab_parts boxes of
+      // slab_rows input pixels starting at the tile's first virtual pixel; double-buffered
+      const uint32_t slab0 = smem_u32(sSlab);
+      const int nchunk = g.Cgp / 64, parts = g.slab_parts, srows = g.slab_rows, cin_goff = g.cin_goff;
+      int lt = 0;
+      for (int t = cid; t < tiles; t += ncl, ++lt) {
+        const TileCoord tc = warp_uniform(tile_coord(g, t, mt, nt, CG));
+        const int my_m0 = tc.m0 + (int)rank * BM;
+        const int sb = lt & 1;
+        const uint32_t use = (uint32_t)(lt >> 1);
+        {
+          STAT_T0();
+          mbar_wait_sleep(sempty0 + 8 * sb, (use & 1) ^ 1);
+          STAT_ADD(st_prod_wait);
+        }
+        STAT_T0();
+        if (leader) {
+          if (rank == 0) mbar_arrive_expect_tx(sfull0 + 8 * sb, CG * slab_bytes);
+          uint32_t dst = slab0 + (uint32_t)sb * slab_bytes;
+          for (int zi = 0; zi < zf; ++zi) {
+            const int cbase = (tc.z0 * zf + zi) * cin_goff;
+            for (int j = 0; j < nchunk; ++j)
+              for (int p = 0; p < parts; ++p, dst += (uint32_t)srows * 128)
+                tma_a2<CG>(dst, &tmA, sfull0 + 8 * sb, cbase + 64 * j, my_m0 + p * srows);
+          }
+        }
+        __syncwarp();
+        STAT_ADD(st_prod_issue);
+      }
+    } else if (SLAB) {
+      // B-only stages of the slab mode
+      for (int t = cid; t < tiles; t += ncl) {
+        const TileCoord tc = warp_uniform(tile_coord(g, t, mt, nt, CG));
+        for (int zi = 0; zi < zf; ++zi) {
+          const int z = tc.z0 * zf + zi;
+          for (int kb = 0; kb < num_kb; ++kb) {
+            if (qo == myq) {
+              mbar_wait_sleep(empty0 + 8 * s, ph ^ 1);
+              if (leader) {
+                if (rank == 0) mbar_arrive_expect_tx(full0 + 8 * s, tx_bytes);
+                load_b(full0 + 8 * s, kb, tc.n0, z);
+              }
+              __syncwarp();
+            }
+            next_stage();
+          }
+        }
+      }
+    } else if (mode == GM_CONV && !a_tiled && nq <= KTAB_MAX) {
       // im2col fast path: the (channel, kx, ky) of every K chunk comes from a table built
       // once, so a stage costs a handful of instructions (the issuing warp's instruction
       // latency, not the TMA unit, had bounded the operand stream: DESIGN.md sec 5).
       const int cpt = Cgp / cw;  // chunks per tap
-      for (int qq = lane; qq < nq; qq += 32) {
-        uint32_t e = 0xFFFFu;  // past the valid K: channel = Cp_in (TMA zero-fills)
-        if (qq < nchunks_k) {
-          const int tap = qq / cpt, kx = tap % KW, ky = tap / KW;
-          e = (uint32_t)((qq - tap * cpt) * cw) | ((uint32_t)(kx * kxs) << 16) | ((uint32_t)ky << 24);
+      if (li == 0) {
+        for (int qq = lane; qq < nq; qq += 32) {
+          uint32_t e = 0xFFFFu;  // past the valid K: channel = Cp_in (TMA zero-fills)
+          if (qq < nchunks_k) {
+            const int tap = qq / cpt, kx = tap % KW, ky = tap / KW;
+            e = (uint32_t)((qq - tap * cpt) * cw) | ((uint32_t)(kx * kxs) << 16) | ((uint32_t)ky << 24);
+          }
+          ktab[qq] = e;
         }
-        ktab[qq] = e;
       }
-      __syncwarp();
-      const uint32_t tx_bytes = CG * (C::A_BYTES + (kDbgNoB ? 0 : C::B_BYTES));
+      asm volatile("bar.sync 1, %0;" ::"n"(NLOAD * 32) : "memory");  // ktab complete for all loaders
       const int sx = g.xstep, OWb = g.OWb, st = g.stride, pd = g.pad, cin_goff = g.cin_goff;
       for (int t = cid; t < tiles; t += ncl) {
         const TileCoord tc = warp_uniform(tile_coord(g, t, mt, nt, CG));
@@ -517,30 +610,34 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         const int oy = rem / OWb;
         const int wy = warp_uniform(oy * st - pd), wx = warp_uniform((rem - oy * OWb) * sx - pd);
         for (int zi = 0; zi < zf; ++zi) {
-          const int cbase = (tc.z0 * zf + zi) * cin_goff;
+          const int z = tc.z0 * zf + zi;
+          const int cbase = z * cin_goff;
           int q = 0;
           for (int kb = 0; kb < num_kb; ++kb) {
-            {
-              STAT_T0();
-              mbar_wait(empty0 + 8 * s, ph ^ 1);
-              STAT_ADD(st_prod_wait);
-            }
-            STAT_T0();
-            const uint32_t fb = full0 + 8 * s;
-            const uint32_t a_dst = sA0 + (uint32_t)s * C::A_BYTES;
-            if (leader) {
-              if (rank == 0) mbar_arrive_expect_tx(fb, tx_bytes);
-              for (int j = 0; j < chunks_per_kb; ++j) {
-                const uint32_t e = ktab[q + j];
-                const int cr = (int)(e & 0xFFFFu);
-                const int c = cr == 0xFFFF ? Cp_in : cbase + cr;
-                tma_i2c<CG>(a_dst + j * cbytes, &tmA, fb, c, wx, wy, img, (uint16_t)((e >> 16) & 0xFF), (uint16_t)(e >> 24));
+            if (qo == myq) {
+              {
+                STAT_T0();
+                mbar_wait_sleep(empty0 + 8 * s, ph ^ 1);
+                STAT_ADD(st_prod_wait);
               }
+              STAT_T0();
+              const uint32_t fb = full0 + 8 * s;
+              const uint32_t a_dst = sA0 + (uint32_t)s * C::A_BYTES;
+              if (leader) {
+                if (rank == 0) mbar_arrive_expect_tx(fb, tx_bytes);
+                for (int j = 0; j < chunks_per_kb; ++j) {
+                  const uint32_t e = ktab[q + j];
+                  const int cr = (int)(e & 0xFFFFu);
+                  const int c = cr == 0xFFFF ? Cp_in : cbase + cr;
+                  tma_i2c<CG>(a_dst + j * cbytes, &tmA, fb, c, wx, wy, img, (uint16_t)((e >> 16) & 0xFF), (uint16_t)(e >> 24));
+                }
+                load_b(fb, kb, tc.n0, z);
+              }
+              __syncwarp();
+              STAT_ADD(st_prod_issue);
             }
-            __syncwarp();
-            STAT_ADD(st_prod_issue);
             q += chunks_per_kb;
-            if (++s == C::STAGES) { s = 0; ph ^= 1; }
+            next_stage();
           }
         }
       }
@@ -573,17 +670,24 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         const int cbase = mode == GM_CONV ? z * g.cin_goff : 0;
         int cc = 0, kx = 0, ky = 0, q = 0;  // chunk counters: channel offset, tap, chunk index
         for (int kb = 0; kb < num_kb; ++kb) {
-          {
-            STAT_T0();
-            mbar_wait(empty0 + 8 * s, ph ^ 1);
-            STAT_ADD(st_prod_wait);
+          const bool mine = qo == myq;
+          const uint32_t fb = full0 + 8 * s;
+          if (mine) {
+            {
+              STAT_T0();
+              mbar_wait_sleep(empty0 + 8 * s, ph ^ 1);
+              STAT_ADD(st_prod_wait);
+            }
+            if (leader) {
+              if (rank == 0) mbar_arrive_expect_tx(fb, tx_bytes);
+              load_b(fb, kb, tc.n0, z);
+            }
           }
           STAT_T0();
-          const uint32_t fb = full0 + 8 * s;
-          if (leader && rank == 0) mbar_arrive_expect_tx(fb, CG * (C::A_BYTES + (kDbgNoB ? 0 : C::B_BYTES)));
           const uint32_t a_dst = sA0 + (uint32_t)s * C::A_BYTES;
+          const bool iss = mine && leader;
           if (mode == GM_DENSE) {
-            if (leader) tma_a2<CG>(a_dst, &tmA, fb, kb * BK, my_m0);
+            if (iss) tma_a2<CG>(a_dst, &tmA, fb, kb * BK, my_m0);
           } else {
             for (int j = 0; j < chunks_per_kb; ++j, ++q) {
               // past the valid K: a channel coordinate beyond the extent -> TMA zero-fills
@@ -591,25 +695,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
               const uint32_t dst = a_dst + j * cbytes;
               if (mode == GM_CONV) {
                 if (a_tiled) {
-                  if (leader) tma_a4<CG>(dst, &tmA, fb, c, wx + kx, wy + ky, img);
-                } else if (leader) {
-#ifdef DJINN_DBG_WALK
-                  if (g.K == 576 && g.OW == 55) {  // diagnostic: tools/tma_bench2.cu's walk (conv1)
-                    const int m0 = my_m0, per_img = g.OW * g.OH, im = m0 / per_img, rem = m0 - im * per_img;
-                    const int oy = rem / g.OW, ox = rem - oy * g.OW;
-                    tma_i2c<CG>(dst, &tmA, fb, 0, ox, oy, im, (uint16_t)(kb % 3), (uint16_t)(kb / 3));
-                  } else {
-                    tma_i2c<CG>(dst, &tmA, fb, c, wx, wy, img, (uint16_t)(kx * kxs), (uint16_t)ky);
-                  }
-#else
+                  if (iss) tma_a4<CG>(dst, &tmA, fb, c, wx + kx, wy + ky, img);
+                } else if (iss) {
                   tma_i2c<CG>(dst, &tmA, fb, c, wx, wy, img, (uint16_t)(kx * kxs), (uint16_t)ky);
-#endif
                 }
               } else if (lcg > 1) {  // LC, lcg taps per row: 3D view {W*C, H, N}
                 const int xe = q < nchunks_k ? (lcx + kx) * Cp_in : g.W * Cp_in;  // K tail: OOB
-                if (leader) tma_a3<CG>(dst, &tmA, fb, xe, lcy + ky, my_m0);
+                if (iss) tma_a3<CG>(dst, &tmA, fb, xe, lcy + ky, my_m0);
               } else {  // LC: rows are images at the fixed output location z
-                if (leader) tma_a4<CG>(dst, &tmA, fb, c, lcx + kx, lcy + ky, my_m0);
+                if (iss) tma_a4<CG>(dst, &tmA, fb, c, lcx + kx, lcy + ky, my_m0);
               }
               if (lcg > 1) {
                 kx += lcg;
@@ -625,30 +719,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           }
           __syncwarp();
           STAT_ADD(st_prod_issue);
-          if (++s == C::STAGES) { s = 0; ph ^= 1; }
-        }
-      }
-    }
-  } else if (warp == TMAB_WARP) {
-    // B (weights) producer: a second issuing warp so the A and B TMA streams overlap.  The
-    // expect-tx of the stage (both operands) is armed by the A producer; tx may complete
-    // before it is armed.
-    if (!kDbgNoB) {
-      const bool leader = elect_one();
-      const uint32_t sB0 = smem_u32(sB);
-      const int bn_off = (int)rank * (BN / CG);
-      int s = 0;
-      uint32_t ph = 0;
-      for (int t = cid; t < tiles; t += ncl) {
-        const TileCoord tc = warp_uniform(tile_coord(g, t, mt, nt, CG));
-        for (int zi = 0; zi < g.zf; ++zi) {
-          const int z = tc.z0 * g.zf + zi;
-          for (int kb = 0; kb < num_kb; ++kb) {
-            mbar_wait(empty0 + 8 * s, ph ^ 1);
-            if (leader) tma_a3<CG>(sB0 + (uint32_t)s * C::B_BYTES, &tmB, full0 + 8 * s, kb * BK, tc.n0 * BN + bn_off, z);
-            __syncwarp();
-            if (++s == C::STAGES) { s = 0; ph ^= 1; }
-          }
+          next_stage();
         }
       }
     }
@@ -667,7 +738,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         const int e = k * 16;
         adelta[k] = (uint32_t)(((e / cw) * cbytes + (e % cw) * 2) >> 4);
       }
-      const uint64_t a_hi = sdesc(0, cw * 2), b_hi = sdesc(0, 128);
+      const uint64_t a_hi = sdesc(0, SLAB ? 128 : cw * 2), b_hi = sdesc(0, 128);
       const uint32_t sA0 = (smem_u32(sA) & 0x3FFFFu) >> 4, sB0 = (smem_u32(sB) & 0x3FFFFu) >> 4;
       int s = 0, lt = 0;
       uint32_t ph = 0;
@@ -676,10 +747,63 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         const uint32_t use = nslots == 2 ? (uint32_t)(lt >> 1) : (uint32_t)lt;
         {
           STAT_T0();
-          mbar_wait(tempty0 + 8 * slot, (use & 1) ^ 1);
+          mbar_wait_sleep(tempty0 + 8 * slot, (use & 1) ^ 1);
           STAT_ADD(st_mma_tempty);
         }
         tc_fence_after();
+        if (SLAB) {
+          // taps are row shifts of the tile's slab: A(tap) = slab chunk + (ky*Wv + kx) rows
+          // (the 128B swizzle is address-based: a start 128*r bytes into a 1024-aligned atom
+          // reads rows r.. correctly; tools/umma_shift_test.cu)
+          const int sb = lt & 1;
+          {
+            STAT_T0();
+            mbar_wait(sfull0 + 8 * sb, (uint32_t)(lt >> 1) & 1);
+            STAT_ADD(st_mma_full);
+          }
+          tc_fence_after();
+          const int nchunk = g.Cgp / 64, Wv = g.Wv, KW = g.KW;
+          const uint32_t slabS = ((smem_u32(sSlab) & 0x3FFFFu) >> 4) + (uint32_t)sb * (slab_bytes >> 4);
+          for (int zi = 0; zi < g.zf; ++zi) {
+            const uint32_t d = tmem + (uint32_t)(slot * slot_cols + zi * BN);
+            int j = 0, kx = 0, ky = 0;
+            for (int kb = 0; kb < num_kb; ++kb) {
+              {
+                STAT_T0();
+                mbar_wait(full0 + 8 * s, ph);
+                STAT_ADD(st_mma_full);
+              }
+              tc_fence_after();
+              STAT_T0();
+              if (elect_one()) {
+                const uint32_t arow = slabS + (uint32_t)((zi * nchunk + j) * (int)(slab_chunk >> 4)) +
+                                      (uint32_t)((ky * Wv + kx) * 8);
+                const uint64_t ad = a_hi | (uint64_t)arow;
+                const uint64_t bd = b_hi | (uint64_t)(sB0 + (uint32_t)s * (C::B_BYTES >> 4));
+#pragma unroll
+                for (int k = 0; k < BK / 16; ++k) {
+                  if (CG == 2) mma_f16_2sm(d, ad + 2 * k, bd + 2 * k, idesc, (kb | k) != 0);
+                  else mma_f16(d, ad + 2 * k, bd + 2 * k, idesc, (kb | k) != 0);
+                }
+                if (CG == 2) mma_commit_2sm(empty0 + 8 * s);
+                else mma_commit(empty0 + 8 * s);
+              }
+              __syncwarp();
+              STAT_ADD(st_mma_issue);
+              if (++j == nchunk) {
+                j = 0;
+                if (++kx == KW) { kx = 0; ++ky; }
+              }
+              if (++s == NST) { s = 0; ph ^= 1; }
+            }
+          }
+          if (elect_one()) {
+            if (CG == 2) { mma_commit_2sm(tfull0 + 8 * slot); mma_commit_2sm(sempty0 + 8 * sb); }
+            else { mma_commit(tfull0 + 8 * slot); mma_commit(sempty0 + 8 * sb); }
+          }
+          __syncwarp();
+          continue;
+        }
         for (int zi = 0; zi < g.zf; ++zi) {
           const uint32_t d = tmem + (uint32_t)(slot * slot_cols + zi * BN);
           for (int kb = 0; kb < num_kb; ++kb) {
@@ -704,7 +828,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             }
             __syncwarp();
             STAT_ADD(st_mma_issue);
-            if (++s == C::STAGES) { s = 0; ph ^= 1; }
+            if (++s == NST) { s = 0; ph ^= 1; }
           }
         }
         if (elect_one()) {
@@ -730,12 +854,29 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       tc.m0 += (int)rank * BM;  // this CTA's rows of the pair tile
       const int slot = lt & 1;
       const uint32_t use = (uint32_t)(lt >> 1);
-      int m;       // output pixel (conv) / GEMM row (dense, LC)
+      int m;       // GEMM row (dense, LC)
       bool mok;
-      if (g.mode == GM_CONV && g.a_tiled) {
-        const int ox = tc.x0 + r % g.bx, oy = tc.y0 + (r / g.bx) % g.by, im = tc.i0 + r / (g.bx * g.by);
-        mok = ox < g.OW && oy < g.OH && im < g.Nimg;
-        m = (im * g.OH + oy) * g.OW + ox;
+      // conv: output pixel (img, oy, ox) of the row (ox: first pixel of its x block) and its
+      // index in the stored output (zero border obd)
+      int img = 0, oy = 0, ox = 0;
+      int64_t opix = 0;
+      if (g.mode == GM_CONV) {
+        if (g.a_tiled) {
+          ox = tc.x0 + r % g.bx; oy = tc.y0 + (r / g.bx) % g.by; img = tc.i0 + r / (g.bx * g.by);
+          mok = ox < g.OW && oy < g.OH && img < g.Nimg;
+        } else {
+          // im2col: rows enumerate (img, oy, x block) densely; slab: the stored input grid
+          const int hh = SLAB ? g.Hv : g.OH, ww = SLAB ? g.Wv : g.OWb;
+          const int mv = tc.m0 + r;
+          img = mv / (hh * ww);
+          const int rem = mv - img * (hh * ww);
+          oy = rem / ww;
+          const int xu = rem - oy * ww;
+          ox = xu * g.xb;
+          mok = img < g.Nimg && oy < g.OH && xu < g.OWb;
+        }
+        opix = ((int64_t)img * (g.OH + 2 * g.obd) + oy + g.obd) * (g.OW + 2 * g.obd) + ox + g.obd;
+        m = (int)opix;
       } else {
         m = tc.m0 + r;
         mok = m < g.M;
@@ -744,7 +885,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         // one lane per warp polls the barrier (256 polling threads slowed the whole SM's
         // TMA stream ~3x); the warp then reconverges
         STAT_T0();
-        if (lane == 0) mbar_wait(tfull0 + 8 * slot, use & 1);
+        if (lane == 0) mbar_wait_sleep(tfull0 + 8 * slot, use & 1);
         __syncwarp();
         STAT_ADD(st_epi_wait);
       }
@@ -759,7 +900,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         // is normalised.
         const int N = g.N, Ctot = g.zf * N;
         const int nch = (Ctot + 15) / 16;
-        const int64_t obase = (int64_t)m * g.out_pitch;
+        const int64_t obase = opix * g.out_pitch;
         const float ka = g.lrn_alpha_over_n, kk = g.lrn_k, nb = -g.lrn_beta;
         int zi_n = 0, n_n = 0;  // (z slice, column) of the next chunk to load: no division
         auto issue = [&](uint32_t (&rr)[16]) {
@@ -769,11 +910,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           n_n += 16;
           if (n_n >= N) { n_n = 0; ++zi_n; }
         };
+        float bq[16];  // bias of the next chunk to convert (loaded one chunk ahead)
+        load_bias16(bq, bias, 0, Ctot);
         auto convert = [&](int i, const uint32_t (&rr)[16], float (&v)[16]) {
           const int c0 = i * 16;
-          float b[16];
-          load_bias16(b, bias, c0, Ctot);
-          bias_act16(v, rr, b, g.act);
+          bias_act16(v, rr, bq, g.act);
+          if (c0 + 16 < Ctot) load_bias16(bq, bias, c0 + 16, Ctot);
           if (c0 + 16 > Ctot) {
 #pragma unroll
             for (int j = 0; j < 16; ++j) v[j] = c0 + j < Ctot ? v[j] : 0.f;
@@ -825,18 +967,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         // is channels [co0, co0+16) of output pixel block*xb + dx.  Conv: row m = (img, oy,
         // block); LC: row m = image, the block is the tile's z.
         const int P = g.out_pitch, OWb = g.OWb;
-        int img, oy, ox0;
+        int ox0 = ox;
+        int64_t pix0 = opix;  // stored index of pixel ox0
         if (g.mode == GM_LC) {
-          img = m;
-          oy = tc.z0 / OWb;
-          ox0 = (tc.z0 - oy * OWb) * g.xb;
-        } else {
-          img = m / (g.OH * OWb);
-          const int rem = m - img * (g.OH * OWb);
-          oy = rem / OWb;
-          ox0 = (rem - oy * OWb) * g.xb;
+          const int ly = tc.z0 / OWb;
+          ox0 = (tc.z0 - ly * OWb) * g.xb;
+          pix0 = ((int64_t)m * g.OH + ly) * g.OW + ox0;
         }
-        const int64_t rowpix = ((int64_t)img * g.OH + oy) * g.OW;
         const float* bb = g.mode == GM_LC ? bias + (int64_t)tc.z0 * g.bias_zstride : bias;
         int dx = 0, co0 = 0;
 #pragma unroll 1
@@ -846,15 +983,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           uint32_t rr[16];
           tmem_ld16(tbase + (uint32_t)c, rr);
           tmem_wait_ld();
-          const int ox = ox0 + dx;
-          if (mok && ox < g.OW && c < g.N) {
+          const int oxd = ox0 + dx;
+          if (mok && oxd < g.OW && c < g.N) {
             float v[16];
             bias_act16(v, rr, b, g.act);
             if (co0 + 16 > g.Co) {
 #pragma unroll
               for (int j = 0; j < 16; ++j) v[j] = co0 + j < g.Co ? v[j] : 0.f;
             }
-            store16<BF16>(g, Y, (rowpix + ox) * P + co0, v, 2);
+            store16<BF16>(g, Y, (pix0 + dx) * P + co0, v, 2);
           }
           co0 += 16;
           if (co0 >= P) { co0 = 0; ++dx; }
@@ -862,7 +999,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       } else {
         for (int zi = 0; zi < g.zf; ++zi) {
           const int z = tc.z0 * g.zf + zi;
-          const int64_t pix = (g.mode == GM_LC) ? (int64_t)m * g.OH * g.OW + z : (int64_t)m;
+          const int64_t pix = (g.mode == GM_LC) ? (int64_t)m * g.OH * g.OW + z : (g.mode == GM_CONV ? opix : (int64_t)m);
           const int goff = (g.mode == GM_CONV) ? z * g.cout_goff : 0;
           const float* bz = bias + (int64_t)z * g.bias_zstride;
           const int nb0 = tc.n0 * BN;
@@ -908,7 +1045,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     }
   }
 #ifdef DJINN_TC_STATS
-  if (blockIdx.x == 0 && (threadIdx.x == TMA_WARP * 32 || threadIdx.x == MMA_WARP * 32 || threadIdx.x == 0))
+  if (blockIdx.x == 0 && (threadIdx.x == LOAD_WARP0 * 32 || threadIdx.x == MMA_WARP * 32 || threadIdx.x == 0))
     printf("[tc BN=%d mode=%d N=%d K=%d tiles=%d grid=%d] warp %d total %llu prod_wait %llu prod_issue %llu mma_full %llu "
            "mma_tempty %llu mma_issue %llu epi_wait %llu epi_work %llu\n",
            BN, g.mode, g.N, g.K, tiles, gridDim.x, warp, clock64() - st_begin, st_prod_wait, st_prod_issue, st_mma_full, st_mma_tempty,
@@ -928,16 +1065,28 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
 int g_num_sms = 0;
 
-template <int BN, bool BF16, int CG>
+// dynamic shared memory of a slab-mode launch: B ring + two slabs + barriers (+ alignment slack)
+constexpr int SLAB_SMEM_MAX = 227 * 1024 - 1024;  // 227 KB per block minus the static ktab
+template <int BN, int CG>
+int slab_smem(const GemmGeom& g, int stages) {
+  using C = Cfg<BN, CG>;
+  const int ring = (stages * C::B_BYTES + 1023) & ~1023;
+  const int slab = g.zf * (g.Cgp / 64) * g.slab_parts * g.slab_rows * 128;
+  return 1024 + ring + 2 * slab + (2 * stages + 8) * 8 + 16;
+}
+
+template <int BN, bool BF16, int CG, bool SLAB>
 cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtensorMap* tmB, const float* bias, void* Y,
                         cudaStream_t st) {
   using C = Cfg<BN, CG>;
-  static bool attr_set = false;  // benign race: idempotent attribute set
-  auto kern = tc_gemm_kernel<BN, BF16, CG>;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+  static int attr_set = 0;  // benign race: idempotent attribute set
+  auto kern = tc_gemm_kernel<BN, BF16, CG, SLAB>;
+  const int smem = SLAB ? slab_smem<BN, CG>(g, g.stages) : C::SMEM;
+  if (SLAB && (g.stages < 2 || smem > SLAB_SMEM_MAX)) return cudaErrorInvalidValue;
+  if (attr_set < smem) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SLAB ? SLAB_SMEM_MAX : C::SMEM);
     if (e != cudaSuccess) return e;
-    attr_set = true;
+    attr_set = SLAB ? SLAB_SMEM_MAX : C::SMEM;
   }
   const int64_t mtiles = (g.mode == GM_CONV && g.a_tiled)
                              ? (int64_t)((g.OW + g.bx - 1) / g.bx) * ((g.OH + g.by - 1) / g.by) *
@@ -950,7 +1099,7 @@ cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtenso
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(clusters * CG);
   cfg.blockDim = dim3(NUM_THREADS);
-  cfg.dynamicSmemBytes = C::SMEM;
+  cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeClusterDimension;
@@ -965,23 +1114,33 @@ cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtenso
 template <bool BF16>
 cudaError_t launch_bn(const GemmGeom& g, int bn, const CUtensorMap* tmA, const CUtensorMap* tmB, const float* bias,
                       void* Y, cudaStream_t st) {
+  if (g.slab) {  // slab convolutions run on CTA pairs only
+    if (g.cg != 2) return cudaErrorInvalidValue;
+    switch (bn) {
+      case 96: return launch_inst<96, BF16, 2, true>(g, tmA, tmB, bias, Y, st);
+      case 128: return launch_inst<128, BF16, 2, true>(g, tmA, tmB, bias, Y, st);
+      case 192: return launch_inst<192, BF16, 2, true>(g, tmA, tmB, bias, Y, st);
+      case 256: return launch_inst<256, BF16, 2, true>(g, tmA, tmB, bias, Y, st);
+      default: return cudaErrorInvalidValue;
+    }
+  }
   if (g.cg == 2) {
     switch (bn) {
-      case 96: return launch_inst<96, BF16, 2>(g, tmA, tmB, bias, Y, st);
-      case 128: return launch_inst<128, BF16, 2>(g, tmA, tmB, bias, Y, st);
-      case 192: return launch_inst<192, BF16, 2>(g, tmA, tmB, bias, Y, st);
-      case 256: return launch_inst<256, BF16, 2>(g, tmA, tmB, bias, Y, st);
+      case 96: return launch_inst<96, BF16, 2, false>(g, tmA, tmB, bias, Y, st);
+      case 128: return launch_inst<128, BF16, 2, false>(g, tmA, tmB, bias, Y, st);
+      case 192: return launch_inst<192, BF16, 2, false>(g, tmA, tmB, bias, Y, st);
+      case 256: return launch_inst<256, BF16, 2, false>(g, tmA, tmB, bias, Y, st);
       default: return cudaErrorInvalidValue;
     }
   }
   switch (bn) {
-    case 16: return launch_inst<16, BF16, 1>(g, tmA, tmB, bias, Y, st);
-    case 32: return launch_inst<32, BF16, 1>(g, tmA, tmB, bias, Y, st);
-    case 64: return launch_inst<64, BF16, 1>(g, tmA, tmB, bias, Y, st);
-    case 96: return launch_inst<96, BF16, 1>(g, tmA, tmB, bias, Y, st);
-    case 128: return launch_inst<128, BF16, 1>(g, tmA, tmB, bias, Y, st);
-    case 192: return launch_inst<192, BF16, 1>(g, tmA, tmB, bias, Y, st);
-    case 256: return launch_inst<256, BF16, 1>(g, tmA, tmB, bias, Y, st);
+    case 16: return launch_inst<16, BF16, 1, false>(g, tmA, tmB, bias, Y, st);
+    case 32: return launch_inst<32, BF16, 1, false>(g, tmA, tmB, bias, Y, st);
+    case 64: return launch_inst<64, BF16, 1, false>(g, tmA, tmB, bias, Y, st);
+    case 96: return launch_inst<96, BF16, 1, false>(g, tmA, tmB, bias, Y, st);
+    case 128: return launch_inst<128, BF16, 1, false>(g, tmA, tmB, bias, Y, st);
+    case 192: return launch_inst<192, BF16, 1, false>(g, tmA, tmB, bias, Y, st);
+    case 256: return launch_inst<256, BF16, 1, false>(g, tmA, tmB, bias, Y, st);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -997,6 +1156,26 @@ int tc_num_sms() {
       g_num_sms = 148;
   }
   return g_num_sms;
+}
+
+bool tc_slab_config(GemmGeom& g, int bn) {
+  if (!g.slab || g.cg != 2 || g.Cgp % 64 || g.zf * bn > 256) return false;
+  int best = 0;
+  for (int st = 16; st >= 4 && !best; --st) {
+    GemmGeom t = g;
+    int smem;
+    switch (bn) {
+      case 96: smem = slab_smem<96, 2>(t, st); break;
+      case 128: smem = slab_smem<128, 2>(t, st); break;
+      case 192: smem = slab_smem<192, 2>(t, st); break;
+      case 256: smem = slab_smem<256, 2>(t, st); break;
+      default: return false;
+    }
+    if (smem <= SLAB_SMEM_MAX) best = st;
+  }
+  if (!best) return false;
+  g.stages = best;
+  return true;
 }
 
 int tc_pick_cg(const GemmGeom& g, int bn) {

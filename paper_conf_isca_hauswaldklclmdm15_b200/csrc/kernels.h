@@ -59,6 +59,15 @@ struct GemmGeom {
   int bx, by, bn;     // conv: output-pixel block of one M tile (bx*by*bn == 128), x fastest
   int zf;             // z values fused per CTA (groups computed by one CTA; TMEM columns zf*BN)
   int epi_lrn;        // 1: Caffe LRN across the zf*N channels of a pixel in the epilogue
+  // slab convolution (stride 1, 64-channel chunks): GEMM row m = virtual pixel of the stored
+  // (bordered) input grid Hv x Wv, m = (img * Hv + y) * Wv + x; a tile's rows read ONE
+  // contiguous slab of input pixels [m0, m0 + 128 + (KH-1)*Wv + KW-1) loaded once by TMA, and
+  // filter tap (ky, kx) is the UMMA A descriptor shifted by ky*Wv + kx rows.  Rows with
+  // y >= OH or x >= OWb are computed and discarded.
+  int slab, Hv, Wv;
+  int slab_parts, slab_rows;  // the slab is loaded as slab_parts TMA boxes of slab_rows rows
+  int stages;         // slab mode: B ring stages (runtime; set by tc_slab_config)
+  int obd;            // conv output: zero border of the stored output tensor (its consumer's pad)
   int lrn_size;
   float lrn_alpha_over_n, lrn_beta, lrn_k;
 };
@@ -87,6 +96,8 @@ cudaError_t launch_simt_gemm(const GemmGeom& g, const float* A, const float* B, 
 int tc_pick_bn(const GemmGeom& g);
 int tc_pick_cg(const GemmGeom& g, int bn);  // 2 when a CTA pair (cta_group::2) pays off
 int tc_num_sms();
+// Slab mode feasibility for tile width bn (CTA pair): sets g.stages; false = use im2col.
+bool tc_slab_config(GemmGeom& g, int bn);
 cudaError_t launch_tc_gemm(const GemmGeom& g, int bn, int dt, const CUtensorMap* tmA,
                            const CUtensorMap* tmB, const float* bias, void* Y, cudaStream_t st);
 
@@ -96,10 +107,11 @@ cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, in
                        float alpha, float beta, float k, int dt, cudaStream_t st);
 
 // --- MAX pooling with a channel-layout change (plain/grouped in, plain/grouped/x-unrolled out), 16-bit,
-// kernel <= stride + 1.
+// kernel <= stride + 1.  obd: zero border of the stored output ((OH+2obd) x (OW+2obd) pixels;
+// the border is never written).
 cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int Cpi, int gsz_i, int gpitch_i, int H,
                               int W, int OH, int OW, int kernel, int stride, int pad, int Cpo, int gsz_o, int gpitch_o,
-                              int xu, int dt, cudaStream_t st);
+                              int xu, int obd, int dt, cudaStream_t st);
 
 // --- LRN + max pooling fused (K4+K5): fp16 NHWC input (pitch Cpi, C channels, pads zero),
 // Caffe LRN across channels in fp32, Caffe MAX pooling of the LRN output (kernel 1 = no pool),

@@ -258,16 +258,28 @@ void Net::build(const std::string& desc) {
   // each group at a pitch of 16/32/64 (<= 64 channels) or a multiple of 64, i.e. one TMA row
   // of 32/64/128 B per tap and chunk.  fp32 path: dense channels.
   auto tap_pitch = [](int c) { return c <= 16 ? 16 : c <= 32 ? 32 : rup(c, 64); };
+  // A slab convolution (stride 1, every group's channel pitch a multiple of 64) reads its zero
+  // padding from memory: its input is stored with a border of `pad` zero pixels (DESIGN.md
+  // sec 4).  DJINN_SLAB=0 turns slab mode off (im2col TMA for every conv).
+  const char* slab_env = getenv("DJINN_SLAB");
+  const bool slab_on = f16 && !(slab_env && slab_env[0] == '0');
+  auto slab_border = [&](const LayerSpec& L, const Shape& sh) {
+    const int gp = sh.gsz < sh.C ? sh.gpitch : sh.Cp;
+    return (slab_on && L.stride == 1 && L.pad > 0 && gp % 64 == 0) ? L.pad : 0;
+  };
   auto layout_for = [&](size_t from, Shape sh) {
     sh.Cp = sh.C;
     sh.gsz = sh.gpitch = 1 << 30;
+    sh.bdr = 0;
     if (!f16) return sh;
     sh.Cp = rup(sh.C, 16);
+    bool border_ok = true;  // only a convolution reading the tensor directly may get a border
     for (size_t j = from; j < layers.size(); ++j) {
       const LayerSpec& L = layers[j];
       // a MAX pool the column kernel handles re-lays the channels itself: its producer
       // writes the plain pitch (no grouped-layout padding read back by the pool)
       if (L.type == "Pooling" && L.pool_max && L.kernel <= L.stride + 1) return sh;
+      if (L.type == "Pooling" || L.type == "LRN") border_ok = false;
       if (L.type == "Convolution" && L.group > 1 && sh.C % L.group == 0) {
         const int cg = sh.C / L.group;
         if (cg % 16 == 0) {
@@ -275,15 +287,26 @@ void Net::build(const std::string& desc) {
           sh.gpitch = tap_pitch(cg);
           sh.Cp = L.group * sh.gpitch;
         }
+        if (border_ok) sh.bdr = slab_border(L, sh);
         return sh;
       }
       if (L.type == "Convolution" || L.type == "LocallyConnected") {
         sh.Cp = tap_pitch(sh.C);
+        if (border_ok && L.type == "Convolution") sh.bdr = slab_border(L, sh);
         return sh;
       }
       if (L.type == "InnerProduct" || L.type == "Softmax") return sh;
     }
     return sh;
+  };
+  // output buffer of a new tensor: the free ping-pong buffer, or a dedicated one for a bordered
+  // tensor (its border is zeroed once at workspace creation and never written)
+  auto pick_buf = [&](const Shape& sh, int cur_buf) {
+    if (sh.bdr > 0) {
+      buf_bytes.push_back(0);
+      return (int)buf_bytes.size() - 1;
+    }
+    return cur_buf == 0 ? 1 : 0;
   };
   const std::vector<int>& d = layers[0].dims;
   Shape cur;
@@ -292,6 +315,7 @@ void Net::build(const std::string& desc) {
   else throw Error(DJINN_E_SHAPE, "Input must have 1 or 3 dims");
   if (cur.C <= 0 || cur.H <= 0 || cur.W <= 0) throw Error(DJINN_E_SHAPE, "bad Input dims");
   cur = layout_for(1, cur);
+  cur.bdr = 0;  // the pack writes no border (a padded first conv then runs on im2col TMA)
   if (cur.gsz < cur.C) throw Error(DJINN_E_UNSUPPORTED, "grouped first convolution on a 16-bit path");
   in_elems = (int64_t)cur.C * cur.H * cur.W;
 
@@ -331,8 +355,9 @@ void Net::build(const std::string& desc) {
       o.kind = OP_LRN;
       o.name = L.name;
       o.in = o.out = cur;
+      if (cur.bdr) throw Error(DJINN_E_UNSUPPORTED, L.name + ": internal: LRN over a bordered tensor");
       o.in_buf = curbuf;
-      o.out_buf = curbuf = 1 - curbuf;
+      o.out_buf = curbuf = pick_buf(o.out, curbuf);
       o.lrn_size = L.lrn_size;
       o.alpha = L.alpha;
       o.beta = L.beta;
@@ -359,12 +384,13 @@ void Net::build(const std::string& desc) {
       o.out.W = pout(cur.W);
       o.out = layout_for(i + 1, o.out);
       if (!(f16 && L.pool_max && L.kernel <= L.stride + 1)) o.out = Shape{cur.C, o.out.H, o.out.W, cur.Cp, cur.gsz, cur.gpitch, 1, 0};
+      if (cur.bdr) throw Error(DJINN_E_UNSUPPORTED, L.name + ": internal: pooling over a bordered tensor");
       o.kernel = L.kernel;
       o.stride = L.stride;
       o.pad = L.pad;
       o.is_max = L.pool_max;
       o.in_buf = curbuf;
-      o.out_buf = curbuf = 1 - curbuf;
+      o.out_buf = curbuf = pick_buf(o.out, curbuf);
       cur = o.out;
       ops.push_back(o);
       continue;
@@ -539,6 +565,27 @@ void Net::build(const std::string& desc) {
       // the least padding waste for this layer's OW x OH x batch.
       const char* amode = getenv("DJINN_CONV_A");
       g.a_tiled = (!lc && amode && strcmp(amode, "tiled") == 0) ? 1 : 0;
+      // Slab convolution: the input's zero padding is stored (border == pad), so the conv is a
+      // pad-0 conv over the stored Hv x Wv grid and every tap of a 128-row tile is a row shift
+      // of one contiguous run of input pixels (one TMA slab per tile instead of KH*KW im2col
+      // boxes: the operand stream through L2 drops ~KH*KW-fold).  Rows are virtual pixels of
+      // the stored grid; the ones outside OH x OWb are computed and discarded.
+      if (slab_on && !lc && !g.a_tiled && g.stride == 1 && g.kxs == 1 && g.Cgp % 64 == 0 && o.in.bdr == g.pad) {
+        const int Hv = o.in.H + 2 * o.in.bdr, Wv = o.in.W + 2 * o.in.bdr;
+        const int R = 128 + (g.KH - 1) * Wv + (g.KW - 1);
+        if (R <= 512) {
+          g.slab = 1;
+          g.Hv = Hv; g.Wv = Wv;
+          g.H = Hv; g.W = Wv; g.pad = 0;  // (also valid for an im2col fallback over the stored grid)
+          g.slab_parts = (R + 255) / 256;
+          g.slab_rows = rup((R + g.slab_parts - 1) / g.slab_parts, 8);
+          o.ohw = Hv * Wv;
+        }
+      }
+      if (!g.slab && o.in.bdr > 0) {  // a bordered input read by im2col: pad-0 conv over the stored grid
+        if (o.in.bdr > g.pad) throw Error(DJINN_E_SHAPE, L.name + ": internal: input border exceeds the padding");
+        g.H = o.in.H + 2 * o.in.bdr; g.W = o.in.W + 2 * o.in.bdr; g.pad -= o.in.bdr;
+      }
       if (!lc) {
         double best = 1e30;
         for (int bx = 1; bx <= 128; bx *= 2)
@@ -615,7 +662,9 @@ void Net::build(const std::string& desc) {
     }
     g.Kpad = f16 ? rup(g.K, 64) : g.K;
     g.out_f32 = last ? 1 : 0;
-    o.out_buf = last ? 2 : 1 - curbuf;
+    if (o.out.bdr && g.mode != GM_CONV) throw Error(DJINN_E_UNSUPPORTED, L.name + ": internal: bordered output");
+    g.obd = o.out.bdr;
+    o.out_buf = last ? 2 : pick_buf(o.out, curbuf);
     if (!last) curbuf = o.out_buf;
     if (last) out_pitch = o.out.Cp;
     o.bn = f16 ? 0 : 64;
@@ -663,7 +712,9 @@ void Net::build(const std::string& desc) {
       os = layout_for(i + 1, os);
       lp.out = os;
       lp.in_buf = o.out_buf;
-      lp.out_buf = curbuf = 1 - o.out_buf;
+      os.bdr = 0;  // the fused LRN + pool kernel writes no border
+      lp.out = os;
+      lp.out_buf = curbuf = pick_buf(os, o.out_buf);
       cur = os;
       ops.push_back(lp);
     }
@@ -715,6 +766,23 @@ void Net::build(const std::string& desc) {
 }
 
 // ============================================================================ weights
+// Tile width / CTA pairing per GEMM, and slab-mode shared memory (falls back to im2col TMA
+// over the stored grid when the slab does not fit).
+void Net::choose_tiles() {
+  if (dt == DT_F32) return;
+  for (Op& o : ops) {
+    if (o.kind != OP_GEMM) continue;
+    GemmGeom g = o.g;
+    g.M = (int)(max_rows * o.ohw);
+    o.bn = tc_pick_bn(g);
+    o.g.cg = tc_pick_cg(g, o.bn);
+    if (o.g.slab && !tc_slab_config(o.g, o.bn)) {
+      o.g.slab = 0;
+      o.ohw = o.g.OH * o.g.OWb;
+    }
+  }
+}
+
 void Net::load_weights(const float* w, size_t n, int mem) {
   const bool f16 = dt != DT_F32;
   if (n != (size_t)n_params)
@@ -839,7 +907,8 @@ Workspace* Net::workspace(cudaStream_t st) {
   auto it = ws.find(st);
   if (it != ws.end()) return it->second.get();
   std::unique_ptr<Workspace> w(new Workspace);
-  for (int b = 0; b < 3; ++b) {
+  w->buf.assign(buf_bytes.size(), nullptr);
+  for (size_t b = 0; b < buf_bytes.size(); ++b) {
     if (!buf_bytes[b]) continue;
     if (cudaMalloc(&w->buf[b], buf_bytes[b]) != cudaSuccess) throw Error(DJINN_E_NOMEM, "workspace allocation");
     ck(cudaMemset(w->buf[b], 0, buf_bytes[b]), "workspace memset");
@@ -860,7 +929,13 @@ Workspace* Net::workspace(cudaStream_t st) {
       // NHWC input [max_rows][H][W][Cp] viewed as a 4D tensor {C, W, H, N}
       uint64_t dims[4] = {(uint64_t)g.Cp_in, (uint64_t)g.W, (uint64_t)g.H, (uint64_t)max_rows};
       uint64_t strides[3] = {(uint64_t)g.Cp_in * 2, (uint64_t)g.W * g.Cp_in * 2, (uint64_t)g.H * g.W * g.Cp_in * 2};
-      if (g.mode == GM_CONV && g.a_tiled) {
+      if (g.mode == GM_CONV && g.slab) {
+        // slab: the stored input as [rows * Hv * Wv][Cp] pixels; box {64 channels, slab_rows}
+        uint64_t d2[2] = {(uint64_t)g.Cp_in, (uint64_t)max_rows * g.Hv * g.Wv};
+        uint64_t s2[1] = {(uint64_t)g.Cp_in * 2};
+        uint32_t box[2] = {64, (uint32_t)g.slab_rows};
+        encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 2, d2, s2, box);
+      } else if (g.mode == GM_CONV && g.a_tiled) {
         uint32_t box[4] = {(uint32_t)g.cw, (uint32_t)(g.bx * g.stride), (uint32_t)(g.by * g.stride), (uint32_t)g.bn};
         const uint32_t estr[4] = {1, (uint32_t)g.stride, (uint32_t)g.stride, 1};
         encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 4, dims, strides, box, g.cw * 2, estr);
@@ -947,7 +1022,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           if (dt != DT_F32 && o.is_max && o.kernel <= o.stride + 1)
             e = launch_pool_remap(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.gsz, o.in.gpitch,
                                   o.in.H, o.in.W, o.out.H, o.out.W, o.kernel, o.stride, o.pad, o.out.Cp, o.out.gsz,
-                                  o.out.gpitch, o.out.xu, dt, st);
+                                  o.out.gpitch, o.out.xu, o.out.bdr, dt, st);
           else
             e = launch_pool(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.H, o.in.W, o.out.H, o.out.W,
                             o.kernel, o.stride, o.pad, o.is_max, o.out.xu, dt, st);
@@ -983,12 +1058,17 @@ std::string Net::plan_string() const {
     << max_rows << " arena " << arena_bytes << " B params " << n_params << "\n";
   for (const Op& o : ops) {
     s << "  " << kinds[o.kind] << " " << o.name << " in " << o.in.C << "x" << o.in.H << "x" << o.in.W << "/p" << o.in.Cp
-      << " -> " << o.out.C << "x" << o.out.H << "x" << o.out.W << "/p" << o.out.Cp << " buf " << o.in_buf << "->"
+      << (o.in.bdr ? "+b" + std::to_string(o.in.bdr) : std::string())
+      << " -> " << o.out.C << "x" << o.out.H << "x" << o.out.W << "/p" << o.out.Cp
+      << (o.out.bdr ? "+b" + std::to_string(o.out.bdr) : std::string()) << " buf " << o.in_buf << "->"
       << o.out_buf;
     if (o.kind == OP_GEMM)
       s << " [" << modes[o.g.mode] << " N=" << o.g.N << " Z=" << o.g.Z << " K=" << o.g.K << " Kpad=" << o.g.Kpad
         << " act=" << o.g.act << " bn=" << o.bn << " cg=" << o.g.cg << " cw=" << o.g.cw << " zf=" << o.g.zf << " KHxKW=" << o.g.KH << "x"
         << o.g.KW << (o.g.xb > 1 ? " xblock=" + std::to_string(o.g.xb) : std::string())
+        << (o.g.slab ? " slab=" + std::to_string(o.g.Hv) + "x" + std::to_string(o.g.Wv) + ":" + std::to_string(o.g.slab_parts) + "x" +
+                           std::to_string(o.g.slab_rows) + " stages=" + std::to_string(o.g.stages)
+                     : std::string())
         << (o.g.kxs > 1 ? " x-unrolled-input=" + std::to_string(o.g.kxs) : std::string())
         << (o.g.lcg > 1 ? " taps/row=" + std::to_string(o.g.lcg) : std::string())
         << (o.g.mode == GM_CONV && o.g.a_tiled ? " block=" + std::to_string(o.g.bx) + "x" + std::to_string(o.g.by) + "x" +

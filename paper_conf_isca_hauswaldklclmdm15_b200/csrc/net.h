@@ -52,7 +52,9 @@ struct Shape {
   int C = 0, H = 1, W = 1, Cp = 0;
   int gsz = 1 << 30, gpitch = 1 << 30;
   int xu = 1, P = 0;  // x-unrolled layout: pixel x stores pixels x..x+xu-1, each at pitch P (Cp = xu*P)
-  int64_t per_row() const { return (int64_t)H * W * Cp; }
+  int bdr = 0;        // zero border: stored (H + 2 bdr) x (W + 2 bdr) pixels, pixel (y, x) at (y + bdr, x + bdr)
+                      // (the input of a slab convolution: its zero padding is stored)
+  int64_t per_row() const { return (int64_t)(H + 2 * bdr) * (W + 2 * bdr) * Cp; }
   int pos(int c) const { return (c / gsz) * gpitch + c % gsz; }
 };
 
@@ -60,7 +62,7 @@ struct Op {
   OpKind kind;
   std::string name;
   Shape in, out;
-  int in_buf = 0, out_buf = 0;  // 0/1 ping-pong, 2 logits, -1 external input
+  int in_buf = 0, out_buf = 0;  // 0/1 ping-pong, 2 logits, 3.. dedicated (bordered), -1 external input
   // gemm
   GemmGeom g{};
   int bn = 0;
@@ -88,7 +90,7 @@ struct ProfRec {  // one timed forward chunk: events[first .. first + n_ops]
 };
 
 struct Workspace {
-  void* buf[3] = {nullptr, nullptr, nullptr};
+  std::vector<void*> buf;  // 0/1 ping-pong, 2 logits, 3.. dedicated bordered tensors (borders stay zero)
   float* in_stage = nullptr;
   void* out_stage = nullptr;
   std::vector<CUtensorMap> tmA;  // per op (dense gemm) over its input buffer
@@ -108,7 +110,7 @@ struct Net {
   int out_pitch = 0;  // logits pitch
   void* arena = nullptr;
   size_t arena_bytes = 0;
-  size_t buf_bytes[3] = {0, 0, 0};
+  std::vector<size_t> buf_bytes = std::vector<size_t>(3, 0);
   std::mutex mu;
   std::map<cudaStream_t, std::unique_ptr<Workspace>> ws;
   bool poisoned = false;
@@ -122,6 +124,7 @@ struct Net {
   ~Net();
 
   void build(const std::string& desc);                          // parse + plan
+  void choose_tiles();                                          // tile widths, CTA pairs, slab smem
   void load_weights(const float* w, size_t n, int mem);         // pack into the arena
   Workspace* workspace(cudaStream_t st);
   void forward(const float* in, int64_t rows, int in_mem, void* out, int out_mem, int mode,
