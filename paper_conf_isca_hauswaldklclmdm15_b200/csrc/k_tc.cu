@@ -101,6 +101,15 @@ __device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
     if (++iters > (1u << 24)) __trap();  // a lost arrival must fault, never hang the GPU
   } while (!done);
 }
+// Loaders' stage waits: spin (the default) -- a suspended waiter's wake-up latency was starving
+// the MMA of re-armed stages; DJINN_LOADER_SLEEP builds the sleeping variant for comparison.
+__device__ __forceinline__ void mbar_wait_ld(uint32_t bar, uint32_t parity) {
+#ifdef DJINN_LOADER_SLEEP
+  mbar_wait_sleep(bar, parity);
+#else
+  mbar_wait(bar, parity);
+#endif
+}
 __device__ __forceinline__ void tma_2d(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1) {
   asm volatile(
       "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
@@ -443,11 +452,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   // non-slab: [A ring][B ring][bars];  slab: [B ring][2 slabs][bars]
   const int NST = SLAB ? g.stages : C::STAGES;  // ring stages
+  // slab mode: a stage holds KPS consecutive K blocks of B (one commit per KPS*4 MMAs: a
+  // tcgen05.commit costs ~400 cycles of pipe time, tools/mma_cg2_bench.cu)
+  const int KPS = SLAB ? g.kps : 1;
+  const int SB_BYTES = KPS * C::B_BYTES;  // bytes of one ring stage of B
   const uint32_t slab_chunk = SLAB ? (uint32_t)(g.slab_parts * g.slab_rows * 128) : 0u;  // one 64-channel chunk
   const uint32_t slab_bytes = SLAB ? (uint32_t)(g.zf * (g.Cgp / 64)) * slab_chunk : 0u;
   uint8_t* sA = smem;
   uint8_t* sB = SLAB ? smem : smem + C::STAGES * C::A_BYTES;
-  uint8_t* sSlab = smem + ((NST * C::B_BYTES + 1023) & ~1023);
+  uint8_t* sSlab = smem + ((NST * SB_BYTES + 1023) & ~1023);
   uint64_t* bars = SLAB ? reinterpret_cast<uint64_t*>(sSlab + 2 * slab_bytes)
                         : reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
   // bars: full[NST], empty[NST], tfull[2], tempty[2], sfull[2], sempty[2]
@@ -524,7 +537,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
     const int bn_off = (int)rank * (BN / CG);
     const bool leader = elect_one();
-    const uint32_t tx_bytes = SLAB ? CG * C::B_BYTES : CG * (C::A_BYTES + (kDbgNoB ? 0 : C::B_BYTES));
+    const uint32_t tx_bytes = CG * ((SLAB ? 0 : C::A_BYTES) + (kDbgNoB ? 0 : C::B_BYTES));
     const int nown = SLAB ? NLOAD - 1 : NLOAD, myq = SLAB ? li - 1 : li;  // stage owner index
     int s = 0, qo = 0;  // ring slot; owner of the current stage (q % nown)
     uint32_t ph = 0;
@@ -567,22 +580,31 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         STAT_ADD(st_prod_issue);
       }
     } else if (SLAB) {
-      // B-only stages of the slab mode
+      // B-only stages of the slab mode: KPS K blocks (steps u = zi * num_kb + kb) per stage
+      const int nsteps = zf * num_kb;
       for (int t = cid; t < tiles; t += ncl) {
         const TileCoord tc = warp_uniform(tile_coord(g, t, mt, nt, CG));
-        for (int zi = 0; zi < zf; ++zi) {
-          const int z = tc.z0 * zf + zi;
-          for (int kb = 0; kb < num_kb; ++kb) {
-            if (qo == myq) {
-              mbar_wait_sleep(empty0 + 8 * s, ph ^ 1);
-              if (leader) {
-                if (rank == 0) mbar_arrive_expect_tx(full0 + 8 * s, tx_bytes);
-                load_b(full0 + 8 * s, kb, tc.n0, z);
+        int zi = 0, kb = 0;  // step counters
+        for (int u0 = 0; u0 < nsteps; u0 += KPS) {
+          const int cnt = min(KPS, nsteps - u0);
+          if (qo == myq) {
+            mbar_wait_ld(empty0 + 8 * s, ph ^ 1);
+            if (leader) {
+              const uint32_t fb = full0 + 8 * s;
+              if (rank == 0) mbar_arrive_expect_tx(fb, kDbgNoB ? 0u : (uint32_t)(CG * C::B_BYTES * cnt));
+              int zz = zi, kk = kb;
+              for (int i = 0; i < cnt; ++i) {
+                if (!kDbgNoB)
+                  tma_a3<CG>(sB0 + (uint32_t)(s * SB_BYTES + i * C::B_BYTES), &tmB, fb, kk * BK, tc.n0 * BN + bn_off,
+                             tc.z0 * zf + zz);
+                if (++kk == num_kb) { kk = 0; ++zz; }
               }
-              __syncwarp();
             }
-            next_stage();
+            __syncwarp();
           }
+          for (int i = 0; i < cnt; ++i)
+            if (++kb == num_kb) { kb = 0; ++zi; }
+          next_stage();
         }
       }
     } else if (mode == GM_CONV && !a_tiled && nq <= KTAB_MAX) {
@@ -617,7 +639,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             if (qo == myq) {
               {
                 STAT_T0();
-                mbar_wait_sleep(empty0 + 8 * s, ph ^ 1);
+                mbar_wait_ld(empty0 + 8 * s, ph ^ 1);
                 STAT_ADD(st_prod_wait);
               }
               STAT_T0();
@@ -675,7 +697,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           if (mine) {
             {
               STAT_T0();
-              mbar_wait_sleep(empty0 + 8 * s, ph ^ 1);
+              mbar_wait_ld(empty0 + 8 * s, ph ^ 1);
               STAT_ADD(st_prod_wait);
             }
             if (leader) {
@@ -740,6 +762,19 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       }
       const uint64_t a_hi = sdesc(0, SLAB ? 128 : cw * 2), b_hi = sdesc(0, 128);
       const uint32_t sA0 = (smem_u32(sA) & 0x3FFFFu) >> 4, sB0 = (smem_u32(sB) & 0x3FFFFu) >> 4;
+      // slab mode: per step u = zi * num_kb + kb, the A row offset within the slab (16-B units)
+      const int nsteps = g.zf * num_kb;
+      const uint32_t slab_s16 = (smem_u32(sSlab) & 0x3FFFFu) >> 4;
+      if (SLAB) {
+        const int nchunk = g.Cgp / 64;
+        for (int u = lane; u < nsteps; u += 32) {
+          const int zi = u / num_kb, kb = u - zi * num_kb, tap = kb / nchunk, j = kb - tap * nchunk;
+          const int ky = tap / g.KW, kx = tap - ky * g.KW;
+          const uint32_t off = (uint32_t)((zi * nchunk + j) * (int)(slab_chunk >> 4)) + (uint32_t)((ky * g.Wv + kx) * 8);
+          ktab[u] = off | (kb == 0 ? (1u << 22) : 0u) | ((uint32_t)zi << 24);
+        }
+        __syncwarp();
+      }
       int s = 0, lt = 0;
       uint32_t ph = 0;
       for (int t = cid; t < tiles; t += ncl, ++lt) {
@@ -754,7 +789,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         if (SLAB) {
           // taps are row shifts of the tile's slab: A(tap) = slab chunk + (ky*Wv + kx) rows
           // (the 128B swizzle is address-based: a start 128*r bytes into a 1024-aligned atom
-          // reads rows r.. correctly; tools/umma_shift_test.cu)
+          // reads rows r.. correctly; tools/umma_shift_test.cu).  The issue loop is kept lean --
+          // the tensor pipe finishes an N=96..128 MMA in 52..64 cycles, so per-stage bookkeeping
+          // was idling it (tools/mma_cg2_bench.cu): the A offset / z slice of every step comes
+          // from the table built below.
           const int sb = lt & 1;
           {
             STAT_T0();
@@ -762,40 +800,37 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             STAT_ADD(st_mma_full);
           }
           tc_fence_after();
-          const int nchunk = g.Cgp / 64, Wv = g.Wv, KW = g.KW;
-          const uint32_t slabS = ((smem_u32(sSlab) & 0x3FFFFu) >> 4) + (uint32_t)sb * (slab_bytes >> 4);
-          for (int zi = 0; zi < g.zf; ++zi) {
-            const uint32_t d = tmem + (uint32_t)(slot * slot_cols + zi * BN);
-            int j = 0, kx = 0, ky = 0;
-            for (int kb = 0; kb < num_kb; ++kb) {
-              {
-                STAT_T0();
-                mbar_wait(full0 + 8 * s, ph);
-                STAT_ADD(st_mma_full);
-              }
-              tc_fence_after();
+          const uint32_t abase = slab_s16 + (uint32_t)sb * (slab_bytes >> 4);
+          const uint32_t dbase = tmem + (uint32_t)(slot * slot_cols);
+          for (int u0 = 0; u0 < nsteps; u0 += KPS) {
+            const int cnt = min(KPS, nsteps - u0);
+            {
               STAT_T0();
-              if (elect_one()) {
-                const uint32_t arow = slabS + (uint32_t)((zi * nchunk + j) * (int)(slab_chunk >> 4)) +
-                                      (uint32_t)((ky * Wv + kx) * 8);
-                const uint64_t ad = a_hi | (uint64_t)arow;
-                const uint64_t bd = b_hi | (uint64_t)(sB0 + (uint32_t)s * (C::B_BYTES >> 4));
-#pragma unroll
-                for (int k = 0; k < BK / 16; ++k) {
-                  if (CG == 2) mma_f16_2sm(d, ad + 2 * k, bd + 2 * k, idesc, (kb | k) != 0);
-                  else mma_f16(d, ad + 2 * k, bd + 2 * k, idesc, (kb | k) != 0);
-                }
-                if (CG == 2) mma_commit_2sm(empty0 + 8 * s);
-                else mma_commit(empty0 + 8 * s);
-              }
-              __syncwarp();
-              STAT_ADD(st_mma_issue);
-              if (++j == nchunk) {
-                j = 0;
-                if (++kx == KW) { kx = 0; ++ky; }
-              }
-              if (++s == NST) { s = 0; ph ^= 1; }
+              mbar_wait(full0 + 8 * s, ph);
+              STAT_ADD(st_mma_full);
             }
+            tc_fence_after();
+            STAT_T0();
+            if (elect_one()) {
+              const uint32_t bstage = sB0 + (uint32_t)s * (uint32_t)(SB_BYTES >> 4);
+              for (int i = 0; i < cnt; ++i) {
+                const uint32_t e = ktab[u0 + i];  // bits 0-21: A offset (16 B), 22: first K step of its z, 24-31: z slice
+                const uint32_t d = dbase + (e >> 24) * BN;
+                const uint64_t ad = a_hi | (uint64_t)(abase + (e & 0x3FFFFFu));
+                const uint64_t bd = b_hi | (uint64_t)(bstage + (uint32_t)i * (C::B_BYTES >> 4));
+                const uint32_t acc0 = (e >> 22) & 1u ? 0u : 1u;
+#pragma unroll
+                for (int k = 0; k < (kDbgNoMma ? 0 : BK / 16); ++k) {
+                  if (CG == 2) mma_f16_2sm(d, ad + 2 * k, bd + 2 * k, idesc, k ? 1u : acc0);
+                  else mma_f16(d, ad + 2 * k, bd + 2 * k, idesc, k ? 1u : acc0);
+                }
+              }
+              if (CG == 2) mma_commit_2sm(empty0 + 8 * s);
+              else mma_commit(empty0 + 8 * s);
+            }
+            __syncwarp();
+            STAT_ADD(st_mma_issue);
+            if (++s == NST) { s = 0; ph ^= 1; }
           }
           if (elect_one()) {
             if (CG == 2) { mma_commit_2sm(tfull0 + 8 * slot); mma_commit_2sm(sempty0 + 8 * sb); }
@@ -1070,7 +1105,7 @@ constexpr int SLAB_SMEM_MAX = 227 * 1024 - 1024;  // 227 KB per block minus the 
 template <int BN, int CG>
 int slab_smem(const GemmGeom& g, int stages) {
   using C = Cfg<BN, CG>;
-  const int ring = (stages * C::B_BYTES + 1023) & ~1023;
+  const int ring = (stages * g.kps * C::B_BYTES + 1023) & ~1023;
   const int slab = g.zf * (g.Cgp / 64) * g.slab_parts * g.slab_rows * 128;
   return 1024 + ring + 2 * slab + (2 * stages + 8) * 8 + 16;
 }
@@ -1159,23 +1194,31 @@ int tc_num_sms() {
 }
 
 bool tc_slab_config(GemmGeom& g, int bn) {
-  if (!g.slab || g.cg != 2 || g.Cgp % 64 || g.zf * bn > 256) return false;
-  int best = 0;
-  for (int st = 16; st >= 4 && !best; --st) {
-    GemmGeom t = g;
-    int smem;
-    switch (bn) {
-      case 96: smem = slab_smem<96, 2>(t, st); break;
-      case 128: smem = slab_smem<128, 2>(t, st); break;
-      case 192: smem = slab_smem<192, 2>(t, st); break;
-      case 256: smem = slab_smem<256, 2>(t, st); break;
-      default: return false;
+  if (!g.slab || g.cg != 2 || g.Cgp % 64 || g.zf * bn > 256 || g.zf * (g.Kpad / BK) > KTAB_MAX) return false;
+  // largest K blocks per stage (fewest commits) that still leaves a ring of >= 3 stages
+  // (kps 1 = a commit every 4 MMAs idles the tensor pipe: im2col is then faster, e.g. IMC conv3)
+  for (int kps : {4, 2}) {
+    int best = 0;
+    for (int st = 16; st >= 3 && !best; --st) {
+      GemmGeom t = g;
+      t.kps = kps;
+      int smem;
+      switch (bn) {
+        case 96: smem = slab_smem<96, 2>(t, st); break;
+        case 128: smem = slab_smem<128, 2>(t, st); break;
+        case 192: smem = slab_smem<192, 2>(t, st); break;
+        case 256: smem = slab_smem<256, 2>(t, st); break;
+        default: return false;
+      }
+      if (smem <= SLAB_SMEM_MAX) best = st;
     }
-    if (smem <= SLAB_SMEM_MAX) best = st;
+    if (best) {
+      g.kps = kps;
+      g.stages = best;
+      return true;
+    }
   }
-  if (!best) return false;
-  g.stages = best;
-  return true;
+  return false;
 }
 
 int tc_pick_cg(const GemmGeom& g, int bn) {

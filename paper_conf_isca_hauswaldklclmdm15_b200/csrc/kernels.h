@@ -67,6 +67,7 @@ struct GemmGeom {
   int slab, Hv, Wv;
   int slab_parts, slab_rows;  // the slab is loaded as slab_parts TMA boxes of slab_rows rows
   int stages;         // slab mode: B ring stages (runtime; set by tc_slab_config)
+  int kps;            // slab mode: K blocks of B per ring stage (one MMA commit per stage)
   int obd;            // conv output: zero border of the stored output tensor (its consumer's pad)
   int lrn_size;
   float lrn_alpha_over_n, lrn_beta, lrn_k;

@@ -1067,7 +1067,7 @@ std::string Net::plan_string() const {
         << " act=" << o.g.act << " bn=" << o.bn << " cg=" << o.g.cg << " cw=" << o.g.cw << " zf=" << o.g.zf << " KHxKW=" << o.g.KH << "x"
         << o.g.KW << (o.g.xb > 1 ? " xblock=" + std::to_string(o.g.xb) : std::string())
         << (o.g.slab ? " slab=" + std::to_string(o.g.Hv) + "x" + std::to_string(o.g.Wv) + ":" + std::to_string(o.g.slab_parts) + "x" +
-                           std::to_string(o.g.slab_rows) + " stages=" + std::to_string(o.g.stages)
+                           std::to_string(o.g.slab_rows) + " stages=" + std::to_string(o.g.stages) + "x" + std::to_string(o.g.kps)
                      : std::string())
         << (o.g.kxs > 1 ? " x-unrolled-input=" + std::to_string(o.g.kxs) : std::string())
         << (o.g.lcg > 1 ? " taps/row=" + std::to_string(o.g.lcg) : std::string())
