@@ -152,7 +152,9 @@ DJINN_API int djinn_plan_info(const djinn_net* net, char* buf, size_t cap);
 /* djinn_profile -- enable (1) / disable (0) per-op device timing of subsequent
  * djinn_forward calls on this net: a CUDA event is recorded on the forward's stream
  * before each kernel and after the last one (PAPER.md L151-173 profiles per kernel,
- * weighted by kernel time).  Enabling clears earlier records. */
+ * weighted by kernel time).  enable = 2 + k times plan op k only (one event before and
+ * one after its kernel; the rest of the forward keeps its programmatic-launch overlap).
+ * Enabling clears earlier records.  k out of range: DJINN_E_INVAL. */
 DJINN_API int djinn_profile(djinn_net* net, int enable);
 
 /* djinn_profile_read -- synchronise the recorded events and return, per op of the plan

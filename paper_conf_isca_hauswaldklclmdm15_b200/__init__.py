@@ -133,8 +133,9 @@ def djinn_plan_info(net: int) -> str:
     return buf.value.decode()
 
 
-def djinn_profile(net: int, enable: bool) -> None:
-    _check(lib().djinn_profile(net, 1 if enable else 0))
+def djinn_profile(net: int, enable: bool, op: Optional[int] = None) -> None:
+    """Per-op device timing on/off; ``op`` = time that plan op only."""
+    _check(lib().djinn_profile(net, 0 if not enable else (1 if op is None else 2 + int(op))))
 
 
 def djinn_profile_read(net: int, reset: bool = True):

@@ -179,7 +179,9 @@ int djinn_profile(djinn_net* net, int enable) {
     if (!net) return fail(DJINN_E_INVAL, "net is NULL");
     std::lock_guard<std::mutex> lk(net->impl.mu);
     net->impl.prof_clear();
+    if (enable >= 2 && enable - 2 >= (int)net->impl.ops.size()) return fail(DJINN_E_INVAL, "profile op out of range");
     net->impl.profile = enable != 0;
+    net->impl.profile_op = enable >= 2 ? enable - 2 : -1;
     return DJINN_OK;
   });
 }
@@ -200,8 +202,9 @@ int djinn_profile_read(djinn_net* net, double* ms, int64_t* count, int cap, int 
         float t = 0.f;
         if (cudaEventElapsedTime(&t, n.prof_events[r.first + i], n.prof_events[r.first + i + 1]) != cudaSuccess)
           return fail(DJINN_E_CUDA, "cudaEventElapsedTime");
-        acc[i] += t;
-        cnt[i] += 1;
+        const int op = r.op >= 0 ? r.op : i;
+        acc[op] += t;
+        cnt[op] += 1;
       }
     }
     for (int i = 0; i < nops && i < cap; ++i) {

@@ -31,6 +31,8 @@ static inline int nblocks(int64_t n, int t) { return (int)((n + t - 1) / t); }
 template <typename T>
 __global__ void pack16_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int C, int H, int W,
                               int mode, int f, int xs, int Ho, int Wo, int Cp) {
+  pdl_trigger();
+  pdl_wait();
   const int chunks = Cp / 8;
   const int per_row = Ho * Wo * chunks;  // 32-bit index math inside a row
   for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
@@ -70,6 +72,8 @@ __global__ void pack16_kernel(const float* __restrict__ x, T* __restrict__ y, in
 // fp32 storage: one element per thread, (row, pixel, c) order -> coalesced writes.
 __global__ void pack32_kernel(const float* __restrict__ x, float* __restrict__ y, int64_t rows,
                               int C, int HW, int Cp) {
+  pdl_trigger();
+  pdl_wait();
   const int64_t total = rows * (int64_t)HW * Cp;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
        i += (int64_t)gridDim.x * blockDim.x) {
@@ -87,6 +91,8 @@ __global__ void pack32_kernel(const float* __restrict__ x, float* __restrict__ y
 template <typename T>
 __global__ void pack_xform_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int C, int H, int W,
                                   int mode, int f, int xs, int Ho, int Wo, int Cp) {
+  pdl_trigger();
+  pdl_wait();
   const int per_row = Ho * Wo;
   for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
     const float* src = x + r * C * (int64_t)H * W;
@@ -123,6 +129,8 @@ __global__ void pack_xform_kernel(const float* __restrict__ x, T* __restrict__ y
 template <typename T, int MODE, int C, int F, int CP, int XS>
 __global__ void pack_xform_fixed_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int H, int W,
                                         int Ho, int Wo) {
+  pdl_trigger();
+  pdl_wait();
   const int per_row = Ho * Wo;
   for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
     const float* src = x + r * C * (int64_t)H * W;
@@ -158,11 +166,11 @@ static bool launch_pack_fixed(const float* x, void* y, int64_t rows, int C, int 
                               int Wo, int Cp, cudaStream_t st) {
   dim3 g(min(nblocks(Ho * Wo, 128), 1024), (unsigned)(rows < 65535 ? rows : 65535));
   if (mode == 2 && C == 3 && f == 18 && xs == 8 && Cp == 64)
-    pack_xform_fixed_kernel<T, 2, 3, 18, 64, 8><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
+    launch_pdl(pack_xform_fixed_kernel<T, 2, 3, 18, 64, 8>, dim3(g), dim3(128), 0, st, x, (T*)y, rows, H, W, Ho, Wo);
   else if (mode == 2 && C == 1 && f == 12 && xs == 8 && Cp == 16)
-    pack_xform_fixed_kernel<T, 2, 1, 12, 16, 8><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
+    launch_pdl(pack_xform_fixed_kernel<T, 2, 1, 12, 16, 8>, dim3(g), dim3(128), 0, st, x, (T*)y, rows, H, W, Ho, Wo);
   else if (mode == 1 && C == 3 && f == 4 && Cp == 64)
-    pack_xform_fixed_kernel<T, 1, 3, 4, 64, 1><<<g, 128, 0, st>>>(x, (T*)y, rows, H, W, Ho, Wo);
+    launch_pdl(pack_xform_fixed_kernel<T, 1, 3, 4, 64, 1>, dim3(g), dim3(128), 0, st, x, (T*)y, rows, H, W, Ho, Wo);
   else
     return false;
   return true;
@@ -178,20 +186,20 @@ cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int 
   const int T = 256;
   if (dt == DT_F32) {
     int64_t n = rows * (int64_t)H * W * Cp;
-    pack32_kernel<<<min(nblocks(n, T), 148 * 32), T, 0, st>>>(x, (float*)y, rows, C, H * W, Cp);
+    launch_pdl(pack32_kernel, dim3(min(nblocks(n, T), 148 * 32)), dim3(T), 0, st, x, (float*)y, rows, C, H * W, Cp);
   } else if (mode != 0) {
     dim3 g(min(nblocks(Ho * Wo, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
     if (dt == DT_F16)
-      pack_xform_kernel<__half><<<g, T, 0, st>>>(x, (__half*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
+      launch_pdl(pack_xform_kernel<__half>, dim3(g), dim3(T), 0, st, x, (__half*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
     else
-      pack_xform_kernel<__nv_bfloat16><<<g, T, 0, st>>>(x, (__nv_bfloat16*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
+      launch_pdl(pack_xform_kernel<__nv_bfloat16>, dim3(g), dim3(T), 0, st, x, (__nv_bfloat16*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
   } else {
     const int per_row = Ho * Wo * (Cp / 8);
     dim3 g(min(nblocks(per_row, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
     if (dt == DT_F16)
-      pack16_kernel<__half><<<g, T, 0, st>>>(x, (__half*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
+      launch_pdl(pack16_kernel<__half>, dim3(g), dim3(T), 0, st, x, (__half*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
     else
-      pack16_kernel<__nv_bfloat16><<<g, T, 0, st>>>(x, (__nv_bfloat16*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
+      launch_pdl(pack16_kernel<__nv_bfloat16>, dim3(g), dim3(T), 0, st, x, (__nv_bfloat16*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
   }
   return cudaGetLastError();
 }
@@ -202,6 +210,8 @@ cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int 
 template <typename T>
 __global__ void lrn_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t pixels, int C, int Cp, int gsz,
                            int gpitch, int size, float alpha_over_n, float beta, float k) {
+  pdl_trigger();
+  pdl_wait();
   const int half = (size - 1) / 2;
   const int64_t total = pixels * Cp;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
@@ -229,9 +239,9 @@ cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, in
   const int g = min(nblocks(n, T), 148 * 32);
   const float an = alpha / size;
   if (gsz > C) { gsz = C; gpitch = Cp; }
-  if (dt == DT_F32) lrn_kernel<float><<<g, T, 0, st>>>((const float*)x, (float*)y, pixels, C, Cp, gsz, gpitch, size, an, beta, k);
-  else if (dt == DT_F16) lrn_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, pixels, C, Cp, gsz, gpitch, size, an, beta, k);
-  else lrn_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, pixels, C, Cp, gsz, gpitch, size, an, beta, k);
+  if (dt == DT_F32) launch_pdl(lrn_kernel<float>, dim3(g), dim3(T), 0, st, (const float*)x, (float*)y, pixels, C, Cp, gsz, gpitch, size, an, beta, k);
+  else if (dt == DT_F16) launch_pdl(lrn_kernel<__half>, dim3(g), dim3(T), 0, st, (const __half*)x, (__half*)y, pixels, C, Cp, gsz, gpitch, size, an, beta, k);
+  else launch_pdl(lrn_kernel<__nv_bfloat16>, dim3(g), dim3(T), 0, st, (const __nv_bfloat16*)x, (__nv_bfloat16*)y, pixels, C, Cp, gsz, gpitch, size, an, beta, k);
   return cudaGetLastError();
 }
 
@@ -245,6 +255,8 @@ template <typename TO>
 __global__ void lrn_pool_kernel(const __half* __restrict__ x, TO* __restrict__ y, int64_t rows, int C, int Cpi, int H,
                                 int W, int OH, int OW, int kern, int stride, int pad, int gsz, int gpitch, int Cpo,
                                 float an, float nbeta, float k) {
+  pdl_trigger();
+  pdl_wait();
   const int chunks = Cpo / 8;
   const int per_row = OH * OW * chunks;
   for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
@@ -309,10 +321,10 @@ cudaError_t launch_lrn_pool(const void* x, void* y, int64_t rows, int C, int Cpi
   dim3 g(min(nblocks(per_row, 256), 1024), (unsigned)(rows < 65535 ? rows : 65535));
   const float an = alpha / size;
   if (dt == DT_F16)
-    lrn_pool_kernel<__half><<<g, 256, 0, st>>>((const __half*)x, (__half*)y, rows, C, Cpi, H, W, OH, OW, kernel, stride,
+    launch_pdl(lrn_pool_kernel<__half>, dim3(g), dim3(256), 0, st, (const __half*)x, (__half*)y, rows, C, Cpi, H, W, OH, OW, kernel, stride,
                                                pad, out_gsz, out_gpitch, Cpo, an, -beta, k);
   else
-    lrn_pool_kernel<__nv_bfloat16><<<g, 256, 0, st>>>((const __half*)x, (__nv_bfloat16*)y, rows, C, Cpi, H, W, OH, OW,
+    launch_pdl(lrn_pool_kernel<__nv_bfloat16>, dim3(g), dim3(256), 0, st, (const __half*)x, (__nv_bfloat16*)y, rows, C, Cpi, H, W, OH, OW,
                                                       kernel, stride, pad, out_gsz, out_gpitch, Cpo, an, -beta, k);
   return cudaGetLastError();
 }
@@ -323,6 +335,8 @@ cudaError_t launch_lrn_pool(const void* x, void* y, int64_t rows, int C, int Cpi
 template <typename T>
 __global__ void pool_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t rows, int Cp, int H,
                             int W, int OH, int OW, int kern, int stride, int pad, int is_max) {
+  pdl_trigger();
+  pdl_wait();
   const int64_t total = rows * (int64_t)OH * OW * Cp;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
        i += (int64_t)gridDim.x * blockDim.x) {
@@ -353,6 +367,8 @@ __global__ void pool_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t 
 template <typename T>
 __global__ void pool16_xu_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t rows, int Cp, int H, int W,
                                  int OH, int OW, int kern, int stride, int pad, int is_max, int out_xu) {
+  pdl_trigger();
+  pdl_wait();
   const int cchunks = Cp / 8;
   const int per_row = OH * OW * cchunks, Cpo = out_xu * Cp;
   for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
@@ -394,6 +410,8 @@ __global__ void pool16_xu_kernel(const T* __restrict__ x, T* __restrict__ y, int
 template <typename T>
 __global__ void pool16_kernel(const T* __restrict__ x, T* __restrict__ y, int64_t rows, int Cp, int H, int W,
                               int OH, int OW, int kern, int stride, int pad, int is_max, int out_xu) {
+  pdl_trigger();
+  pdl_wait();
   const int cchunks = Cp / 8, chunks = cchunks * out_xu;
   const int per_row = OH * OW * chunks;
   for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
@@ -460,6 +478,8 @@ template <typename T, int K>
 __global__ void pool_max_remap_kernel(const T* __restrict__ x, T* __restrict__ y, int C, int Cpi, int gsz_i,
                                       int gpitch_i, int H, int W, int OH, int OW, int kern, int stride, int pad,
                                       int Cpo, int gsz_o, int gpitch_o, int xu, int obd) {
+  pdl_trigger();
+  pdl_wait();
   __shared__ int in_off[64];  // per output chunk: input channel offset, -1 = zero chunk
   const int P = Cpo / xu, chunks = P / 8;
   if (threadIdx.y == 0 && threadIdx.x < chunks) {
@@ -527,7 +547,7 @@ cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int C
     dim3 blk(chunks, pix), g((OH * OW + pix - 1) / pix, (unsigned)nr);
     const size_t xo = (size_t)r0 * H * W * Cpi, yo = (size_t)r0 * (OH + 2 * obd) * (OW + 2 * obd) * Cpo;
 #define DJ_POOL_LAUNCH(T, KK)                                                                                   \
-  pool_max_remap_kernel<T, KK><<<g, blk, 0, st>>>((const T*)x + xo, (T*)y + yo, C, Cpi, gsz_i, gpitch_i, H, W, OH, OW, \
+  launch_pdl(pool_max_remap_kernel<T, KK>, dim3(g), dim3(blk), 0, st, (const T*)x + xo, (T*)y + yo, C, Cpi, gsz_i, gpitch_i, H, W, OH, OW, \
                                                   kernel, stride, pad, Cpo, gsz_o, gpitch_o, xu, obd)
     if (dt == DT_F16) {
       if (kernel == 3) DJ_POOL_LAUNCH(__half, 3);
@@ -551,25 +571,25 @@ cudaError_t launch_pool(const void* x, void* y, int64_t rows, int C, int Cp, int
     const int per_row = OH * OW * (Cp / 8);
     dim3 g(min(nblocks(per_row, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
     if (dt == DT_F16)
-      pool16_xu_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
+      launch_pdl(pool16_xu_kernel<__half>, dim3(g), dim3(T), 0, st, (const __half*)x, (__half*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
     else
-      pool16_xu_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
+      launch_pdl(pool16_xu_kernel<__nv_bfloat16>, dim3(g), dim3(T), 0, st, (const __nv_bfloat16*)x, (__nv_bfloat16*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
     return cudaGetLastError();
   }
   if (dt != DT_F32 && Cp % 8 == 0) {
     const int per_row = OH * OW * (Cp / 8) * out_xu;
     dim3 g(min(nblocks(per_row, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
     if (dt == DT_F16)
-      pool16_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
+      launch_pdl(pool16_kernel<__half>, dim3(g), dim3(T), 0, st, (const __half*)x, (__half*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
     else
-      pool16_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
+      launch_pdl(pool16_kernel<__nv_bfloat16>, dim3(g), dim3(T), 0, st, (const __nv_bfloat16*)x, (__nv_bfloat16*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max, out_xu);
     return cudaGetLastError();
   }
   const int64_t n = rows * (int64_t)OH * OW * Cp;
   const int g = min(nblocks(n, T), 148 * 32);
-  if (dt == DT_F32) pool_kernel<float><<<g, T, 0, st>>>((const float*)x, (float*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
-  else if (dt == DT_F16) pool_kernel<__half><<<g, T, 0, st>>>((const __half*)x, (__half*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
-  else pool_kernel<__nv_bfloat16><<<g, T, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
+  if (dt == DT_F32) launch_pdl(pool_kernel<float>, dim3(g), dim3(T), 0, st, (const float*)x, (float*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
+  else if (dt == DT_F16) launch_pdl(pool_kernel<__half>, dim3(g), dim3(T), 0, st, (const __half*)x, (__half*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
+  else launch_pdl(pool_kernel<__nv_bfloat16>, dim3(g), dim3(T), 0, st, (const __nv_bfloat16*)x, (__nv_bfloat16*)y, rows, Cp, H, W, OH, OW, kernel, stride, pad, is_max);
   return cudaGetLastError();
 }
 
@@ -582,6 +602,8 @@ __device__ __forceinline__ void argmax_combine(float& v, int& i, float v2, int i
 
 __global__ void softmax_kernel(const float* __restrict__ z, int64_t rows, int N, int pitch,
                                void* __restrict__ out, int mode) {
+  pdl_trigger();
+  pdl_wait();
   __shared__ float s_v[32];
   __shared__ int s_i[32];
   const int64_t r = blockIdx.x;
@@ -644,6 +666,8 @@ __global__ void softmax_kernel(const float* __restrict__ z, int64_t rows, int N,
 // Single pass, values held in registers: one warp per row (N <= 32*VPT).
 template <int VPT>
 __global__ void softmax_warp_kernel(const float* __restrict__ z, int64_t rows, int N, int pitch, float* __restrict__ out) {
+  pdl_trigger();
+  pdl_wait();
   const int lane = threadIdx.x & 31;
   const int64_t r = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5);
   if (r >= rows) return;
@@ -679,6 +703,8 @@ __global__ void softmax_warp_kernel(const float* __restrict__ z, int64_t rows, i
 // per row, float4 loads, exp values kept in registers between the reductions.
 template <int VQ>
 __global__ void softmax_block_kernel(const float* __restrict__ z, int64_t rows, int N, int pitch, float* __restrict__ out) {
+  pdl_trigger();
+  pdl_wait();
   __shared__ float red[8];
   const int64_t r = blockIdx.x;
   const int t = threadIdx.x, lane = t & 31, wid = t >> 5;
@@ -747,12 +773,12 @@ cudaError_t launch_softmax(const float* logits, int64_t rows, int N, int pitch, 
   if (mode == 0 && N <= 256 && pitch % 4 == 0) {
     const int rpb = 8;  // rows (warps) per 256-thread block
     const unsigned g = (unsigned)((rows + rpb - 1) / rpb);
-    if (N <= 64) softmax_warp_kernel<2><<<g, 256, 0, st>>>(logits, rows, N, pitch, (float*)out);
-    else softmax_warp_kernel<8><<<g, 256, 0, st>>>(logits, rows, N, pitch, (float*)out);
+    if (N <= 64) launch_pdl(softmax_warp_kernel<2>, dim3(g), dim3(256), 0, st, logits, rows, N, pitch, (float*)out);
+    else launch_pdl(softmax_warp_kernel<8>, dim3(g), dim3(256), 0, st, logits, rows, N, pitch, (float*)out);
   } else if (mode == 0 && N <= 8192 && pitch % 4 == 0) {
-    softmax_block_kernel<8><<<(unsigned)rows, 256, 0, st>>>(logits, rows, N, pitch, (float*)out);
+    launch_pdl(softmax_block_kernel<8>, dim3((unsigned)rows), dim3(256), 0, st, logits, rows, N, pitch, (float*)out);
   } else {
-    softmax_kernel<<<(unsigned)rows, 256, 0, st>>>(logits, rows, N, pitch, out, mode);
+    launch_pdl(softmax_kernel, dim3((unsigned)rows), dim3(256), 0, st, logits, rows, N, pitch, out, mode);
   }
   return cudaGetLastError();
 }

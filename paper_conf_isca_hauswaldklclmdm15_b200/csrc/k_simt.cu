@@ -26,6 +26,8 @@ __global__ void __launch_bounds__(NT) simt_gemm_kernel(GemmGeom g, const float* 
                                                        const float* __restrict__ B,
                                                        const float* __restrict__ bias,
                                                        float* __restrict__ Y) {
+  pdl_trigger();
+  pdl_wait();
   __shared__ float As[TK][TM + 4];
   __shared__ float Bs[TK][TN + 4];
   const int t = threadIdx.x;
@@ -127,7 +129,7 @@ __global__ void __launch_bounds__(NT) simt_gemm_kernel(GemmGeom g, const float* 
 cudaError_t launch_simt_gemm(const GemmGeom& g, const float* A, const float* B, const float* bias,
                              float* Y, cudaStream_t st) {
   dim3 grid((g.M + TM - 1) / TM, (max(g.N, g.write_cols) + TN - 1) / TN, g.Z);
-  simt_gemm_kernel<<<grid, NT, 0, st>>>(g, A, B, bias, Y);
+  launch_pdl(simt_gemm_kernel, dim3(grid), dim3(NT), 0, st, g, A, B, bias, Y);
   return cudaGetLastError();
 }
 

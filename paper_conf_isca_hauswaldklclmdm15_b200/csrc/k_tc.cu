@@ -110,6 +110,24 @@ __device__ __forceinline__ void mbar_wait_ld(uint32_t bar, uint32_t parity) {
   mbar_wait(bar, parity);
 #endif
 }
+// Polling with a short back-off: for waiters whose stages cover many MMA cycles (slab mode's
+// B-only loaders: a stage is 8-16 MMAs), so a ~100 ns late wake-up costs nothing, while a tight
+// spin took 17% of the SM's issue slots from the epilogue warps (ncu, IMC conv1+norm1).
+__device__ __forceinline__ void mbar_wait_backoff(uint32_t bar, uint32_t parity) {
+  uint32_t done, iters = 0;
+  for (;;) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(bar), "r"(parity)
+        : "memory");
+    if (done) break;
+    if (++iters > (1u << 26)) __trap();  // a lost arrival must fault, never hang the GPU
+    __nanosleep(96);
+  }
+}
 __device__ __forceinline__ void tma_2d(uint32_t dst, const CUtensorMap* map, uint32_t bar, int c0, int c1) {
   asm volatile(
       "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
@@ -271,14 +289,34 @@ __device__ __forceinline__ float tanh_approx(float v) {
   asm("tanh.approx.f32 %0, %1;" : "=f"(r) : "f"(v));
   return r;
 }
+// Bare MUFU approximations with flush-to-zero: exp2f / __log2f / __expf / __fdividef compile to
+// MUFU plus an FSETP + FMUL denormal range fixup per call (ncu, IMC conv1+norm1: the fixups were
+// ~5 of the LRN epilogue's ~15 instructions per element).  Arguments here are never denormal
+// where it matters (LRN: t = k + alpha/n * sum >= k; sigmoid: 1 + e^-x >= 1).
+__device__ __forceinline__ float ex2_ftz(float x) {
+  float r;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+__device__ __forceinline__ float lg2_ftz(float x) {
+  float r;
+  asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+__device__ __forceinline__ float rcp_ftz(float x) {
+  float r;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
+__device__ __forceinline__ float sigmoid_fast(float v) { return rcp_ftz(1.f + ex2_ftz(-1.4426950408889634f * v)); }
 // Activations on MUFU (16-bit storage tolerates their ~2^-11..2^-21 relative error).
 __device__ __forceinline__ float act_fast(float v, int act) {
   switch (act) {
     case ACT_RELU: return fmaxf(v, 0.f);
-    case ACT_SIGMOID: return __fdividef(1.f, 1.f + __expf(-v));
+    case ACT_SIGMOID: return sigmoid_fast(v);
     case ACT_TANH: return tanh_approx(v);
     case ACT_HARDTANH: return fminf(fmaxf(v, -1.f), 1.f);
-    case ACT_SIGMOID_C: return __fdividef(1.f, 1.f + __expf(-v)) - 0.5f;  // sigma - 1/2 (abs. err ~1e-7)
+    case ACT_SIGMOID_C: return sigmoid_fast(v) - 0.5f;  // sigma - 1/2 (abs. err ~1e-7)
     default: return v;
   }
 }
@@ -295,11 +333,11 @@ __device__ __forceinline__ void bias_act16(float (&v)[16], const uint32_t (&r)[1
       break;
     case ACT_SIGMOID:
 #pragma unroll
-      for (int j = 0; j < 16; ++j) v[j] = __fdividef(1.f, 1.f + __expf(-v[j]));
+      for (int j = 0; j < 16; ++j) v[j] = sigmoid_fast(v[j]);
       break;
     case ACT_SIGMOID_C:
 #pragma unroll
-      for (int j = 0; j < 16; ++j) v[j] = __fdividef(1.f, 1.f + __expf(-v[j])) - 0.5f;
+      for (int j = 0; j < 16; ++j) v[j] = sigmoid_fast(v[j]) - 0.5f;
       break;
     case ACT_TANH:
 #pragma unroll
@@ -445,6 +483,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const GemmGeom g, const float* __restrict__ bias, void* __restrict__ Y) {
   using C = Cfg<BN, CG>;
+  pdl_trigger();
   // cta_group::2: a CTA pair computes a (2*128) x BN tile; rank 0 (leader) issues the MMAs.
   const uint32_t rank = CG == 2 ? cluster_rank() : 0;
   const int cid = blockIdx.x / CG, ncl = gridDim.x / CG;
@@ -520,6 +559,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   if (CG == 2) cluster_sync();  // peer barriers initialised before any remote arrive / TMA tx
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  pdl_wait();  // the previous kernel of the stream has completed: its output is visible
 
   if (warp >= LOAD_WARP0 && warp < LOAD_WARP0 + NLOAD) {
     // TMA loaders.  Each loader warp runs the whole loop (warp-uniform values stay in uniform
@@ -588,7 +628,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         for (int u0 = 0; u0 < nsteps; u0 += KPS) {
           const int cnt = min(KPS, nsteps - u0);
           if (qo == myq) {
-            mbar_wait_ld(empty0 + 8 * s, ph ^ 1);
+            if (g.ldwait == 1) mbar_wait_backoff(empty0 + 8 * s, ph ^ 1);
+            else if (g.ldwait == 2) mbar_wait_sleep(empty0 + 8 * s, ph ^ 1);
+            else mbar_wait(empty0 + 8 * s, ph ^ 1);
             if (leader) {
               const uint32_t fb = full0 + 8 * s;
               if (rank == 0) mbar_arrive_expect_tx(fb, kDbgNoB ? 0u : (uint32_t)(CG * C::B_BYTES * cnt));
@@ -985,7 +1027,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 #pragma unroll
           for (int j = 0; j < 16; ++j) {
             const float s5 = (sq[j] + sq[j + 1]) + (sq[j + 2] + sq[j + 3]) + sq[j + 4];  // window c-2 .. c+2
-            o[j] = cur[j] * exp2f(nb * __log2f(fmaf(ka, s5, kk)));
+#if defined(DJINN_DBG_LRN0)
+            o[j] = cur[j] * fmaf(ka, s5, kk);  // diagnostic: no MUFU
+#elif defined(DJINN_DBG_LRN1)
+            o[j] = cur[j] * rsqrtf(fmaf(ka, s5, kk));  // diagnostic: one MUFU
+#else
+            o[j] = cur[j] * ex2_ftz(nb * lg2_ftz(fmaf(ka, s5, kk)));
+#endif
           }
           pm2 = sq[16];
           pm1 = sq[17];
@@ -1136,13 +1184,15 @@ cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtenso
   cfg.blockDim = dim3(NUM_THREADS);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = CG;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = pdl_enabled() ? 2 : 1;
   return cudaLaunchKernelEx(&cfg, kern, *tmA, *tmB, g, bias, Y);
 }
 

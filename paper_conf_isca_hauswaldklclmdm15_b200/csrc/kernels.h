@@ -8,6 +8,32 @@
 
 namespace djinn {
 
+// ---- programmatic dependent launch (PDL) --------------------------------------------------
+// Every kernel of a forward pass is launched with programmatic stream serialization: kernel i+1
+// may be scheduled while kernel i drains its last wave, runs its prologue (barrier init, TMEM
+// allocation, tensor-map prefetch) and then blocks in pdl_wait() -- griddepcontrol.wait returns
+// once kernel i has COMPLETED and its memory is visible -- before its first global access.
+// Each kernel calls pdl_trigger() on entry.  DJINN_PDL=0 disables the attribute (plain stream order).
+#if defined(__CUDACC__)
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+#endif
+bool pdl_enabled();
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+
 enum DType { DT_F32 = 0, DT_BF16 = 1, DT_F16 = 2 };
 // ACT_SIGMOID_C stores sigma(x) - 1/2 ("centered" storage, an exact reparametrisation: the
 // consumer's bias absorbs + 1/2 * rowsum(W)); it keeps 16-bit activations near 0 where their
@@ -68,6 +94,7 @@ struct GemmGeom {
   int slab_parts, slab_rows;  // the slab is loaded as slab_parts TMA boxes of slab_rows rows
   int stages;         // slab mode: B ring stages (runtime; set by tc_slab_config)
   int kps;            // slab mode: K blocks of B per ring stage (one MMA commit per stage)
+  int ldwait;         // slab mode: B-loader stage wait (0 spin, 1 poll + nanosleep back-off, 2 suspend hint)
   int obd;            // conv output: zero border of the stored output tensor (its consumer's pad)
   int lrn_size;
   float lrn_alpha_over_n, lrn_beta, lrn_k;

@@ -117,6 +117,23 @@ PNode parse_prototxt(const std::string& text) {
 }
 
 // ============================================================================ helpers
+// slab-mode B-loader wait policy (GemmGeom::ldwait), DJINN_LDWAIT=0/1/2 (default spin)
+static int ldwait_mode() {
+  static const int m = [] {
+    const char* e = getenv("DJINN_LDWAIT");
+    return e ? atoi(e) : 0;
+  }();
+  return m;
+}
+
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char* e = getenv("DJINN_PDL");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
 std::atomic<int64_t>& launch_counter() {
   static std::atomic<int64_t> c{0};
   return c;
@@ -984,16 +1001,17 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
       src = w->in_stage;
     }
     uint8_t* dst = out_mem == DJINN_MEM_HOST ? (uint8_t*)w->out_stage : (uint8_t*)out + r0 * out_row_bytes;
+    const int pop = profile ? profile_op : -1;  // one timed op, or all (-1)
     if (profile) {
       std::lock_guard<std::mutex> lk(mu);
-      prof_recs.push_back({prof_used, (int)ops.size()});
-      for (size_t i = 0; i <= ops.size(); ++i) prof_event();
+      prof_recs.push_back({prof_used, pop < 0 ? (int)ops.size() : 1, pop});
+      for (size_t i = 0; i <= (pop < 0 ? ops.size() : 1); ++i) prof_event();
     }
     const size_t pbase = profile ? prof_recs.back().first : 0;
     for (size_t i = 0; i < ops.size(); ++i) {
       const Op& o = ops[i];
       cudaError_t e = cudaSuccess;
-      if (profile) ck(cudaEventRecord(prof_events[pbase + i], st), "profile event");
+      if (profile && (pop < 0 || pop == (int)i)) ck(cudaEventRecord(prof_events[pbase + (pop < 0 ? i : 0)], st), "profile event");
       switch (o.kind) {
         case OP_PACK:
           e = launch_pack_input(src, w->buf[0], n, o.in.C, o.in.H, o.in.W, o.xform, o.xf, o.xs, o.out.H, o.out.W, o.out.Cp,
@@ -1001,6 +1019,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           break;
         case OP_GEMM: {
           GemmGeom g = o.g;
+          g.ldwait = ldwait_mode();
           g.M = (int)(n * o.ohw);
           g.Nimg = (int)n;
           const void* A = w->buf[o.in_buf];
@@ -1041,8 +1060,9 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
         poisoned = true;
         throw Error(DJINN_E_CUDA, o.name + ": " + cudaGetErrorString(e));
       }
+      if (profile && pop == (int)i) ck(cudaEventRecord(prof_events[pbase + 1], st), "profile event");
     }
-    if (profile) ck(cudaEventRecord(prof_events[pbase + ops.size()], st), "profile event");
+    if (profile && pop < 0) ck(cudaEventRecord(prof_events[pbase + ops.size()], st), "profile event");
     if (out_mem == DJINN_MEM_HOST)
       ck(cudaMemcpyAsync((uint8_t*)out + r0 * out_row_bytes, w->out_stage, (size_t)n * out_row_bytes,
                          cudaMemcpyDeviceToHost, st),

@@ -87,6 +87,7 @@ struct Op {
 struct ProfRec {  // one timed forward chunk: events[first .. first + n_ops]
   size_t first;
   int n_ops;
+  int op;         // -1: every op (n_ops + 1 events); >= 0: only op `op` (events[first], events[first + 1])
 };
 
 struct Workspace {
@@ -116,6 +117,7 @@ struct Net {
   bool poisoned = false;
   // per-op profiling (djinn_profile)
   bool profile = false;
+  int profile_op = -1;  // -1: time every op; k >= 0: time op k only (djinn_profile(net, 2 + k))
   std::vector<cudaEvent_t> prof_events;
   size_t prof_used = 0;
   std::vector<ProfRec> prof_recs;

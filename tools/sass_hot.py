@@ -14,7 +14,7 @@ hi = int(sys.argv[4], 16) if len(sys.argv) > 4 else None
 ia, isrc, ist = h.index("Address"), h.index("Source"), h.index("Warp Stall Sampling (All Samples)")
 ie = h.index("Instructions Executed")
 stall_cols = [i for i, c in enumerate(h) if c.startswith("stall_") and "Not Issued" not in c]
-seen, data = set(), []
+seen, data, base = set(), [], None
 for r in rows[2:]:
     try:
         key = r[ia]
@@ -22,8 +22,9 @@ for r in rows[2:]:
             continue
         seen.add(key)
         addr = int(key, 16)
-        base = data[0][2] if data else addr
-        off = addr - base if data else 0
+        if base is None:
+            base = addr
+        off = addr - base
         if lo is not None and not (lo <= off < hi):
             continue
         st = Counter({h[i][6:]: int(r[i] or 0) for i in stall_cols})
