@@ -5,6 +5,8 @@
 #include <cuda_fp16.h>
 #include <float.h>
 
+#include <algorithm>
+
 #include "kernels.h"
 
 namespace djinn {
@@ -246,86 +248,147 @@ cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, in
 }
 
 // ------------------------------------------------------------------------------------------
-// K4+K5 fused: y = maxpool(LRN(x)).  One thread per (output pixel, 8-channel chunk of the output
-// layout); for every pixel of the pooling window it loads the 8 channels plus the neighbouring
-// chunks (the LRN window needs c-2 .. c+2), evaluates Caffe's LRN in fp32 and keeps the max.
-// The conv before it stores its ReLU output in fp16, so LRN's input keeps
-// 11 mantissa bits on the bf16 path too.
+// K4+K5 fused: y = maxpool(LRN(x)), Caffe LRN across channels (window c-2..c+2 clipped to
+// [0, C)) in fp32, then Caffe MAX pooling with kernel 3 / stride 2 / pad 0 (AlexNet norm1+pool1,
+// norm2+pool2).  The conv before it stores its bias+ReLU output in fp16 (plain layout, pitch
+// Cpi, channels >= C zero).
+//
+// Every input element's LRN is evaluated ONCE (the MUFU work is the kernel's floor): a warp
+// owns 16 channels of 32 adjacent input columns and walks down the rows of its band; the
+// vertical window max lives in registers (rows 2oy, 2oy+1, 2oy+2; row 2oy+2 also opens window
+// oy+1), the horizontal one takes two warp shuffles, and the even lanes 0..28 store output
+// pixels ox = (x0 + lane) / 2.  Warps start every 30 columns (2 columns of overlap).
+// Block: 32 x (C/16) threads = one column segment of one image band; grid (segments, rows, bands).
 template <typename TO>
-__global__ void lrn_pool_kernel(const __half* __restrict__ x, TO* __restrict__ y, int64_t rows, int C, int Cpi, int H,
-                                int W, int OH, int OW, int kern, int stride, int pad, int gsz, int gpitch, int Cpo,
-                                float an, float nbeta, float k) {
+__global__ void __launch_bounds__(512) lrn_pool_kernel(const __half* __restrict__ x, TO* __restrict__ y, int C, int Cpi,
+                                                       int H, int W, int OH, int OW, int bands, int gsz, int gpitch,
+                                                       int Cpo, int obd, float an, float nbeta, float k) {
   pdl_trigger();
   pdl_wait();
-  const int chunks = Cpo / 8;
-  const int per_row = OH * OW * chunks;
-  for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
-    const __half* xr = x + r * (int64_t)H * W * Cpi;
-    TO* yr = y + r * (int64_t)OH * OW * Cpo;
-    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < per_row; i += gridDim.x * blockDim.x) {
-      const int p8 = i % chunks, pix = i / chunks;
-      const int pos = p8 * 8, grp = pos / gpitch, within = pos - grp * gpitch;
-      const int c0 = grp * gsz + within;  // logical channel of this output chunk
-      __align__(16) TO o[8];
-      if (within >= gsz || c0 >= C) {
+  const int lane = threadIdx.x, c0 = threadIdx.y * 16;
+  const int x0 = blockIdx.x * 30, xx = x0 + lane;
+  const int64_t r = blockIdx.y;
+  const int per_band = (OH + bands - 1) / bands;
+  const int oy0 = blockIdx.z * per_band, oy1 = min(OH, oy0 + per_band);
+  if (oy0 >= oy1) return;
+  const bool xin = xx < W;
+  const __half* xr = x + ((r * H) * (int64_t)W + (xin ? xx : W - 1)) * Cpi + c0;
+  // output channel positions of this thread's 16 channels (16 | gsz: a chunk never straddles groups)
+  const int grp = c0 / gsz, cin = c0 - grp * gsz;
+  TO* yr = y + (r * (OH + 2 * obd) + obd) * (int64_t)(OW + 2 * obd) * Cpo + grp * gpitch + cin;
+  const bool pad_writer = gpitch > gsz && cin + 16 == gsz;
+  const bool has_lo = c0 >= 2, has_hi = c0 + 16 < C;
+  __half2 acc[8];
+  int emitted = oy0 - 1;
+  auto emit = [&](int oy) {
+    // horizontal window: columns 2ox .. 2ox+2 (clipped to W - 1: a duplicate cannot change a max)
+    __half2 m[8];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) o[j] = cvt<TO>(0.f);
-        *reinterpret_cast<uint4*>(yr + (int64_t)pix * Cpo + pos) = *reinterpret_cast<const uint4*>(o);
-        continue;
+    for (int j = 0; j < 8; ++j) {
+      const uint32_t u = *reinterpret_cast<const uint32_t*>(&acc[j]);
+      const uint32_t u1 = __shfl_down_sync(0xffffffffu, u, 1), u2 = __shfl_down_sync(0xffffffffu, u, 2);
+      __half2 v = acc[j];
+      if (xx + 1 < W) v = __hmax2(v, *reinterpret_cast<const __half2*>(&u1));
+      if (xx + 2 < W) v = __hmax2(v, *reinterpret_cast<const __half2*>(&u2));
+      m[j] = v;
+    }
+    const int ox = xx >> 1;
+    if (!(lane & 1) && lane <= 28 && ox < OW) {
+      TO* yo = yr + ((int64_t)oy * (OW + 2 * obd) + ox + obd) * Cpo;
+      __align__(16) TO o[16];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const float2 f = __half22float2(m[j]);
+        o[2 * j] = cvt<TO>(f.x);
+        o[2 * j + 1] = cvt<TO>(f.y);
       }
-      const int oy = pix / OW, ox = pix - (pix / OW) * OW;
-      int hs = oy * stride - pad, ws = ox * stride - pad;
-      int he = min(hs + kern, H + pad), we = min(ws + kern, W + pad);
-      hs = max(hs, 0); ws = max(ws, 0); he = min(he, H); we = min(we, W);
-      float acc[8];
+      reinterpret_cast<uint4*>(yo)[0] = reinterpret_cast<const uint4*>(o)[0];
+      reinterpret_cast<uint4*>(yo)[1] = reinterpret_cast<const uint4*>(o)[1];
+      if (pad_writer)
+        for (int e = 16; e < 16 + gpitch - gsz; e += 8) *reinterpret_cast<uint4*>(yo + e) = make_uint4(0, 0, 0, 0);
+    }
+    emitted = oy;
+  };
+  const int ylast = min(2 * oy1, H - 1);
+  for (int yy = 2 * oy0; yy <= ylast; ++yy) {
+    const __half* px = xr + (int64_t)yy * W * Cpi;
+    const uint4 ua = __ldg(reinterpret_cast<const uint4*>(px));
+    const uint4 ub = __ldg(reinterpret_cast<const uint4*>(px) + 1);
+    const uint32_t ulo = has_lo ? __ldg(reinterpret_cast<const unsigned int*>(px - 2)) : 0u;
+    const uint32_t uhi = has_hi ? __ldg(reinterpret_cast<const unsigned int*>(px + 16)) : 0u;
+    float v[20];
+    {
+      const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&ulo));
+      const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&uhi));
+      v[0] = lo.x; v[1] = lo.y; v[18] = hi.x; v[19] = hi.y;
+      const __half2* ha = reinterpret_cast<const __half2*>(&ua);
+      const __half2* hb = reinterpret_cast<const __half2*>(&ub);
 #pragma unroll
-      for (int j = 0; j < 8; ++j) acc[j] = -FLT_MAX;
-      for (int h = hs; h < he; ++h)
-        for (int w = ws; w < we; ++w) {
-          const __half* px = xr + ((int64_t)h * W + w) * Cpi + c0;
-          float v[24];
-          const uint4 uc = __ldg(reinterpret_cast<const uint4*>(px));
-          const uint4 up = c0 >= 8 ? __ldg(reinterpret_cast<const uint4*>(px - 8)) : make_uint4(0, 0, 0, 0);
-          const uint4 un = c0 + 8 < C ? __ldg(reinterpret_cast<const uint4*>(px + 8)) : make_uint4(0, 0, 0, 0);
-          const __half* hp = reinterpret_cast<const __half*>(&up);
-          const __half* hc = reinterpret_cast<const __half*>(&uc);
-          const __half* hn = reinterpret_cast<const __half*>(&un);
+      for (int j = 0; j < 4; ++j) {
+        const float2 fa = __half22float2(ha[j]), fb = __half22float2(hb[j]);
+        v[2 + 2 * j] = fa.x; v[3 + 2 * j] = fa.y; v[10 + 2 * j] = fb.x; v[11 + 2 * j] = fb.y;
+      }
+    }
+    float sq[20];
 #pragma unroll
-          for (int j = 0; j < 8; ++j) {
-            v[j] = __half2float(hp[j]);
-            v[8 + j] = __half2float(hc[j]);
-            v[16 + j] = __half2float(hn[j]);
-          }
+    for (int j = 0; j < 20; ++j) sq[j] = v[j] * v[j];
+    float p2[19];
 #pragma unroll
-          for (int j = 0; j < 8; ++j) {
-            const float s5 = (v[6 + j] * v[6 + j] + v[7 + j] * v[7 + j]) + (v[8 + j] * v[8 + j] + v[9 + j] * v[9 + j]) +
-                             v[10 + j] * v[10 + j];
-            const float l = v[8 + j] * exp2f(nbeta * __log2f(fmaf(an, s5, k)));
-            acc[j] = fmaxf(acc[j], l);
-          }
-        }
+    for (int j = 0; j < 19; ++j) p2[j] = sq[j] + sq[j + 1];
+    __half2 l[8];
 #pragma unroll
-      for (int j = 0; j < 8; ++j) o[j] = cvt<TO>(acc[j]);
-      *reinterpret_cast<uint4*>(yr + (int64_t)pix * Cpo + pos) = *reinterpret_cast<const uint4*>(o);
+    for (int j = 0; j < 8; ++j) {
+      const float s0 = (p2[2 * j] + p2[2 * j + 2]) + sq[2 * j + 4], s1 = (p2[2 * j + 1] + p2[2 * j + 3]) + sq[2 * j + 5];
+      float r0, r1;
+      asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(r0) : "f"(fmaf(an, s0, k)));
+      asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(r1) : "f"(fmaf(an, s1, k)));
+      asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r0) : "f"(nbeta * r0));
+      asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r1) : "f"(nbeta * r1));
+      l[j] = __floats2half2_rn(v[2 + 2 * j] * r0, v[3 + 2 * j] * r1);
+    }
+    if (!xin) {
+#pragma unroll
+      for (int j = 0; j < 8; ++j) l[j] = __float2half2_rn(0.f);
+    }
+    if ((yy & 1) == 0) {
+      const int j = yy >> 1;
+      if (j - 1 >= oy0) {  // row 2(j-1)+2 closes window j-1
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc[q] = __hmax2(acc[q], l[q]);
+        emit(j - 1);
+      }
+      if (j < oy1) {
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc[q] = l[q];
+      }
+    } else {
+#pragma unroll
+      for (int q = 0; q < 8; ++q) acc[q] = __hmax2(acc[q], l[q]);
     }
   }
+  if (emitted < oy1 - 1) emit(oy1 - 1);  // last window clipped at the bottom edge (ceil geometry)
 }
 
 cudaError_t launch_lrn_pool(const void* x, void* y, int64_t rows, int C, int Cpi, int H, int W, int OH, int OW,
-                            int kernel, int stride, int pad, int out_gsz, int out_gpitch, int Cpo, int size,
+                            int kernel, int stride, int pad, int out_gsz, int out_gpitch, int Cpo, int obd, int size,
                             float alpha, float beta, float k, int dt, cudaStream_t st) {
-  if (size != 5 || C % 8 || Cpi % 8 || Cpo % 8) return cudaErrorInvalidValue;
-  if (out_gsz > C) { out_gsz = C; out_gpitch = Cpo; }
-  if (out_gsz % 8 || out_gpitch % 8) return cudaErrorInvalidValue;
-  const int per_row = OH * OW * (Cpo / 8);
-  dim3 g(min(nblocks(per_row, 256), 1024), (unsigned)(rows < 65535 ? rows : 65535));
+  if (size != 5 || kernel != 3 || stride != 2 || pad != 0 || C % 16 || Cpi % 8 || Cpi < C || C > 512 || Cpo % 8 ||
+      rows > 65535 || obd < 0)
+    return cudaErrorInvalidValue;
+  if (out_gsz >= C) { out_gsz = C; out_gpitch = Cpo; }
+  if (out_gsz % 16 || out_gpitch % 8) return cudaErrorInvalidValue;
+  const int segs = (W + 29) / 30;
+  // bands of output rows: enough warps for ~3 waves (each band re-reads one boundary input row)
+  const int64_t warps = (int64_t)segs * rows * (C / 16);
+  int bands = (int)std::min<int64_t>(std::max<int64_t>(1, (3 * 148 * 64 + warps - 1) / warps), OH);
+  dim3 g(segs, (unsigned)rows, bands), b(32, C / 16);
   const float an = alpha / size;
   if (dt == DT_F16)
-    launch_pdl(lrn_pool_kernel<__half>, dim3(g), dim3(256), 0, st, (const __half*)x, (__half*)y, rows, C, Cpi, H, W, OH, OW, kernel, stride,
-                                               pad, out_gsz, out_gpitch, Cpo, an, -beta, k);
+    launch_pdl(lrn_pool_kernel<__half>, g, b, 0, st, (const __half*)x, (__half*)y, C, Cpi, H, W, OH, OW, bands, out_gsz,
+               out_gpitch, Cpo, obd, an, -beta, k);
   else
-    launch_pdl(lrn_pool_kernel<__nv_bfloat16>, dim3(g), dim3(256), 0, st, (const __half*)x, (__nv_bfloat16*)y, rows, C, Cpi, H, W, OH, OW,
-                                                      kernel, stride, pad, out_gsz, out_gpitch, Cpo, an, -beta, k);
+    launch_pdl(lrn_pool_kernel<__nv_bfloat16>, g, b, 0, st, (const __half*)x, (__nv_bfloat16*)y, C, Cpi, H, W, OH, OW,
+               bands, out_gsz, out_gpitch, Cpo, obd, an, -beta, k);
   return cudaGetLastError();
 }
 

@@ -397,6 +397,13 @@ __device__ __forceinline__ void store16(const GemmGeom& g, void* Y, int64_t off,
 #ifdef DJINN_DBG_NOSTORE
   if (v[0] != 12345.f) return;
 #endif
+#ifdef DJINN_DBG_COALESCED
+  {  // diagnostic (wrong results): the warp's 16-byte stores land contiguously, same byte count
+    const unsigned am = __activemask();
+    const int64_t b0 = __shfl_sync(am, off, __ffs(am) - 1);
+    off = b0 + (off % g.out_pitch) * 32 + (threadIdx.x & 31) * 8;
+  }
+#endif
   if (g.out_f32) {
     float* yp = reinterpret_cast<float*>(Y) + off;
 #pragma unroll
@@ -502,12 +509,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   uint8_t* sSlab = smem + ((NST * SB_BYTES + 1023) & ~1023);
   uint64_t* bars = SLAB ? reinterpret_cast<uint64_t*>(sSlab + 2 * slab_bytes)
                         : reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
-  // bars: full[NST], empty[NST], tfull[2], tempty[2], sfull[2], sempty[2]
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * NST + 8);
+  // bars: full[NST], empty[NST], tfull[4], tempty[4], sfull[2], sempty[2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * NST + 12);
   __shared__ uint32_t ktab[KTAB_MAX];
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + NST);
-  const uint32_t tfull0 = smem_u32(bars + 2 * NST), tempty0 = smem_u32(bars + 2 * NST + 2);
-  const uint32_t sfull0 = smem_u32(bars + 2 * NST + 4), sempty0 = smem_u32(bars + 2 * NST + 6);
+  const uint32_t tfull0 = smem_u32(bars + 2 * NST), tempty0 = smem_u32(bars + 2 * NST + 4);
+  const uint32_t sfull0 = smem_u32(bars + 2 * NST + 8), sempty0 = smem_u32(bars + 2 * NST + 10);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int num_kb = g.Kpad / BK;
@@ -520,7 +527,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   const int tiles = mt * nt * zt;
   int slot_cols = 32;  // TMEM columns per accumulator slot (power of two >= zf*BN)
   while (slot_cols < g.zf * BN) slot_cols <<= 1;
-  const int nslots = 2;  // launch_inst guarantees zf * BN <= 256 (two accumulator slots)
+  // Accumulator slots: 4 when they fit in TMEM's 512 columns (zf * BN <= 128), else 2
+  // (launch_inst guarantees zf * BN <= 256).  Each warpgroup drains every other tile; with 2
+  // slots the MMA of tile t+2 waits for the epilogue of tile t to finish within ONE tile time,
+  // with 4 it may run 3 tiles ahead (IMC conv1: the epilogue's latency, not its work, had
+  // stalled the MMA).  g.tslots = 2 forces two.
+  const int nslots = (4 * slot_cols <= 512 && g.tslots != 2) ? 4 : 2;
+  const int slot_sh = nslots == 4 ? 2 : 1;
   int tcols = 32;
   while (tcols < nslots * slot_cols) tcols <<= 1;
 
@@ -530,9 +543,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       mbar_init(full0 + 8 * s, 1);
       mbar_init(empty0 + 8 * s, 1);
     }
-    for (int s = 0; s < 2; ++s) {
+    for (int s = 0; s < 4; ++s) {
       mbar_init(tfull0 + 8 * s, 1);
-      mbar_init(tempty0 + 8 * s, (EPI_WARPS / 2) * CG);  // one warpgroup per slot; leader's: both CTAs'
+      mbar_init(tempty0 + 8 * s, (EPI_WARPS / 2) * CG);  // one warpgroup per tile; leader's: both CTAs'
+    }
+    for (int s = 0; s < 2; ++s) {
       mbar_init(sfull0 + 8 * s, 1);
       mbar_init(sempty0 + 8 * s, 1);
     }
@@ -820,8 +835,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       int s = 0, lt = 0;
       uint32_t ph = 0;
       for (int t = cid; t < tiles; t += ncl, ++lt) {
-        const int slot = nslots == 2 ? (lt & 1) : 0;
-        const uint32_t use = nslots == 2 ? (uint32_t)(lt >> 1) : (uint32_t)lt;
+        const int slot = lt & (nslots - 1);
+        const uint32_t use = (uint32_t)(lt >> slot_sh);
         {
           STAT_T0();
           mbar_wait_sleep(tempty0 + 8 * slot, (use & 1) ^ 1);
@@ -929,8 +944,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       if ((lt & 1) != wg) continue;
       TileCoord tc = tile_coord(g, t, mt, nt, CG);
       tc.m0 += (int)rank * BM;  // this CTA's rows of the pair tile
-      const int slot = lt & 1;
-      const uint32_t use = (uint32_t)(lt >> 1);
+      const int slot = lt & (nslots - 1);
+      const uint32_t use = (uint32_t)(lt >> slot_sh);
       int m;       // GEMM row (dense, LC)
       bool mok;
       // conv: output pixel (img, oy, ox) of the row (ox: first pixel of its x block) and its
@@ -1155,7 +1170,7 @@ int slab_smem(const GemmGeom& g, int stages) {
   using C = Cfg<BN, CG>;
   const int ring = (stages * g.kps * C::B_BYTES + 1023) & ~1023;
   const int slab = g.zf * (g.Cgp / 64) * g.slab_parts * g.slab_rows * 128;
-  return 1024 + ring + 2 * slab + (2 * stages + 8) * 8 + 16;
+  return 1024 + ring + 2 * slab + (2 * stages + 12) * 8 + 16;
 }
 
 template <int BN, bool BF16, int CG, bool SLAB>

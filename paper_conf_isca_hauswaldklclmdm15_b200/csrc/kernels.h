@@ -94,6 +94,7 @@ struct GemmGeom {
   int slab_parts, slab_rows;  // the slab is loaded as slab_parts TMA boxes of slab_rows rows
   int stages;         // slab mode: B ring stages (runtime; set by tc_slab_config)
   int kps;            // slab mode: K blocks of B per ring stage (one MMA commit per stage)
+  int tslots;         // TMEM accumulator slots: 0 = as many as fit (<= 4), 2 = two (DJINN_TSLOTS=2)
   int ldwait;         // slab mode: B-loader stage wait (0 spin, 1 poll + nanosleep back-off, 2 suspend hint)
   int obd;            // conv output: zero border of the stored output tensor (its consumer's pad)
   int lrn_size;
@@ -142,10 +143,11 @@ cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int C
                               int xu, int obd, int dt, cudaStream_t st);
 
 // --- LRN + max pooling fused (K4+K5): fp16 NHWC input (pitch Cpi, C channels, pads zero),
-// Caffe LRN across channels in fp32, Caffe MAX pooling of the LRN output (kernel 1 = no pool),
-// output in type dt with a grouped channel layout (gsz, gpitch, pitch Cpo; pads written as 0).
+// Caffe LRN across channels in fp32, Caffe MAX pooling (kernel 3, stride 2, pad 0) of the LRN
+// output; output in type dt with a grouped channel layout (gsz, gpitch, pitch Cpo; pads written
+// as 0) and a zero border of obd pixels (never written).  Each LRN value is computed once.
 cudaError_t launch_lrn_pool(const void* x, void* y, int64_t rows, int C, int Cpi, int H, int W, int OH, int OW,
-                            int kernel, int stride, int pad, int out_gsz, int out_gpitch, int Cpo, int size,
+                            int kernel, int stride, int pad, int out_gsz, int out_gpitch, int Cpo, int obd, int size,
                             float alpha, float beta, float k, int dt, cudaStream_t st);
 
 // --- pooling (K5), NHWC, Caffe ceil geometry ------------------------------------------------

@@ -126,6 +126,14 @@ static int ldwait_mode() {
   return m;
 }
 
+static int tslots_mode() {
+  static const int m = [] {
+    const char* e = getenv("DJINN_TSLOTS");
+    return e ? atoi(e) : 0;
+  }();
+  return m;
+}
+
 bool pdl_enabled() {
   static const bool on = [] {
     const char* e = getenv("DJINN_PDL");
@@ -727,9 +735,7 @@ void Net::build(const std::string& desc) {
         ++n_layers;
       }
       os = layout_for(i + 1, os);
-      lp.out = os;
       lp.in_buf = o.out_buf;
-      os.bdr = 0;  // the fused LRN + pool kernel writes no border
       lp.out = os;
       lp.out_buf = curbuf = pick_buf(os, o.out_buf);
       cur = os;
@@ -1020,6 +1026,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
         case OP_GEMM: {
           GemmGeom g = o.g;
           g.ldwait = ldwait_mode();
+          g.tslots = tslots_mode();
           g.M = (int)(n * o.ohw);
           g.Nimg = (int)n;
           const void* A = w->buf[o.in_buf];
@@ -1048,7 +1055,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           break;
         case OP_LRNPOOL:
           e = launch_lrn_pool(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.H, o.in.W, o.out.H, o.out.W,
-                              o.kernel, o.stride, o.pad, o.out.gsz, o.out.gpitch, o.out.Cp, o.lrn_size, o.alpha,
+                              o.kernel, o.stride, o.pad, o.out.gsz, o.out.gpitch, o.out.Cp, o.out.bdr, o.lrn_size, o.alpha,
                               o.beta, o.lrn_k, dt, st);
           break;
         case OP_SOFTMAX:
