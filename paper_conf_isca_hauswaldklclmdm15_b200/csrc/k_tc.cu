@@ -352,17 +352,10 @@ __device__ __forceinline__ void bias_act16(float (&v)[16], const uint32_t (&r)[1
   }
 }
 
-// 16 bias values starting at n (zeros at n >= nvalid); vector loads when the chunk is full.
-__device__ __forceinline__ void load_bias16(float (&b)[16], const float* __restrict__ bz, int n, int nvalid) {
-  if (n + 16 <= nvalid) {
+__device__ __forceinline__ void lds16(float (&b)[16], const float* s) {
 #pragma unroll
-    for (int q = 0; q < 4; ++q) *reinterpret_cast<float4*>(b + 4 * q) = __ldg(reinterpret_cast<const float4*>(bz + n) + q);
-  } else {
-#pragma unroll
-    for (int j = 0; j < 16; ++j) b[j] = n + j < nvalid ? __ldg(bz + n + j) : 0.f;
-  }
+  for (int q = 0; q < 4; ++q) *reinterpret_cast<float4*>(b + 4 * q) = reinterpret_cast<const float4*>(s)[q];
 }
-
 template <bool BF16>
 __device__ __forceinline__ uint32_t pack2(float a, float b) {
   if (BF16) {
@@ -512,6 +505,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   // bars: full[NST], empty[NST], tfull[4], tempty[4], sfull[2], sempty[2]
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * NST + 12);
   __shared__ uint32_t ktab[KTAB_MAX];
+  // per-epilogue-warp bias of the tile being drained, indexed by TMEM column (LRN path: by channel)
+  __shared__ __align__(16) float sbias[EPI_WARPS][256];
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + NST);
   const uint32_t tfull0 = smem_u32(bars + 2 * NST), tempty0 = smem_u32(bars + 2 * NST + 4);
   const uint32_t sfull0 = smem_u32(bars + 2 * NST + 8), sempty0 = smem_u32(bars + 2 * NST + 10);
@@ -973,6 +968,29 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         m = tc.m0 + r;
         mok = m < g.M;
       }
+      // The tile's bias goes to shared memory before the wait for its accumulator: per-chunk
+      // global bias loads in the drain loops had exposed an L2 round trip per 16-32 columns
+      // (ncu, IMC conv1: the first FADD after each load was the top stall, ~7k cycles per tile).
+      // (each warp keeps its own copy: no cross-warp barrier in the drain loop)
+      float* sb = sbias[warp];
+      {
+        __syncwarp();  // this warp's reads of the previous tile's table are done
+        const int ncols = g.zf * BN;
+        for (int c = lane; c < ncols; c += 32) {
+          float b = 0.f;
+          if (g.epi_lrn) {
+            if (c < g.zf * g.N) b = __ldg(bias + c);
+          } else if (g.xb > 1) {
+            const int dx = c / g.out_pitch, co = c - dx * g.out_pitch;
+            if (co < g.Co) b = __ldg(g.mode == GM_LC ? bias + (int64_t)tc.z0 * g.bias_zstride + dx * g.Co + co : bias + co);
+          } else {
+            const int zi = c / BN, nb = tc.n0 * BN + (c - zi * BN);
+            if (nb < g.N) b = __ldg(bias + (int64_t)(tc.z0 * g.zf + zi) * g.bias_zstride + nb);
+          }
+          sb[c] = b;
+        }
+        __syncwarp();
+      }
       {
         // one lane per warp polls the barrier (256 polling threads slowed the whole SM's
         // TMA stream ~3x); the warp then reconverges
@@ -1003,11 +1021,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           if (n_n >= N) { n_n = 0; ++zi_n; }
         };
         float bq[16];  // bias of the next chunk to convert (loaded one chunk ahead)
-        load_bias16(bq, bias, 0, Ctot);
+        lds16(bq, sb);
         auto convert = [&](int i, const uint32_t (&rr)[16], float (&v)[16]) {
           const int c0 = i * 16;
           bias_act16(v, rr, bq, g.act);
-          if (c0 + 16 < Ctot) load_bias16(bq, bias, c0 + 16, Ctot);
+          if (c0 + 16 < Ctot) lds16(bq, sb + c0 + 16);
           if (c0 + 16 > Ctot) {
 #pragma unroll
             for (int j = 0; j < 16; ++j) v[j] = c0 + j < Ctot ? v[j] : 0.f;
@@ -1072,12 +1090,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           ox0 = (tc.z0 - ly * OWb) * g.xb;
           pix0 = ((int64_t)m * g.OH + ly) * g.OW + ox0;
         }
-        const float* bb = g.mode == GM_LC ? bias + (int64_t)tc.z0 * g.bias_zstride : bias;
         int dx = 0, co0 = 0;
 #pragma unroll 1
         for (int c = 0; c < BN; c += 16) {
           float b[16];
-          load_bias16(b, g.mode == GM_LC ? bb + dx * g.Co : bb, co0, g.Co);
+          lds16(b, sb + c);
           uint32_t rr[16];
           tmem_ld16(tbase + (uint32_t)c, rr);
           tmem_wait_ld();
@@ -1099,14 +1116,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           const int z = tc.z0 * g.zf + zi;
           const int64_t pix = (g.mode == GM_LC) ? (int64_t)m * g.OH * g.OW + z : (g.mode == GM_CONV ? opix : (int64_t)m);
           const int goff = (g.mode == GM_CONV) ? z * g.cout_goff : 0;
-          const float* bz = bias + (int64_t)z * g.bias_zstride;
           const int nb0 = tc.n0 * BN;
 #pragma unroll 1
           for (int c = 0; c < BN; c += 32) {
             const bool two = c + 16 < BN;
             float b0[16], b1[16];
-            load_bias16(b0, bz, nb0 + c, g.N);  // bias loads in flight during the TMEM load
-            if (two) load_bias16(b1, bz, nb0 + c + 16, g.N);
+            lds16(b0, sb + zi * BN + c);
+            if (two) lds16(b1, sb + zi * BN + c + 16);
             uint32_t r0[16], r1[16];
             tmem_ld16(tbase + (uint32_t)(zi * BN + c), r0);
             if (two) tmem_ld16(tbase + (uint32_t)(zi * BN + c + 16), r1);
@@ -1164,7 +1180,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 int g_num_sms = 0;
 
 // dynamic shared memory of a slab-mode launch: B ring + two slabs + barriers (+ alignment slack)
-constexpr int SLAB_SMEM_MAX = 227 * 1024 - 1024;  // 227 KB per block minus the static ktab
+constexpr int SLAB_SMEM_MAX = 227 * 1024 - 1024 - 8192;  // 227 KB per block minus the static ktab and sbias
 template <int BN, int CG>
 int slab_smem(const GemmGeom& g, int stages) {
   using C = Cfg<BN, CG>;
