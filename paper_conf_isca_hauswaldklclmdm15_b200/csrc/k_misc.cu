@@ -253,28 +253,63 @@ cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, in
 // norm2+pool2).  The conv before it stores its bias+ReLU output in fp16 (plain layout, pitch
 // Cpi, channels >= C zero).
 //
-// Every input element's LRN is evaluated ONCE (the MUFU work is the kernel's floor): a warp
-// owns 16 channels of 32 adjacent input columns and walks down the rows of its band; the
-// vertical window max lives in registers (rows 2oy, 2oy+1, 2oy+2; row 2oy+2 also opens window
-// oy+1), the horizontal one takes two warp shuffles, and the even lanes 0..28 store output
-// pixels ox = (x0 + lane) / 2.  Warps start every 30 columns (2 columns of overlap).
-// Block: 32 x (C/16) threads = one column segment of one image band; grid (segments, rows, bands).
+// Every input element's LRN is evaluated once (the MUFU work -- lg2 + ex2 per element at 16
+// per clock per SM -- is the kernel's floor).  One block walks down the input rows of one image
+// band; each row (W pixels x Cpi channels, contiguous) is staged in shared memory by cp.async,
+// NBUF-1 rows ahead, with a 16-byte pad per pixel so that lanes reading consecutive pixels hit
+// distinct banks (direct global loads with a 32-lane pixel stride had run L1-bound at 90%).
+// Warp (seg, chunk) owns channels 16*chunk .. +15 of the 32 columns starting at 30*seg: the
+// vertical window max (rows 2oy, 2oy+1, 2oy+2; row 2oy+2 also opens window oy+1) lives in
+// registers, the horizontal one takes two warp shuffles, and the even lanes 0..28 store output
+// pixels ox = (30*seg + lane) / 2.
+constexpr int LRNPOOL_NBUF = 4;
+// 2^y on the FMA pipe (y >= -126): y = n + f with n = rint(y), |f| <= 1/2, 2^f by its degree-4
+// Taylor polynomial (relative error <= 4.2e-5), 2^n added to the exponent field.  Moves half of
+// the LRN's transcendental work off the MUFU (16 results per clock per SM).
+__device__ __forceinline__ float exp2_fma(float y) {
+  y = fmaxf(y, -126.f);
+  const float t = y + 12582912.f;  // 1.5 * 2^23: rint(y) in the low mantissa bits
+  const float n = t - 12582912.f;
+  const float f = y - n;
+  float p = fmaf(0.0096181291f, f, 0.0555041087f);
+  p = fmaf(p, f, 0.2402265070f);
+  p = fmaf(p, f, 0.6931471806f);
+  p = fmaf(p, f, 1.0f);
+  return __int_as_float(__float_as_int(p) + ((__float_as_int(t) - 0x4B400000) << 23));
+}
 template <typename TO>
-__global__ void __launch_bounds__(512) lrn_pool_kernel(const __half* __restrict__ x, TO* __restrict__ y, int C, int Cpi,
-                                                       int H, int W, int OH, int OW, int bands, int gsz, int gpitch,
-                                                       int Cpo, int obd, float an, float nbeta, float k) {
+__global__ void __launch_bounds__(1024) lrn_pool_kernel(const __half* __restrict__ x, TO* __restrict__ y, int C, int Cpi,
+                                                        int H, int W, int OH, int OW, int bands, int gsz, int gpitch,
+                                                        int Cpo, int obd, float an, float nbeta, float k) {
   pdl_trigger();
   pdl_wait();
-  const int lane = threadIdx.x, c0 = threadIdx.y * 16;
-  const int x0 = blockIdx.x * 30, xx = x0 + lane;
-  const int64_t r = blockIdx.y;
+  extern __shared__ __align__(16) uint8_t srows[];
+  const int RP = Cpi * 2 + 16;  // bytes per staged pixel
+  const int nch = C / 16;
+  const int lane = threadIdx.x, seg = threadIdx.y / nch, chunk = threadIdx.y - seg * nch;
+  const int c0 = chunk * 16;
+  const int xx = seg * 30 + lane;
+  const int64_t r = blockIdx.x;
   const int per_band = (OH + bands - 1) / bands;
-  const int oy0 = blockIdx.z * per_band, oy1 = min(OH, oy0 + per_band);
+  const int oy0 = blockIdx.y * per_band, oy1 = min(OH, oy0 + per_band);
   if (oy0 >= oy1) return;
+  const int tid = threadIdx.y * 32 + lane, nthr = blockDim.y * 32;
+  // staging: thread tid copies 16-byte piece q of pixels px0, px0 + pstep, ... (the launch makes
+  // the block size a multiple of the pieces per pixel, so (px, q) need no division per copy)
+  const int pieces_px = Cpi / 8, pstep = nthr / pieces_px;
+  const int q_st = tid % pieces_px, px0 = tid / pieces_px;
+  const __half* xr = x + r * H * (int64_t)W * Cpi + px0 * Cpi + q_st * 8;
+  const uint32_t sm0 = (uint32_t)__cvta_generic_to_shared(srows) + px0 * RP + q_st * 16;
+  auto stage = [&](int yy) {
+    const uint32_t dst0 = sm0 + (yy % LRNPOOL_NBUF) * W * RP;
+    const __half* src0 = xr + (int64_t)yy * W * Cpi;
+    for (int px = px0, i = 0; px < W; px += pstep, ++i)
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst0 + i * pstep * RP),
+                   "l"(src0 + (int64_t)i * pstep * Cpi)
+                   : "memory");
+  };
   const bool xin = xx < W;
-  const __half* xr = x + ((r * H) * (int64_t)W + (xin ? xx : W - 1)) * Cpi + c0;
-  // output channel positions of this thread's 16 channels (16 | gsz: a chunk never straddles groups)
-  const int grp = c0 / gsz, cin = c0 - grp * gsz;
+  const int grp = c0 / gsz, cin = c0 - grp * gsz;  // 16 | gsz: a chunk never straddles groups
   TO* yr = y + (r * (OH + 2 * obd) + obd) * (int64_t)(OW + 2 * obd) * Cpo + grp * gpitch + cin;
   const bool pad_writer = gpitch > gsz && cin + 16 == gsz;
   const bool has_lo = c0 >= 2, has_hi = c0 + 16 < C;
@@ -309,13 +344,21 @@ __global__ void __launch_bounds__(512) lrn_pool_kernel(const __half* __restrict_
     }
     emitted = oy;
   };
-  const int ylast = min(2 * oy1, H - 1);
-  for (int yy = 2 * oy0; yy <= ylast; ++yy) {
-    const __half* px = xr + (int64_t)yy * W * Cpi;
-    const uint4 ua = __ldg(reinterpret_cast<const uint4*>(px));
-    const uint4 ub = __ldg(reinterpret_cast<const uint4*>(px) + 1);
-    const uint32_t ulo = has_lo ? __ldg(reinterpret_cast<const unsigned int*>(px - 2)) : 0u;
-    const uint32_t uhi = has_hi ? __ldg(reinterpret_cast<const unsigned int*>(px + 16)) : 0u;
+  const int yfirst = 2 * oy0, ylast = min(2 * oy1, H - 1);
+  for (int yy = yfirst; yy < yfirst + LRNPOOL_NBUF - 1; ++yy) {
+    if (yy <= ylast) stage(yy);
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  }
+  for (int yy = yfirst; yy <= ylast; ++yy) {
+    asm volatile("cp.async.wait_group %0;" ::"n"(LRNPOOL_NBUF - 2) : "memory");  // row yy has landed
+    __syncthreads();  // ... for every thread, and every warp is done reading row yy - 1's buffer
+    if (yy + LRNPOOL_NBUF - 1 <= ylast) stage(yy + LRNPOOL_NBUF - 1);  // refills row yy - 1's buffer
+    asm volatile("cp.async.commit_group;" ::: "memory");
+    const uint8_t* px = srows + (yy % LRNPOOL_NBUF) * W * RP + (xin ? xx : W - 1) * RP + c0 * 2;
+    const uint4 ua = reinterpret_cast<const uint4*>(px)[0];
+    const uint4 ub = reinterpret_cast<const uint4*>(px)[1];
+    const uint32_t ulo = has_lo ? *reinterpret_cast<const uint32_t*>(px - 4) : 0u;
+    const uint32_t uhi = has_hi ? *reinterpret_cast<const uint32_t*>(px + 32) : 0u;
     float v[20];
     {
       const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&ulo));
@@ -332,23 +375,26 @@ __global__ void __launch_bounds__(512) lrn_pool_kernel(const __half* __restrict_
     float sq[20];
 #pragma unroll
     for (int j = 0; j < 20; ++j) sq[j] = v[j] * v[j];
-    float p2[19];
+    // sliding window sums s[j] = sq[j] + ... + sq[j + 4] (all terms >= 0: no cancellation)
+    float sw[16];
+    sw[0] = (sq[0] + sq[1]) + (sq[2] + sq[3]) + sq[4];
 #pragma unroll
-    for (int j = 0; j < 19; ++j) p2[j] = sq[j] + sq[j + 1];
+    for (int j = 1; j < 16; ++j) sw[j] = (sw[j - 1] - sq[j - 1]) + sq[j + 4];
     __half2 l[8];
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
-      const float s0 = (p2[2 * j] + p2[2 * j + 2]) + sq[2 * j + 4], s1 = (p2[2 * j + 1] + p2[2 * j + 3]) + sq[2 * j + 5];
+      const float s0 = sw[2 * j], s1 = sw[2 * j + 1];
       float r0, r1;
       asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(r0) : "f"(fmaf(an, s0, k)));
       asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(r1) : "f"(fmaf(an, s1, k)));
+#ifdef DJINN_LRN_POLY
+      r0 = exp2_fma(nbeta * r0);
+      r1 = exp2_fma(nbeta * r1);
+#else
       asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r0) : "f"(nbeta * r0));
       asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r1) : "f"(nbeta * r1));
+#endif
       l[j] = __floats2half2_rn(v[2 + 2 * j] * r0, v[3 + 2 * j] * r1);
-    }
-    if (!xin) {
-#pragma unroll
-      for (int j = 0; j < 8; ++j) l[j] = __float2half2_rn(0.f);
     }
     if ((yy & 1) == 0) {
       const int j = yy >> 1;
@@ -372,24 +418,34 @@ __global__ void __launch_bounds__(512) lrn_pool_kernel(const __half* __restrict_
 cudaError_t launch_lrn_pool(const void* x, void* y, int64_t rows, int C, int Cpi, int H, int W, int OH, int OW,
                             int kernel, int stride, int pad, int out_gsz, int out_gpitch, int Cpo, int obd, int size,
                             float alpha, float beta, float k, int dt, cudaStream_t st) {
-  if (size != 5 || kernel != 3 || stride != 2 || pad != 0 || C % 16 || Cpi % 8 || Cpi < C || C > 512 || Cpo % 8 ||
-      rows > 65535 || obd < 0)
+  const int segs = (W + 29) / 30;
+  if (size != 5 || kernel != 3 || stride != 2 || pad != 0 || C % 16 || Cpi % 8 || Cpi < C || Cpo % 8 ||
+      rows > 65535 || obd < 0 || segs * (C / 16) * 32 > 1024)
     return cudaErrorInvalidValue;
   if (out_gsz >= C) { out_gsz = C; out_gpitch = Cpo; }
   if (out_gsz % 16 || out_gpitch % 8) return cudaErrorInvalidValue;
-  const int segs = (W + 29) / 30;
-  // bands of output rows: enough warps for ~3 waves (each band re-reads one boundary input row)
-  const int64_t warps = (int64_t)segs * rows * (C / 16);
-  int bands = (int)std::min<int64_t>(std::max<int64_t>(1, (3 * 148 * 64 + warps - 1) / warps), OH);
-  dim3 g(segs, (unsigned)rows, bands), b(32, C / 16);
+  const size_t smem = (size_t)LRNPOOL_NBUF * W * (Cpi * 2 + 16);
+  if (smem > 100 * 1024) return cudaErrorInvalidValue;
+  // bands of output rows: enough blocks for ~4 waves (each band re-reads one boundary input row)
+  const int threads = segs * (C / 16) * 32;
+  if (threads % (Cpi / 8)) return cudaErrorInvalidValue;  // the staging loop's piece mapping
+  const int per_sm = std::max(1, std::min(2048 / threads, (int)((200 * 1024) / smem)));
+  int bands = (int)std::min<int64_t>(std::max<int64_t>(1, (4LL * 148 * per_sm + rows - 1) / rows), OH);
+  dim3 g((unsigned)rows, bands), b(32, segs * (C / 16));
   const float an = alpha / size;
-  if (dt == DT_F16)
-    launch_pdl(lrn_pool_kernel<__half>, g, b, 0, st, (const __half*)x, (__half*)y, C, Cpi, H, W, OH, OW, bands, out_gsz,
-               out_gpitch, Cpo, obd, an, -beta, k);
-  else
-    launch_pdl(lrn_pool_kernel<__nv_bfloat16>, g, b, 0, st, (const __half*)x, (__nv_bfloat16*)y, C, Cpi, H, W, OH, OW,
-               bands, out_gsz, out_gpitch, Cpo, obd, an, -beta, k);
-  return cudaGetLastError();
+  cudaError_t e;
+  if (dt == DT_F16) {
+    e = cudaFuncSetAttribute(lrn_pool_kernel<__half>, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+    if (e == cudaSuccess)
+      e = launch_pdl(lrn_pool_kernel<__half>, g, b, smem, st, (const __half*)x, (__half*)y, C, Cpi, H, W, OH, OW, bands,
+                     out_gsz, out_gpitch, Cpo, obd, an, -beta, k);
+  } else {
+    e = cudaFuncSetAttribute(lrn_pool_kernel<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+    if (e == cudaSuccess)
+      e = launch_pdl(lrn_pool_kernel<__nv_bfloat16>, g, b, smem, st, (const __half*)x, (__nv_bfloat16*)y, C, Cpi, H, W,
+                     OH, OW, bands, out_gsz, out_gpitch, Cpo, obd, an, -beta, k);
+  }
+  return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 // ------------------------------------------------------------------------------------------

@@ -134,6 +134,12 @@ static int tslots_mode() {
   return m;
 }
 
+// Which conv+LRN(+pool) triples run LRN + pool as a separate kernel (bit k = k-th LRN); the
+// others fuse LRN into the conv epilogue.  Measured on B200.
+#ifndef LRN_POOL_DEFAULT
+#define LRN_POOL_DEFAULT 2
+#endif
+
 bool pdl_enabled() {
   static const bool on = [] {
     const char* e = getenv("DJINN_PDL");
@@ -292,6 +298,7 @@ void Net::build(const std::string& desc) {
     const int gp = sh.gsz < sh.C ? sh.gpitch : sh.Cp;
     return (slab_on && L.stride == 1 && L.pad > 0 && gp % 64 == 0) ? L.pad : 0;
   };
+  int lrn_ordinal = 0;  // LRN layers after a conv seen so far (DJINN_LRN_POOL bit index)
   auto layout_for = [&](size_t from, Shape sh) {
     sh.Cp = sh.C;
     sh.gsz = sh.gpitch = 1 << 30;
@@ -627,19 +634,25 @@ void Net::build(const std::string& desc) {
         throw Error(DJINN_E_SHAPE, L.name + ": internal: input channel pitch not TMA-chunkable");
       // Caffe LRN right after (the activation of) this conv: fuse it into the epilogue when one
       // tile holds every channel of a pixel (all groups side by side in TMEM).
-      const char* lrn_sep = getenv("DJINN_LRN_POOL");
-      if (f16 && !lc && i + 1 < layers.size() && layers[i + 1].type == "LRN" && layers[i + 1].lrn_size == 5 &&
-          lrn_sep && lrn_sep[0] == '1' && L.num_output % 8 == 0) {
-        // Alternative (DJINN_LRN_POOL=1): the conv's epilogue stays bias + ReLU and stores fp16
-        // (only LRN reads it), and LRN + the MAX pooling after it run as one separate kernel.
-        // Measured slower than the epilogue fusion below.
+      const bool lrn_next = f16 && !lc && i + 1 < layers.size() && layers[i + 1].type == "LRN" &&
+                            layers[i + 1].lrn_size == 5;
+      // LRN + MAX pool (kernel 3, stride 2, pad 0) as one separate kernel instead of the epilogue
+      // fusion: bit k of DJINN_LRN_POOL (default LRN_POOL_DEFAULT) selects it for the k-th LRN.
+      const bool pool_next = i + 2 < layers.size() && layers[i + 2].type == "Pooling" && layers[i + 2].pool_max &&
+                             layers[i + 2].kernel == 3 && layers[i + 2].stride == 2 && layers[i + 2].pad == 0;
+      const int lrn_mask = getenv("DJINN_LRN_POOL") ? atoi(getenv("DJINN_LRN_POOL")) : LRN_POOL_DEFAULT;
+      const bool lrn_sep = lrn_next && pool_next && L.num_output % 16 == 0 && ((lrn_mask >> lrn_ordinal) & 1);
+      if (lrn_next) ++lrn_ordinal;
+      if (lrn_sep) {
+        // The conv's epilogue stays bias + ReLU and stores fp16 (only LRN reads it); LRN + the
+        // MAX pooling after it run as one kernel (k_misc.cu lrn_pool_kernel).
         lrn_pool_next = true;
         g.out_half = 1;
         o.out.Cp = rup(o.out.C, 16);
         o.out.gsz = o.out.gpitch = 1 << 30;
         g.out_pitch = o.out.Cp;
         g.write_cols = grp == 1 ? o.out.Cp : Cog;
-      } else if (f16 && !lc && i + 1 < layers.size() && layers[i + 1].type == "LRN" && layers[i + 1].lrn_size == 5) {
+      } else if (lrn_next) {
         const int bn = tc_pick_bn(g);
         if (Cog <= 256 && (grp == 1 || bn == Cog) && grp * bn <= 256) {
           const LayerSpec& R = layers[i + 1];
