@@ -33,19 +33,24 @@ def test_counts_match_the_oracle(app, prec):
 def test_plan_first_layer_transforms_and_lrn_fusion():
     imc = dj.djinn_describe(dj.net_description("imc"), dj.DJINN_BF16, 64)[0]
     assert "space-to-depth 4" in imc
-    assert "conv1+norm1" in imc and "conv2+norm2" in imc and "lrn-epilogue" in imc
+    # default (DJINN_LRN_POOL=2): norm1 in conv1's epilogue, norm2 + pool2 as one LRN+pool kernel
+    assert "conv1+norm1" in imc and "lrn-epilogue" in imc and "lrn+pool norm2+pool2" in imc
     assert "48x57x57/p64" in imc                      # s2d: 4*4*3 channels at a 128-byte pitch
     assert "96x27x27/p128" in imc                     # conv2 input: two groups of 48 at pitch 64
     face = dj.djinn_describe(dj.net_description("face"), dj.DJINN_FP16, 64)[0]
     assert "kx-unroll 18" in face and "KHxKW=11x1" in face and "xblock=8" in face   # 8 outputs per GEMM row
     assert "32x71x71/p64" in face and "x-unrolled-input=2" in face                  # M2 -> C3
     assert "taps/row=4" in face                                                      # L4-L6
-    os.environ["DJINN_LRN_POOL"] = "1"                       # alternative: separate LRN+pool kernel
-    try:
-        sep = dj.djinn_describe(dj.net_description("imc"), dj.DJINN_BF16, 64)[0]
-    finally:
-        del os.environ["DJINN_LRN_POOL"]
+    def plan_with(mask):
+        os.environ["DJINN_LRN_POOL"] = mask              # bit k: k-th LRN as a separate LRN+pool kernel
+        try:
+            return dj.djinn_describe(dj.net_description("imc"), dj.DJINN_BF16, 64)[0]
+        finally:
+            del os.environ["DJINN_LRN_POOL"]
+    sep = plan_with("3")
     assert "lrn+pool norm1+pool1" in sep and "lrn+pool norm2+pool2" in sep and "fp16-out" in sep
+    fused = plan_with("0")
+    assert "conv1+norm1" in fused and "conv2+norm2" in fused and "lrn+pool" not in fused
     fp32 = dj.djinn_describe(dj.net_description("imc"), dj.DJINN_FP32, 64)[0]
     assert "lrn norm1" in fp32 and "space-to-depth" not in fp32   # fp32 path: plain SIMT plan
 
