@@ -197,6 +197,10 @@ def main():
     ap.add_argument("--apps", default=",".join(APPS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--services", default=os.environ.get("DJINN_BENCH_SERVICES", "concurrent"),
+                    choices=["concurrent", "serial"],
+                    help="concurrent: each Tonic app on its own stream (the paper's concurrent services "
+                         "sharing one GPU, L203-211); serial: all apps on one stream")
     ap.add_argument("--profile-json", default=None, help="write per-op timings here")
     args = ap.parse_args()
     if args.impl == "reference":
@@ -236,9 +240,30 @@ def main():
         del w
     torch.cuda.synchronize()
 
+    # One stream per Tonic service: each app's batch is forked from the timing
+    # stream and joined back, so small services fill the gaps of large ones and, in host-fed
+    # mode, one app's H2D overlaps another's kernels and D2H.
+    concurrent = args.services == "concurrent"
+    app_streams = {a: (torch.cuda.Stream() if concurrent else stream) for a in apps}
+
+    def run_services(call):
+        if not concurrent:
+            for a in apps:
+                call(a, sh)
+            return
+        fork = torch.cuda.Event()
+        fork.record(stream)
+        for a in apps:
+            app_streams[a].wait_event(fork)
+            call(a, app_streams[a].cuda_stream)
+        for a in apps:
+            join = torch.cuda.Event()
+            join.record(app_streams[a])
+            stream.wait_event(join)
+
     def step():
-        for app in apps:
-            dj.djinn_forward(nets[app].handle, inputs[app], BATCH_ROWS[app], outputs[app], dj.DJINN_OUT_PROB, sh)
+        run_services(lambda a, s: dj.djinn_forward(nets[a].handle, inputs[a], BATCH_ROWS[a], outputs[a],
+                                                   dj.DJINN_OUT_PROB, s))
 
     def barrier():
         if world > 1:
@@ -340,8 +365,8 @@ def main():
         hout = {a: torch.empty(BATCH_ROWS[a], nets[a].out_elems).pin_memory() for a in apps}
 
         def step_host():
-            for a in apps:
-                dj.djinn_forward(nets[a].handle, hin[a], BATCH_ROWS[a], hout[a], dj.DJINN_OUT_PROB, sh)
+            run_services(lambda a, s: dj.djinn_forward(nets[a].handle, hin[a], BATCH_ROWS[a], hout[a],
+                                                       dj.DJINN_OUT_PROB, s))
         for _ in range(2):
             step_host()
         k = max(3, args.steps // 4)
@@ -365,7 +390,9 @@ def main():
                            "batch_rows_per_gpu": {a: BATCH_ROWS[a] for a in apps},
                            "queries_per_step_per_gpu": sum(BATCH_ROWS[a] / ROWS_PER_QUERY[a] for a in apps),
                            "l2": "step working set (~2 GB of inputs/activations) >> 126 MB L2",
-                           "parallelism": f"replica x{world}, query shards, no per-step collective"},
+                           "parallelism": f"replica x{world}, query shards, no per-step collective",
+                           "services": args.services,
+                           "host_fed_pipe_chunks": os.environ.get("DJINN_PIPE_CHUNKS", "auto (<=4 by copy size)")},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
                 "clocks": clk.summary(), "per_app": per_app,
                 "top_ops": [{k: o[k] for k in ("app", "op", "kind", "ms_total", "avg_us", "tflops", "gbs", "bound",

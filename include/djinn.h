@@ -112,10 +112,16 @@ DJINN_API int djinn_load_net(const char* desc, size_t desc_len, const float* wei
  *   output    : per out_mode (see DJINN_OUT_*), host or device (out_mem); must hold
  *               rows * out_elems_per_row floats (PROB/LOGITS) or rows int32 (ARGMAX).
  *   stream    : cudaStream_t to run on (NULL = legacy default stream).  The call is
- *               asynchronous with respect to the host for device buffers; with host
- *               buffers the copies are enqueued on the same stream and the caller must
- *               synchronise the stream (djinn_sync) before reading `output` or reusing
- *               `input`.
+ *               asynchronous with respect to the host.  With host buffers (the paper's
+ *               PCIe-fed service, L231-253) the rows are cut into 2 chunks when the copies
+ *               exceed 32 MB
+ *               (DJINN_PIPE_CHUNKS env overrides) and the library's own copy streams
+ *               overlap chunk i+1's H2D and chunk i-1's D2H with chunk i's kernels on
+ *               `stream`; host `input` is read as soon as the call is issued (not
+ *               ordered after earlier work on `stream`), and `stream` reaches the end of
+ *               this call only after the last D2H has landed.  The caller synchronises
+ *               `stream` (djinn_sync) before reading a host `output` or reusing `input`;
+ *               page-locked host buffers are needed for the copies to be asynchronous.
  * Thread safety: concurrent calls on one net are safe when they use different streams
  * (weights are read-only; each stream gets its own workspace).  Not concurrent with
  * djinn_free.

@@ -916,6 +916,11 @@ Workspace::~Workspace() {
   for (void* p : buf) if (p) cudaFree(p);
   if (in_stage) cudaFree(in_stage);
   if (out_stage) cudaFree(out_stage);
+  for (int s = 0; s < 2; ++s)
+    for (cudaEvent_t e : {in_ready[s], in_free[s], out_ready[s], out_free[s]})
+      if (e) cudaEventDestroy(e);
+  if (cin) cudaStreamDestroy(cin);
+  if (cout) cudaStreamDestroy(cout);
 }
 
 cudaEvent_t Net::prof_event() {
@@ -1003,23 +1008,68 @@ Workspace* Net::workspace(cudaStream_t st) {
 }
 
 // ============================================================================ forward
+// Host-fed pipeline depth: rows of one call are cut into this many chunks when the host
+// copies are large, so chunk i+1's H2D, chunk i's kernels and chunk i-1's D2H overlap (PCIe
+// is the bound in this mode).  DJINN_PIPE_CHUNKS overrides (1 = no split).
+static int pipe_chunks(size_t io_bytes) {
+  const char* v = getenv("DJINN_PIPE_CHUNKS");
+  if (v && atoi(v) > 0) return atoi(v);
+  return io_bytes >= (32u << 20) ? 2 : 1;   // measured on B200 (bench e2e): 2 >= 4 > 1
+}
+
 void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_mem, int mode, cudaStream_t st) {
   if (poisoned) throw Error(DJINN_E_CUDA, "net is poisoned by an earlier CUDA error");
   Workspace* w = workspace(st);
-  if (in_mem == DJINN_MEM_HOST && !w->in_stage)
+  const bool hin = in_mem == DJINN_MEM_HOST, hout = out_mem == DJINN_MEM_HOST;
+  if (hin && !w->in_stage)
     if (cudaMalloc(&w->in_stage, (size_t)max_rows * in_elems * 4) != cudaSuccess) throw Error(DJINN_E_NOMEM, "input staging");
-  if (out_mem == DJINN_MEM_HOST && !w->out_stage)
+  if (hout && !w->out_stage)
     if (cudaMalloc(&w->out_stage, (size_t)max_rows * out_elems * 4) != cudaSuccess) throw Error(DJINN_E_NOMEM, "output staging");
+  if ((hin || hout) && !w->cin) {
+    ck(cudaStreamCreateWithFlags(&w->cin, cudaStreamNonBlocking), "copy stream");
+    ck(cudaStreamCreateWithFlags(&w->cout, cudaStreamNonBlocking), "copy stream");
+    for (int s = 0; s < 2; ++s)
+      for (cudaEvent_t* e : {&w->in_ready[s], &w->in_free[s], &w->out_ready[s], &w->out_free[s]})
+        ck(cudaEventCreateWithFlags(e, cudaEventDisableTiming), "cudaEventCreate");
+  }
   const size_t out_row_bytes = mode == DJINN_OUT_ARGMAX ? 4 : (size_t)out_elems * 4;
-  std::atomic<int64_t>& launches = launch_counter();
-  for (int64_t r0 = 0; r0 < rows; r0 += max_rows) {
-    const int64_t n = std::min<int64_t>(max_rows, rows - r0);
-    const float* src = in + r0 * in_elems;
-    if (in_mem == DJINN_MEM_HOST) {
-      ck(cudaMemcpyAsync(w->in_stage, src, (size_t)n * in_elems * 4, cudaMemcpyHostToDevice, st), "input H2D");
-      src = w->in_stage;
+  // Chunk size: max_rows for device buffers; with host buffers the batch is split into
+  // pipe_chunks() chunks using two staging slots (one slot when two do not fit in max_rows).
+  int64_t cs = max_rows;
+  int slots = 1;
+  if (hin || hout) {
+    const int64_t nr = std::min<int64_t>(rows, max_rows);
+    const size_t io = (size_t)nr * ((hin ? in_elems * 4 : 0) + (hout ? out_row_bytes : 0));
+    const int P = pipe_chunks(io);
+    cs = std::max<int64_t>(1, (nr + P - 1) / P);
+    slots = 2 * cs <= max_rows ? 2 : 1;
+    if (slots == 1) cs = max_rows;
+    if (cs != w->pipe_cs) {
+      // slot boundaries moved: the new slots may overlap either old one, so drain both
+      for (int s2 = 0; s2 < 2; ++s2) {
+        ck(cudaStreamWaitEvent(w->cin, w->in_free[s2], 0), "event wait");
+        ck(cudaStreamWaitEvent(st, w->out_free[s2], 0), "event wait");
+      }
+      w->pipe_cs = cs;
     }
-    uint8_t* dst = out_mem == DJINN_MEM_HOST ? (uint8_t*)w->out_stage : (uint8_t*)out + r0 * out_row_bytes;
+  }
+  std::atomic<int64_t>& launches = launch_counter();
+  int last_slot = -1;
+  for (int64_t r0 = 0, c = 0; r0 < rows; r0 += cs, ++c) {
+    const int64_t n = std::min<int64_t>(cs, rows - r0);
+    const int sl = (int)(c % slots);
+    const float* src = in + r0 * in_elems;
+    if (hin) {
+      // H2D into slot `sl` once the kernels of its previous chunk have consumed it
+      float* stage = w->in_stage + (size_t)sl * cs * in_elems;
+      ck(cudaStreamWaitEvent(w->cin, w->in_free[sl], 0), "event wait");
+      ck(cudaMemcpyAsync(stage, src, (size_t)n * in_elems * 4, cudaMemcpyHostToDevice, w->cin), "input H2D");
+      ck(cudaEventRecord(w->in_ready[sl], w->cin), "event record");
+      ck(cudaStreamWaitEvent(st, w->in_ready[sl], 0), "event wait");
+      src = stage;
+    }
+    if (hout) ck(cudaStreamWaitEvent(st, w->out_free[sl], 0), "event wait");  // slot's previous D2H done
+    uint8_t* dst = hout ? (uint8_t*)w->out_stage + (size_t)sl * cs * out_row_bytes : (uint8_t*)out + r0 * out_row_bytes;
     const int pop = profile ? profile_op : -1;  // one timed op, or all (-1)
     if (profile) {
       std::lock_guard<std::mutex> lk(mu);
@@ -1081,13 +1131,21 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
         throw Error(DJINN_E_CUDA, o.name + ": " + cudaGetErrorString(e));
       }
       if (profile && pop == (int)i) ck(cudaEventRecord(prof_events[pbase + 1], st), "profile event");
+      if (i == 0 && hin) ck(cudaEventRecord(w->in_free[sl], st), "event record");  // pack has read the slot
     }
     if (profile && pop < 0) ck(cudaEventRecord(prof_events[pbase + ops.size()], st), "profile event");
-    if (out_mem == DJINN_MEM_HOST)
-      ck(cudaMemcpyAsync((uint8_t*)out + r0 * out_row_bytes, w->out_stage, (size_t)n * out_row_bytes,
-                         cudaMemcpyDeviceToHost, st),
+    if (hout) {
+      ck(cudaEventRecord(w->out_ready[sl], st), "event record");
+      ck(cudaStreamWaitEvent(w->cout, w->out_ready[sl], 0), "event wait");
+      ck(cudaMemcpyAsync((uint8_t*)out + r0 * out_row_bytes, dst, (size_t)n * out_row_bytes, cudaMemcpyDeviceToHost,
+                         w->cout),
          "output D2H");
+      ck(cudaEventRecord(w->out_free[sl], w->cout), "event record");
+      last_slot = sl;
+    }
   }
+  // The caller's stream completes only after the last D2H has landed in host memory.
+  if (last_slot >= 0) ck(cudaStreamWaitEvent(st, w->out_free[last_slot], 0), "event wait");
 }
 
 std::string Net::plan_string() const {

@@ -94,6 +94,11 @@ struct Workspace {
   std::vector<void*> buf;  // 0/1 ping-pong, 2 logits, 3.. dedicated bordered tensors (borders stay zero)
   float* in_stage = nullptr;
   void* out_stage = nullptr;
+  // host-fed mode: H2D on `cin`, D2H on `cout`, compute on the caller's stream; two staging
+  // slots, each with a "filled" and a "drained" event (Net::forward)
+  cudaStream_t cin = nullptr, cout = nullptr;
+  cudaEvent_t in_ready[2] = {}, in_free[2] = {}, out_ready[2] = {}, out_free[2] = {};
+  int64_t pipe_cs = 0;  // chunk rows of the last host-fed call (slot offsets depend on it)
   std::vector<CUtensorMap> tmA;  // per op (dense gemm) over its input buffer
   ~Workspace();
 };

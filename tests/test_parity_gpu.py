@@ -91,6 +91,29 @@ def test_chunking_and_host_buffers_match_device_path():
     np.testing.assert_array_equal(dev.numpy(), full)
 
 
+@pytest.mark.parametrize("in_host,out_host", [(True, True), (True, False), (False, True)])
+def test_host_fed_pipeline_matches_device_path(in_host, out_host, monkeypatch):
+    """Host-fed mode: the batch is cut into chunks whose H2D, kernels and
+    D2H overlap on three streams with two staging slots.  Back-to-back calls with different
+    chunk sizes and row counts (no sync in between) must equal the device path bitwise."""
+    app, prec = "dig", "bf16"
+    x = recipes.gen_input_rows(app, 0, 300, prec)
+    net = dj.DjinnNet(dj.net_description(app), blob(app, prec), prec, 128)
+    dev = net.forward(torch.from_numpy(x).cuda(), dj.DJINN_OUT_PROB).cpu()
+    xin = torch.from_numpy(x).pin_memory() if in_host else torch.from_numpy(x).cuda()
+    s = torch.cuda.Stream()
+    outs = []
+    for chunks, rows in ((4, 300), (1, 300), (3, 97), (7, 300), (2, 128), (5, 1)):
+        monkeypatch.setenv("DJINN_PIPE_CHUNKS", str(chunks))
+        o = torch.full((rows, 10), -1.0).pin_memory() if out_host else torch.full((rows, 10), -1.0, device="cuda")
+        dj.djinn_forward(net.handle, xin, rows, o, dj.DJINN_OUT_PROB, s.cuda_stream)
+        outs.append((rows, o))
+    dj.djinn_sync(net.handle, s.cuda_stream)
+    net.close()
+    for rows, o in outs:
+        assert torch.equal(o.cpu(), dev[:rows]), rows
+
+
 def test_rows_zero_and_error_paths():
     net = dj.DjinnNet(dj.net_description("pos"), blob("pos", "bf16"), "bf16", 16)
     out = torch.empty(0, 45, device="cuda")
