@@ -49,7 +49,15 @@ constexpr int BM = 128, BK = 64;
 // Warp roles: 0-7 epilogue, 8-11 TMA loaders, 12 TMEM allocator + MMA issuer.  A warp issues one
 // TMA box per ~375 cycles however large the box (tools/tma_bench3.cu: the rate scales with the
 // number of issuing warps, not with bytes), so stages are dealt round-robin to four loaders.
-constexpr int EPI_WARPS = 8, LOAD_WARP0 = 8, NLOAD = 4, MMA_WARP = 12, NUM_THREADS = 32 * 13;
+#ifndef DJINN_EPI_WG
+#define DJINN_EPI_WG 3
+#endif
+// Epilogue warpgroups take tiles round robin: each has EPI_WG MMA tile-times for its tile (the
+// epilogue is latency-bound, ncu: ~45 % issue-active; role timing: the MMA warp waited on TMEM
+// slots 44 % of IMC conv1 with 2 warpgroups).
+constexpr int EPI_WG = DJINN_EPI_WG;
+constexpr int EPI_WARPS = 4 * EPI_WG, LOAD_WARP0 = EPI_WARPS, NLOAD = EPI_WG == 3 ? 3 : 4, MMA_WARP = EPI_WARPS + NLOAD,
+              NUM_THREADS = 32 * (MMA_WARP + 1);
 
 constexpr int KTAB_MAX = 256;  // im2col producer: per-K-chunk (channel, kx, ky) table entries
 template <int BN, int CG = 1>
@@ -374,6 +382,11 @@ constexpr bool kDbgNoEpi = true;
 #else
 constexpr bool kDbgNoEpi = false;
 #endif
+#ifdef DJINN_DBG_LDONLY
+constexpr bool kDbgLdOnly = true;  // DJINN_DBG_LDONLY: plain epilogue loads TMEM, computes and stores nothing
+#else
+constexpr bool kDbgLdOnly = false;
+#endif
 #ifdef DJINN_DBG_NOB
 constexpr bool kDbgNoB = true;  // DJINN_DBG_NOB: the B operand is not loaded
 #else
@@ -506,7 +519,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * NST + 12);
   __shared__ uint32_t ktab[KTAB_MAX];
   // per-epilogue-warp bias of the tile being drained, indexed by TMEM column (LRN path: by channel)
-  __shared__ __align__(16) float sbias[EPI_WARPS][256];
+  // (one double-buffered table per warpgroup: 6 KB, so the slab ring keeps its stages)
+  __shared__ __align__(16) float sbias[EPI_WG][2][256];
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + NST);
   const uint32_t tfull0 = smem_u32(bars + 2 * NST), tempty0 = smem_u32(bars + 2 * NST + 4);
   const uint32_t sfull0 = smem_u32(bars + 2 * NST + 8), sempty0 = smem_u32(bars + 2 * NST + 10);
@@ -522,13 +536,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   const int tiles = mt * nt * zt;
   int slot_cols = 32;  // TMEM columns per accumulator slot (power of two >= zf*BN)
   while (slot_cols < g.zf * BN) slot_cols <<= 1;
-  // Accumulator slots: 4 when they fit in TMEM's 512 columns (zf * BN <= 128), else 2
-  // (launch_inst guarantees zf * BN <= 256).  Each warpgroup drains every other tile; with 2
-  // slots the MMA of tile t+2 waits for the epilogue of tile t to finish within ONE tile time,
-  // with 4 it may run 3 tiles ahead (IMC conv1: the epilogue's latency, not its work, had
-  // stalled the MMA).  g.tslots = 2 forces two.
-  const int nslots = (4 * slot_cols <= 512 && g.tslots != 2) ? 4 : 2;
-  const int slot_sh = nslots == 4 ? 2 : 1;
+  // Accumulator slots.  Every slot is drained by ONE warpgroup (slot = lt % nslots, warpgroup =
+  // lt % nwg with nwg dividing nslots), so its tfull / tempty phases are awaited in order and
+  // a parity wait can never alias a phase two uses ahead.  nwg = 3 (g.epi_wg, LRN epilogues):
+  // 3 slots when they fit (zf * BN <= 128).  nwg = 2: 4 slots when they fit (the MMA may run
+  // 3 tiles ahead; IMC conv1: the epilogue's latency had stalled the MMA).  Otherwise 2 slots
+  // drained by warpgroups 0-1.  g.tslots = 2 forces two.
+  const int wg_req = (EPI_WG == 3 && g.epi_wg == 3) ? 3 : 2;
+  const int nslots = g.tslots == 2 || 3 * slot_cols > 512 ? 2 : (wg_req == 3 ? 3 : 4);
+  const int nwg = nslots == 3 ? 3 : 2;
   int tcols = 32;
   while (tcols < nslots * slot_cols) tcols <<= 1;
 
@@ -540,7 +556,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     }
     for (int s = 0; s < 4; ++s) {
       mbar_init(tfull0 + 8 * s, 1);
-      mbar_init(tempty0 + 8 * s, (EPI_WARPS / 2) * CG);  // one warpgroup per tile; leader's: both CTAs'
+      mbar_init(tempty0 + 8 * s, 4 * CG);  // one warpgroup per tile; leader's: both CTAs'
     }
     for (int s = 0; s < 2; ++s) {
       mbar_init(sfull0 + 8 * s, 1);
@@ -830,8 +846,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       int s = 0, lt = 0;
       uint32_t ph = 0;
       for (int t = cid; t < tiles; t += ncl, ++lt) {
-        const int slot = lt & (nslots - 1);
-        const uint32_t use = (uint32_t)(lt >> slot_sh);
+        const int slot = lt % nslots;
+        const uint32_t use = (uint32_t)(lt / nslots);
         {
           STAT_T0();
           mbar_wait_sleep(tempty0 + 8 * slot, (use & 1) ^ 1);
@@ -926,21 +942,21 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       }
     }
   } else if (warp < EPI_WARPS) {
-    // ---- epilogue (warps 0-7): TMEM -> registers -> bias + act (+ LRN) -> global ----
-    // The two warpgroups alternate tiles: warpgroup h drains TMEM slot h (local tiles lt with
-    // lt % 2 == h), so every thread owns one whole output row (pixel) of its tile: the LRN
-    // channel window slides through registers with no halo recomputation, and each warpgroup
-    // has two MMA tile-times for its tile.
+    // ---- epilogue (warps 0 .. EPI_WARPS-1): TMEM -> registers -> bias + act (+ LRN) -> global ----
+    // The warpgroups take tiles round robin: warpgroup h drains local tiles lt with
+    // lt % nwg == h (warpgroups >= nwg idle), so every thread owns one whole output row (pixel)
+    // of its tile: the LRN channel window slides through registers with no halo recomputation,
+    // and each warpgroup has nwg MMA tile-times for its tile.
     const int quarter = warp & 3, wg = warp >> 2;
     const uint32_t lane_base = (uint32_t)(quarter * 32) << 16;
     const int r = quarter * 32 + lane;
-    int lt = 0;
+    int lt = 0, wtile = 0;
     for (int t = cid; t < tiles; t += ncl, ++lt) {
-      if ((lt & 1) != wg) continue;
+      if (lt % nwg != wg) continue;
       TileCoord tc = tile_coord(g, t, mt, nt, CG);
       tc.m0 += (int)rank * BM;  // this CTA's rows of the pair tile
-      const int slot = lt & (nslots - 1);
-      const uint32_t use = (uint32_t)(lt >> slot_sh);
+      const int slot = lt % nslots;
+      const uint32_t use = (uint32_t)(lt / nslots);
       int m;       // GEMM row (dense, LC)
       bool mok;
       // conv: output pixel (img, oy, ox) of the row (ox: first pixel of its x block) and its
@@ -971,12 +987,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       // The tile's bias goes to shared memory before the wait for its accumulator: per-chunk
       // global bias loads in the drain loops had exposed an L2 round trip per 16-32 columns
       // (ncu, IMC conv1: the first FADD after each load was the top stall, ~7k cycles per tile).
-      // (each warp keeps its own copy: no cross-warp barrier in the drain loop)
-      float* sb = sbias[warp];
+      // The warpgroup's 128 threads fill one of its two tables (alternating per tile) and meet
+      // at a named barrier; a warp can be at most one tile ahead of the others, so the table it
+      // fills is never one that a slower warp still reads.
+      float* sb = sbias[wg][wtile & 1];
+      ++wtile;
       {
-        __syncwarp();  // this warp's reads of the previous tile's table are done
         const int ncols = g.zf * BN;
-        for (int c = lane; c < ncols; c += 32) {
+        for (int c = r; c < ncols; c += 128) {
           float b = 0.f;
           if (g.epi_lrn) {
             if (c < g.zf * g.N) b = __ldg(bias + c);
@@ -989,7 +1007,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           }
           sb[c] = b;
         }
-        __syncwarp();
+        asm volatile("bar.sync %0, 128;" ::"r"(2 + wg) : "memory");
       }
       {
         // one lane per warp polls the barrier (256 polling threads slowed the whole SM's
@@ -1128,6 +1146,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             if (two) tmem_ld16(tbase + (uint32_t)(zi * BN + c + 16), r1);
             tmem_wait_ld();
             const int nb = nb0 + c;
+            if (kDbgLdOnly) continue;
             if (mok && nb < g.write_cols) {
               float v[16];
               bias_act16(v, r0, b0, g.act);
@@ -1180,7 +1199,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 int g_num_sms = 0;
 
 // dynamic shared memory of a slab-mode launch: B ring + two slabs + barriers (+ alignment slack)
-constexpr int SLAB_SMEM_MAX = 227 * 1024 - 1024 - 8192;  // 227 KB per block minus the static ktab and sbias
+constexpr int SLAB_SMEM_MAX = 227 * 1024 - 1024 - EPI_WG * 2048;  // 227 KB per block minus the static ktab and sbias
 template <int BN, int CG>
 int slab_smem(const GemmGeom& g, int stages) {
   using C = Cfg<BN, CG>;

@@ -95,6 +95,7 @@ struct GemmGeom {
   int stages;         // slab mode: B ring stages (runtime; set by tc_slab_config)
   int kps;            // slab mode: K blocks of B per ring stage (one MMA commit per stage)
   int tslots;         // TMEM accumulator slots: 0 = as many as fit (<= 4), 2 = two (DJINN_TSLOTS=2)
+  int epi_wg;         // epilogue warpgroups draining tiles: 3 (3 slots) or 2 (up to 4 slots)
   int ldwait;         // slab mode: B-loader stage wait (0 spin, 1 poll + nanosleep back-off, 2 suspend hint)
   int obd;            // conv output: zero border of the stored output tensor (its consumer's pad)
   int lrn_size;

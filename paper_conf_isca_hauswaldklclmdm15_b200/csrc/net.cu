@@ -126,6 +126,18 @@ static int ldwait_mode() {
   return m;
 }
 
+// Epilogue warpgroups per tile stream (GemmGeom::epi_wg): 3 for LRN epilogues (latency-bound:
+// IMC conv1+norm1 516 -> 440 us on B200), 2 elsewhere, where a 4th TMEM slot of MMA lookahead
+// is worth more (IMC conv5 164 -> 132 us).  DJINN_EPI_WG=2/3 forces one for every GEMM.
+static int epi_wg_mode(const GemmGeom& g) {
+  static const int m = [] {
+    const char* e = getenv("DJINN_EPI_WG");
+    return e ? atoi(e) : 0;
+  }();
+  if (m == 2 || m == 3) return m;
+  return g.epi_lrn ? 3 : 2;
+}
+
 static int tslots_mode() {
   static const int m = [] {
     const char* e = getenv("DJINN_TSLOTS");
@@ -1090,6 +1102,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           GemmGeom g = o.g;
           g.ldwait = ldwait_mode();
           g.tslots = tslots_mode();
+          g.epi_wg = epi_wg_mode(g);
           g.M = (int)(n * o.ohw);
           g.Nimg = (int)n;
           const void* A = w->buf[o.in_buf];
