@@ -16,6 +16,10 @@ L = [f"# {tag} bench summary (bench.py default run on {d['n_gpus']} x B200)\n",
      f"value {d['value']:.0f} mixed queries/s, {d['ms_per_step']:.3f} ms/step, dtype {d['dtype']}, "
      f"launches {d['gpu_launches']} ({d['gpu_launches'] / d['steps']:.0f}/step), clocks {d['clocks']}\n",
      f"e2e (pinned host buffers): {d['e2e']['value']:.0f} q/s, {d['e2e']['ms_per_step']:.2f} ms/step\n" if d.get("e2e") else "",
+     (f"concurrent services (one stream per app): {d['concurrent_services']['value']:.0f} q/s, "
+      f"{d['concurrent_services']['ms_per_step']:.3f} ms/step"
+      + (f"; host-fed {d['concurrent_services']['e2e']['ms_per_step']:.2f} ms/step" if d['concurrent_services'].get('e2e') else "")
+      + "\n") if d.get("concurrent_services") else "",
      f"cpu_baseline (fp64 oracle, {d['cpu_baseline']['cores']} threads): {d['cpu_baseline']['value']:.2f} q/s\n"
      if d.get("cpu_baseline") else "",
      f"roofline: {json.dumps(r)}\n",
