@@ -368,6 +368,18 @@ def main():
                                                        dj.DJINN_OUT_PROB, s), concurrent)
         for _ in range(2):
             step_host()
+        # per-app host-fed throughput and the PCIe bandwidth each service needs to run at its
+        # device-resident rate (the paper's bandwidth-requirement study, Figs. 11-13)
+        for a in apps:
+            k = max(3, args.steps // 4)
+            t = timed(lambda a=a: dj.djinn_forward(nets[a].handle, hin[a], BATCH_ROWS[a], hout[a],
+                                                   dj.DJINN_OUT_PROB, sh), k) / k
+            byts = (hin[a].numel() + hout[a].numel()) * 4
+            q = BATCH_ROWS[a] / ROWS_PER_QUERY[a]
+            per_app[a]["host_fed"] = {
+                "queries_per_s": q * world / (t / 1e3), "ms_per_batch": t,
+                "bytes_per_query": byts / q, "pcie_gbs_achieved": byts / (t / 1e3) / 1e9,
+                "pcie_gbs_needed_at_device_rate": byts / (per_app[a]["ms_per_batch"] / 1e3) / 1e9}
         k = max(3, args.steps // 4)
         t = timed(step_host, k) / k
         e2e = {"value": sum(BATCH_ROWS[a] / ROWS_PER_QUERY[a] for a in apps) * world / (t / 1e3), "unit": "queries/s",

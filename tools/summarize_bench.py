@@ -26,6 +26,15 @@ L = [f"# {tag} bench summary (bench.py default run on {d['n_gpus']} x B200)\n",
      "| app | queries/s | ms/batch | roofline ms | frac |", "|---|---|---|---|---|"]
 for a, v in d["per_app"].items():
     L.append(f"| {a} | {v['queries_per_s']:.0f} | {v['ms_per_batch']:.3f} | {v['roofline_ms']:.3f} | {v['roofline_frac']:.3f} |")
+if any("host_fed" in v for v in d["per_app"].values()):
+    L += ["", "host-fed (pinned H2D + D2H per batch, one app alone):", "",
+          "| app | queries/s | ms/batch | bytes/query | PCIe GB/s achieved | GB/s needed at device rate |",
+          "|---|---|---|---|---|---|"]
+    for a, v in d["per_app"].items():
+        h = v.get("host_fed")
+        if h:
+            L.append(f"| {a} | {h['queries_per_s']:.0f} | {h['ms_per_batch']:.3f} | {h['bytes_per_query']:.0f} | "
+                     f"{h['pcie_gbs_achieved']:.1f} | {h['pcie_gbs_needed_at_device_rate']:.0f} |")
 L += ["", "| app/op | kind | avg us | roofline us | TF/s | GB/s | bound |", "|---|---|---|---|---|---|---|"]
 for o in d["top_ops"]:
     L.append(f"| {o['app']}/{o['op']} | {o['kind']} | {o['avg_us']:.1f} | {o['roofline_us']:.1f} | {o['tflops']:.1f} | "
