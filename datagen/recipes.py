@@ -10,6 +10,10 @@ restated in DESIGN.md sec 3):
 * DIG: pixels k/256, k ~ U{0..255}, 1x28x28; a query is 100 images (L156).
 * ASR: N(0,1) per feature (CMVN-like), 440-dim rows; a query is 548 rows (L158).
 * POS/CHK/NER: U(-1,1) window vectors (300 / 300 / 375); a query is 28 rows (L159-161).
+* POS/CHK/NER with the on-GPU SENNA lookup (``*_ids``): per window word
+  the table indices, word index floor(V * u^3) (skewed toward frequent words, Zipf-like),
+  the other features uniform; tables U(-1,1) (the same marginal as the window vectors
+  above), followed by exactly the base app's MLP weights.
 * Weights: raw_W ~ U(-1,1) * sqrt(3 / fan_in), then multiplied per output channel
   by a stored calibration scale; bias = stored per-channel shift + jitter * U(-1,1).
   The calibration vectors are written by ``oracle/calibrate.py`` (which calls only
@@ -34,8 +38,16 @@ CALIB_DIR = os.path.join(os.path.dirname(os.path.abspath(__file__)), "calib")
 INPUT_SHAPE = {
     "imc": (3, 227, 227), "dig": (1, 28, 28), "face": (3, 152, 152), "asr": (440,),
     "pos": (300,), "chk": (300,), "ner": (375,),
+    "pos_ids": (15,), "chk_ids": (15,), "ner_ids": (30,),
 }
-ROWS_PER_QUERY = {"imc": 1, "dig": 100, "face": 1, "asr": 548, "pos": 28, "chk": 28, "ner": 28}
+ROWS_PER_QUERY = {"imc": 1, "dig": 100, "face": 1, "asr": 548, "pos": 28, "chk": 28, "ner": 28,
+                  "pos_ids": 28, "chk_ids": 28, "ner_ids": 28}
+# token-id apps: (base app whose MLP follows, window, table vocabularies) -- the tables' dims
+# live in the net description; the generator only needs the index ranges
+ID_APPS = {"pos_ids": ("pos", 5, (130000, 5, 455)), "chk_ids": ("chk", 5, (130000, 5, 45)),
+           "ner_ids": ("ner", 5, (130000, 5, 2, 2, 2, 2))}
+ID_TABLE_DIMS = {"pos_ids": (50, 5, 5), "chk_ids": (50, 5, 5), "ner_ids": (50, 5, 5, 5, 5, 5)}
+_TID_TABLES = 90
 
 _TID_NOISE, _TID_IMG = 1, 2
 CALIB_SEED_XOR = 0xCA11B
@@ -84,6 +96,12 @@ def gen_input_rows(app: str, start_row: int, n_rows: int, grid: str = "fp32",
         x = rng.normal(seed, _TID_NOISE, start_row * per, n_rows * per).reshape((n_rows,) + shp)
     elif app in ("pos", "chk", "ner"):
         x = rng.uniform(seed, _TID_NOISE, start_row * per, n_rows * per, -1.0, 1.0).reshape((n_rows,) + shp)
+    elif app in ID_APPS:
+        _, window, vocab = ID_APPS[app]
+        u = rng.uniform(seed, _TID_NOISE, start_row * per, n_rows * per).reshape(n_rows, window, len(vocab))
+        u[:, :, 0] = u[:, :, 0] ** 3
+        x = np.floor(u * np.asarray(vocab, dtype=np.float64)).reshape(n_rows, per)
+        return x.astype(np.float32)      # indices: exact integers, no grid rounding
     else:
         raise ValueError(app)
     return rng.round_to_grid(x, grid)
@@ -142,6 +160,12 @@ def gen_weights(app: str, grid: str = "fp32", calib: dict | None = None) -> List
 
     Returns a list of {"layer", "type", "w", "b"} in net order.  Biases are kept in
     fp32 (the GPU path keeps bias in fp32 for every precision)."""
+    if app in ID_APPS:               # lookup tables, then the base app's MLP
+        base, _, vocab = ID_APPS[app]
+        n = int(sum(v * d for v, d in zip(vocab, ID_TABLE_DIMS[app])))
+        tab = rng.uniform(rng.app_seed(app), _TID_TABLES, 0, n, -1.0, 1.0)
+        return [{"layer": "emb", "type": "Embedding", "w": rng.round_to_grid(tab, grid),
+                 "b": np.zeros(0, np.float32)}] + gen_weights(base, grid)
     calib = load_calib(app) if calib is None else calib
     out = []
     for p, e in enumerate(calib["params"]):

@@ -21,7 +21,8 @@ _M1 = np.uint64(0xBF58476D1CE4E5B9)
 _M2 = np.uint64(0x94D049BB133111EB)
 
 # Seeds: 0x15CA2015 ^ app_id.
-APP_IDS = {"imc": 1, "dig": 2, "face": 3, "asr": 4, "pos": 5, "chk": 6, "ner": 7}
+APP_IDS = {"imc": 1, "dig": 2, "face": 3, "asr": 4, "pos": 5, "chk": 6, "ner": 7,
+           "pos_ids": 8, "chk_ids": 9, "ner_ids": 10}
 
 
 def app_seed(app: str) -> int:

@@ -103,6 +103,15 @@ class OracleNet:
                 e.update(co=co, k=k, stride=s, w_shape=(OH, OW, co, C, k, k),
                          b_shape=(co, OH, OW), fan_in=C * k * k)
                 shape = (co, OH, OW)
+            elif t == "Embedding":
+                # SENNA window lookup (ops.embedding): input = window * T indices per row
+                p = _one(L, "embedding_param")
+                window, vocab, dims = _one(p, "window", 1), list(p["vocab"]), list(p["dim"])
+                if len(vocab) != len(dims) or shape != (window * len(vocab),):
+                    raise ValueError("Embedding: input must hold window * tables indices")
+                e.update(window=window, vocab=vocab, dims=dims,
+                         w_shape=(int(sum(v * d for v, d in zip(vocab, dims))),), b_shape=(0,), fan_in=1)
+                shape = (window * int(sum(dims)),)
             elif t == "InnerProduct":
                 no = _one(_one(L, "inner_product_param"), "num_output")
                 K = int(np.prod(shape))
@@ -145,6 +154,8 @@ class OracleNet:
             return ops.conv2d(x, w, b, L["stride"], L["pad"], L["group"])
         if t == "LocallyConnected":
             return ops.local(x, w, b, L["stride"])
+        if t == "Embedding":
+            return ops.embedding(x.reshape(x.shape[0], -1), w, L["window"], L["vocab"], L["dims"])
         if t == "InnerProduct":
             return ops.inner_product(x.reshape(x.shape[0], -1), w, b)
         if t in ("ReLU", "Sigmoid", "TanH", "HardTanh"):

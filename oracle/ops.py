@@ -132,3 +132,36 @@ def argmax(x):
     out = np.empty(N, dtype=np.int32)
     lib().orc_argmax(_p(x), N, D, out.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)))
     return out
+
+
+def embedding(ids, tables, window: int, vocab, dims):
+    """SENNA window feature vector ("SENNA ... [builds]
+    word vectors" for the NLP services; window approach of the cited SENNA work [ext: ref 19]).
+
+    ids    : [rows, window * T] per word w the T feature indices (word, caps, suffix / tag /
+             gazetteer ...), word-major: ids[r, w*T + t].
+    tables : flat fp64, table t = [vocab[t], dims[t]] C-order, tables back to back.
+    Row r of the result is concat over w of concat over t of table_t[ids[r, w*T+t]], i.e.
+    out[r, w*D + sum(dims[:t]) + j] with D = sum(dims).  An index that is not an integer in
+    [0, vocab[t]) selects the zero vector (reading R17).
+    Written as the plain definition: one lookup per (row, word, table)."""
+    ids = np.asarray(ids, dtype=np.float64)
+    tables = np.asarray(tables, dtype=np.float64).ravel()
+    T = len(vocab)
+    D = int(sum(dims))
+    rows = ids.shape[0]
+    out = np.zeros((rows, window * D), dtype=np.float64)
+    base = 0
+    mats = []
+    for t in range(T):
+        mats.append(tables[base: base + vocab[t] * dims[t]].reshape(vocab[t], dims[t]))
+        base += vocab[t] * dims[t]
+    for r in range(rows):
+        for w in range(window):
+            col = w * D
+            for t in range(T):
+                v = ids[r, w * T + t]
+                if v == np.floor(v) and 0 <= v < vocab[t]:
+                    out[r, col: col + dims[t]] = mats[t][int(v)]
+                col += dims[t]
+    return out

@@ -208,3 +208,56 @@ def test_softmax_textbook_and_invariants():
 def test_argmax_ties_lowest_index():
     z = np.array([[0.0, 3.0, 1.0, 3.0], [5.0, 5.0, 5.0, 5.0]])
     np.testing.assert_array_equal(ops.argmax(z), [1, 0])
+
+
+# ---------------------------------------------------------------- SENNA window lookup (f3)
+def test_embedding_hand_example():
+    """Window 2 over tables A (3 x 2) and B (2 x 1), word-major ids (a0, b0, a1, b1):
+    the row is A[a0] ++ B[b0] ++ A[a1] ++ B[b1] (SENNA window concatenation)."""
+    A = np.array([[1., 2.], [3., 4.], [5., 6.]])
+    B = np.array([[7.], [8.]])
+    tables = np.concatenate([A.ravel(), B.ravel()])
+    ids = np.array([[2, 1, 0, 0], [1, 0, 1, 1]], dtype=np.float32)
+    y = ops.embedding(ids, tables, 2, [3, 2], [2, 1])
+    np.testing.assert_array_equal(y, [[5, 6, 8, 1, 2, 7], [3, 4, 7, 3, 4, 8]])
+
+
+def test_embedding_equals_one_hot_matmul():
+    """Lookup = one-hot(ids) @ table for every (word, table) block."""
+    r = np.random.default_rng(5)
+    vocab, dims, window = [7, 3, 4], [4, 2, 3], 3
+    tabs = [r.standard_normal((v, d)) for v, d in zip(vocab, dims)]
+    ids = np.stack([r.integers(0, v, size=(11, window)) for v in vocab], axis=2).reshape(11, -1)
+    y = ops.embedding(ids, np.concatenate([t.ravel() for t in tabs]), window, vocab, dims)
+    blocks = []
+    for w in range(window):
+        for t, v in enumerate(vocab):
+            onehot = np.eye(v)[ids[:, w * len(vocab) + t]]
+            blocks.append(onehot @ tabs[t])
+    np.testing.assert_allclose(y, np.concatenate(blocks, axis=1), rtol=0, atol=0)
+
+
+def test_embedding_invalid_index_selects_zero_vector():
+    tables = np.arange(1., 7.)                    # one table 3 x 2
+    ids = np.array([[-1.], [3.], [1.5], [2.]])
+    y = ops.embedding(ids, tables, 1, [3], [2])
+    np.testing.assert_array_equal(y, [[0, 0], [0, 0], [0, 0], [5, 6]])
+
+
+@pytest.mark.parametrize("app", ["pos_ids", "chk_ids", "ner_ids"])
+def test_id_nets_equal_base_net_on_gathered_windows(app):
+    """An *_ids net = lookup followed by exactly the base app's MLP; its input is 4 B per
+    feature index instead of 4 B per window-vector element."""
+    from datagen import recipes
+    from oracle import OracleNet
+    from oracle.calibrate import net_text
+    W = recipes.gen_weights(app, "bf16")
+    x = recipes.gen_input_rows(app, 0, 20, "bf16")
+    net = OracleNet(net_text(app))
+    base = OracleNet(net_text(app[:3]))
+    assert net.n_layers() == base.n_layers() + 1
+    assert base.input_shape[0] / net.input_shape[0] >= 12      # >= 12x fewer input bytes per row
+    lg, _ = net.forward(x, W)
+    emb = ops.embedding(x, W[0]["w"], net.layers[1]["window"], net.layers[1]["vocab"], net.layers[1]["dims"])
+    lg2, _ = base.forward(emb, W[1:])
+    np.testing.assert_array_equal(lg, lg2)
