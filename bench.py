@@ -197,6 +197,8 @@ def main():
     ap.add_argument("--apps", default=",".join(APPS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-ids", action="store_true", help="skip the token-id NLP services (SENNA lookup)")
+    ap.add_argument("--profile-json", default=None, help="write per-op timings here")
     ap.add_argument("--no-concurrent", action="store_true",
                     help="skip the extra concurrent-services measurement (each app on its own stream)")
     args = ap.parse_args()
@@ -386,6 +388,35 @@ def main():
                "ms_per_step": t, "h2d_bytes_per_step": int(sum(hin[a].numel() * 4 for a in apps)),
                "d2h_bytes_per_step": int(sum(hout[a].numel() * 4 for a in apps))}
 
+    # ---- NLP services with the on-GPU SENNA lookup: queries carry feature
+    # indices (4 B per word and feature) instead of window vectors; device-resident and
+    # host-fed q/s at the same batch as the window-vector services
+    ids = None
+    if not args.no_ids and any(a in apps for a in ("pos", "chk", "ner")):
+        ids = {}
+        for base in ("pos", "chk", "ner"):
+            if base not in apps:
+                continue
+            a = base + "_ids"
+            rows = BATCH_ROWS[base]
+            w = recipes.flat_blob(recipes.gen_weights(a, grid))
+            net = dj.DjinnNet(dj.net_description(a), w, grid, rows, local)
+            r0, nrows = parallel.weak_shard(rows, rank)
+            xd = torch.from_numpy(recipes.gen_input_rows(a, r0, nrows, grid)).cuda()
+            od = torch.empty(rows, net.out_elems, device="cuda")
+            xh, oh = xd.cpu().pin_memory(), torch.empty(rows, net.out_elems).pin_memory()
+            q = rows / ROWS_PER_QUERY[a]
+            res = {}
+            for tag, xi, oo in (("device", xd, od), ("host_fed", xh, oh)):
+                for _ in range(3):
+                    dj.djinn_forward(net.handle, xi, rows, oo, dj.DJINN_OUT_PROB, sh)
+                k = max(5, args.steps // 2)
+                t = timed(lambda: dj.djinn_forward(net.handle, xi, rows, oo, dj.DJINN_OUT_PROB, sh), k) / k
+                res[tag] = {"queries_per_s": q * world / (t / 1e3), "ms_per_batch": t}
+            res["host_fed"]["bytes_per_query"] = (xh.numel() + oh.numel()) * 4 / q
+            ids[a] = res
+            net.close()
+
     # ---- concurrent services (one stream per app): device-resident and host-fed steps
     conc = None
     if not args.no_concurrent:
@@ -420,7 +451,8 @@ def main():
                            "parallelism": f"replica x{world}, query shards, no per-step collective",
                            "services": "serial (one stream, PDL-chained); see concurrent_services",
                            "host_fed_pipe_chunks": os.environ.get("DJINN_PIPE_CHUNKS", "auto (<=4 by copy size)")},
-                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "concurrent_services": conc, "gpu_launches": int(launches),
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "concurrent_services": conc, "nlp_token_ids": ids,
+                "gpu_launches": int(launches),
                 "clocks": clk.summary(), "per_app": per_app,
                 "top_ops": [{k: o[k] for k in ("app", "op", "kind", "ms_total", "avg_us", "tflops", "gbs", "bound",
                                                "roofline_us")} for o in ops[:12]]}

@@ -81,12 +81,20 @@ enum { DJINN_OUT_PROB = 0, DJINN_OUT_ARGMAX = 1, DJINN_OUT_LOGITS = 2 };
  *                    stride), InnerProduct (num_output), ReLU, Sigmoid, TanH, HardTanh,
  *                    LRN (local_size, alpha, beta, k; ACROSS_CHANNELS), Pooling
  *                    (pool MAX|AVE, kernel_size, stride, pad; Caffe ceil geometry),
- *                    Dropout (identity at inference), Softmax (last).  Copied.
+ *                    Dropout (identity at inference), Softmax (last), and Embedding
+ *                    (embedding_param: window, then `vocab: V dim: D` per table; only
+ *                    directly after an Input of window * tables values): the SENNA
+ *                    window lookup the NLP apps run before DjiNN (L104), done in the
+ *                    service -- row input = per word the T table indices (word-major,
+ *                    exact integers as float32; an index outside [0, V) or not an
+ *                    integer selects the zero vector), output = the concatenated
+ *                    window vector.  Copied.
  *   weights        : canonical blob, little-endian float32: for each parametrised layer
  *                    in file order its weights then its bias, C-order, shapes
  *                      Convolution      W[Co][Ci/group][k][k],  b[Co]
  *                      LocallyConnected W[OH][OW][Co][Ci][k][k], b[Co][OH][OW]
  *                      InnerProduct     W[No][K] with K in Caffe (c,h,w) order, b[No]
+ *                      Embedding        the tables [V_t][D_t] back to back, no bias
  *                    May be NULL: the weight arena is then left uninitialised, to be
  *                    filled through djinn_weight_arena (e.g. an NCCL broadcast from a
  *                    rank that loaded the same description with weights).

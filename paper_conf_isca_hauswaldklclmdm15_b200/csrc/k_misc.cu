@@ -207,6 +207,47 @@ cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int 
 }
 
 // ------------------------------------------------------------------------------------------
+// SENNA window lookup (kernels.h launch_embed).  One thread per output column: consecutive
+// threads copy consecutive elements of one table row, so each (word, table) lookup is one
+// coalesced read of dim[t] elements; the row's indices are L1-resident broadcasts.
+template <typename T>
+__global__ void embed_kernel(const float* __restrict__ x, const T* __restrict__ tab, T* __restrict__ y, int64_t rows,
+                             EmbedGeom eg, int Cp) {
+  pdl_trigger();
+  pdl_wait();
+  const int in_row = eg.window * eg.T, Dw = eg.window * eg.D;
+  const int64_t total = rows * Cp;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / Cp;
+    const int c = (int)(i - r * Cp);
+    T v = cvt<T>(0.f);
+    if (c < Dw) {
+      const int w = c / eg.D;
+      int j = c - w * eg.D, t = 0;
+      while (j >= eg.dim[t]) j -= eg.dim[t++];
+      const float id = __ldg(x + r * in_row + w * eg.T + t);
+      if (id >= 0.f && id < (float)eg.vocab[t] && id == floorf(id))
+        v = tab[eg.toff[t] + (int64_t)id * eg.dim[t] + j];
+    }
+    y[i] = v;
+  }
+}
+
+cudaError_t launch_embed(const float* x, const void* tables, void* y, int64_t rows, const EmbedGeom& eg, int Cp, int dt,
+                         cudaStream_t st) {
+  const int T = 256;
+  const int g = min(nblocks(rows * Cp, T), 148 * 16);
+  if (dt == DT_F32)
+    launch_pdl(embed_kernel<float>, dim3(g), dim3(T), 0, st, x, (const float*)tables, (float*)y, rows, eg, Cp);
+  else if (dt == DT_F16)
+    launch_pdl(embed_kernel<__half>, dim3(g), dim3(T), 0, st, x, (const __half*)tables, (__half*)y, rows, eg, Cp);
+  else
+    launch_pdl(embed_kernel<__nv_bfloat16>, dim3(g), dim3(T), 0, st, x, (const __nv_bfloat16*)tables,
+               (__nv_bfloat16*)y, rows, eg, Cp);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------
 // K4: Caffe LRN across channels.  y = x * (k + alpha/size * sum_{window} x^2)^-beta.
 // One thread per (pixel, channel); the channel window is contiguous in NHWC.
 template <typename T>

@@ -111,6 +111,20 @@ struct GemmGeom {
 cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f, int xs,
                               int Ho, int Wo, int Cp, int dt, cudaStream_t st);
 
+// --- SENNA window lookup (K0 variant) ------------------------------------
+// x: float32 [rows][window * T] feature indices, word-major (x[r][w*T + t]);
+// tables: the path's type, table t = [vocab[t]][dim[t]] at element offset toff[t];
+// y[r][w*D + sum(dim[:t]) + j] = tables_t[x[r][w*T+t]][j], D = sum(dim), pitch Cp (pad
+// columns zero).  An index that is not an integer in [0, vocab[t]) gives the zero vector.
+constexpr int EMBED_MAX_TABLES = 8;
+struct EmbedGeom {
+  int window, T, D;
+  int vocab[EMBED_MAX_TABLES], dim[EMBED_MAX_TABLES];
+  long long toff[EMBED_MAX_TABLES];
+};
+cudaError_t launch_embed(const float* x, const void* tables, void* y, int64_t rows, const EmbedGeom& eg, int Cp, int dt,
+                         cudaStream_t st);
+
 // --- SIMT fp32 implicit GEMM (K7; exact fp32 FFMA accumulation) --------------------------
 // B: [Z][N][K] fp32 (K unpadded), bias fp32.
 cudaError_t launch_simt_gemm(const GemmGeom& g, const float* A, const float* B, const float* bias,

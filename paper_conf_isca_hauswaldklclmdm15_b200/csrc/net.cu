@@ -284,6 +284,19 @@ void Net::build(const std::string& desc) {
       s.lrn_k = p ? (float)p->getf("k", 1.0) : 1.f;
       if (p && p->gets("norm_region", "ACROSS_CHANNELS") != "ACROSS_CHANNELS")
         throw Error(DJINN_E_UNSUPPORTED, s.name + ": only ACROSS_CHANNELS LRN");
+    } else if (s.type == "Embedding") {
+      const PNode* p = L.block("embedding_param");
+      if (!p) throw Error(DJINN_E_PARSE, s.name + ": missing embedding_param");
+      s.window = p->geti("window", 1);
+      auto v = p->scalars.find("vocab"), d = p->scalars.find("dim");
+      if (v == p->scalars.end() || d == p->scalars.end() || v->second.size() != d->second.size())
+        throw Error(DJINN_E_PARSE, s.name + ": embedding_param needs one dim per vocab");
+      for (auto& x : v->second) s.vocab.push_back(atoi(x.c_str()));
+      for (auto& x : d->second) s.edim.push_back(atoi(x.c_str()));
+      if (s.window <= 0 || s.vocab.empty() || (int)s.vocab.size() > EMBED_MAX_TABLES)
+        throw Error(DJINN_E_SHAPE, s.name + ": window / number of tables");
+      for (size_t t = 0; t < s.vocab.size(); ++t)
+        if (s.vocab[t] <= 0 || s.edim[t] <= 0) throw Error(DJINN_E_SHAPE, s.name + ": vocab / dim");
     } else if (act_of(s.type) >= 0 || s.type == "Dropout" || s.type == "Softmax") {
     } else {
       throw Error(DJINN_E_UNSUPPORTED, "layer type '" + s.type + "'");
@@ -358,25 +371,60 @@ void Net::build(const std::string& desc) {
   else if (d.size() == 3) { cur.C = d[0]; cur.H = d[1]; cur.W = d[2]; }
   else throw Error(DJINN_E_SHAPE, "Input must have 1 or 3 dims");
   if (cur.C <= 0 || cur.H <= 0 || cur.W <= 0) throw Error(DJINN_E_SHAPE, "bad Input dims");
-  cur = layout_for(1, cur);
-  cur.bdr = 0;  // the pack writes no border (a padded first conv then runs on im2col TMA)
-  if (cur.gsz < cur.C) throw Error(DJINN_E_UNSUPPORTED, "grouped first convolution on a 16-bit path");
-  in_elems = (int64_t)cur.C * cur.H * cur.W;
-
+  for (size_t i = 2; i < layers.size(); ++i)
+    if (layers[i].type == "Embedding") throw Error(DJINN_E_UNSUPPORTED, layers[i].name + ": Embedding must follow Input");
+  const bool emb = layers.size() > 1 && layers[1].type == "Embedding";
   Op pk;
   pk.kind = OP_PACK;
   pk.name = "pack";
-  pk.in = cur;
-  pk.out = cur;
   pk.in_buf = -1;
   pk.out_buf = 0;
-  ops.push_back(pk);
-  int curbuf = 0;
   n_layers = 0;
   n_params = 0;
   size_t arena_off = 0;
+  if (emb) {
+    // SENNA window lookup: the pack gathers the window vector from the
+    // tables in the arena instead of converting one.  Its output is laid out for layer 2.
+    const LayerSpec& E = layers[1];
+    const int T = (int)E.vocab.size();
+    if (d.size() != 1 || cur.C != E.window * T)
+      throw Error(DJINN_E_SHAPE, E.name + ": Input must hold window * tables indices per row");
+    pk.embed = 1;
+    pk.name = E.name;
+    cur.Cp = cur.C;
+    pk.in = cur;
+    pk.eg.window = E.window;
+    pk.eg.T = T;
+    pk.eg.D = 0;
+    int64_t telems = 0;
+    for (int t = 0; t < T; ++t) {
+      pk.eg.vocab[t] = E.vocab[t];
+      pk.eg.dim[t] = E.edim[t];
+      pk.eg.toff[t] = telems;
+      pk.eg.D += E.edim[t];
+      telems += (int64_t)E.vocab[t] * E.edim[t];
+    }
+    in_elems = cur.C;
+    Shape es;
+    es.C = E.window * pk.eg.D;
+    cur = layout_for(2, es);
+    pk.out = cur;
+    pk.w_off = arena_off;
+    arena_off += ((size_t)telems * (f16 ? 2 : 4) + 255) & ~(size_t)255;
+    n_params += telems;
+    ++n_layers;
+  } else {
+    cur = layout_for(1, cur);
+    cur.bdr = 0;  // the pack writes no border (a padded first conv then runs on im2col TMA)
+    if (cur.gsz < cur.C) throw Error(DJINN_E_UNSUPPORTED, "grouped first convolution on a 16-bit path");
+    in_elems = (int64_t)cur.C * cur.H * cur.W;
+    pk.in = cur;
+    pk.out = cur;
+  }
+  ops.push_back(pk);
+  int curbuf = 0;
 
-  for (size_t i = 1; i < layers.size(); ++i) {
+  for (size_t i = emb ? 2 : 1; i < layers.size(); ++i) {
     const LayerSpec& L = layers[i];
     if (L.type != "Softmax") ++n_layers;
     if (L.type == "Dropout") continue;
@@ -784,7 +832,10 @@ void Net::build(const std::string& desc) {
     const Shape& oin = (o.kind == OP_GEMM && o.g.mode != GM_DENSE) ? o.orig_in : o.in;
     const double in_e = (double)oin.C * oin.H * oin.W, out_e = (double)o.out.C * o.out.H * o.out.W;
     switch (o.kind) {
-      case OP_PACK: o.bytes_row = in_e * 4 + in_e * es; break;
+      case OP_PACK:
+        // lookup: indices in, window vector out, one table row read per (word, table)
+        o.bytes_row = o.embed ? in_e * 4 + 2.0 * out_e * es : in_e * 4 + in_e * es;
+        break;
       case OP_GEMM: {
         const GemmGeom& g = o.g;
         double kreal;
@@ -845,6 +896,21 @@ void Net::load_weights(const float* w, size_t n, int mem) {
   std::vector<uint8_t> host(arena_bytes, 0);
   size_t off = 0;  // floats into the canonical blob
   for (Op& o : ops) {
+    if (o.kind == OP_PACK && o.embed) {  // lookup tables, converted to the path's type
+      int64_t telems = 0;
+      for (int t = 0; t < o.eg.T; ++t) telems += (int64_t)o.eg.vocab[t] * o.eg.dim[t];
+      uint8_t* dst = host.data() + o.w_off;
+      for (int64_t e = 0; e < telems; ++e) {
+        const float v = w[off + e];
+        if (!f16) { reinterpret_cast<float*>(dst)[e] = v; continue; }
+        uint16_t bits;
+        if (dt == DT_BF16) { __nv_bfloat16 h = __float2bfloat16_rn(v); memcpy(&bits, &h, 2); }
+        else { __half h = __float2half_rn(v); memcpy(&bits, &h, 2); }
+        reinterpret_cast<uint16_t*>(dst)[e] = bits;
+      }
+      off += telems;
+      continue;
+    }
     if (o.kind != OP_GEMM) continue;
     const GemmGeom& g = o.g;
     uint8_t* wdst = host.data() + o.w_off;
@@ -1095,6 +1161,10 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
       if (profile && (pop < 0 || pop == (int)i)) ck(cudaEventRecord(prof_events[pbase + (pop < 0 ? i : 0)], st), "profile event");
       switch (o.kind) {
         case OP_PACK:
+          if (o.embed) {
+            e = launch_embed(src, (const uint8_t*)arena + o.w_off, w->buf[0], n, o.eg, o.out.Cp, dt, st);
+            break;
+          }
           e = launch_pack_input(src, w->buf[0], n, o.in.C, o.in.H, o.in.W, o.xform, o.xf, o.xs, o.out.H, o.out.W, o.out.Cp,
                                 dt, st);
           break;
@@ -1185,6 +1255,7 @@ std::string Net::plan_string() const {
         << (o.g.mode == GM_CONV && o.g.a_tiled ? " block=" + std::to_string(o.g.bx) + "x" + std::to_string(o.g.by) + "x" +
                                                   std::to_string(o.g.bn) : std::string())
         << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << (o.g.out_half ? " fp16-out" : "") << "]";
+    if (o.kind == OP_PACK && o.embed) s << " [embedding window " << o.eg.window << " tables " << o.eg.T << " D " << o.eg.D << "]";
     if (o.kind == OP_PACK && o.xform) s << " [" << (o.xform == 1 ? "space-to-depth " : "kx-unroll ") << o.xf << (o.xs > 1 ? " step " + std::to_string(o.xs) : std::string()) << "]";
     s << "\n";
   }

@@ -41,6 +41,8 @@ struct LayerSpec {
   int lrn_size = 5;
   float alpha = 1.f, beta = 0.75f, lrn_k = 1.f;
   std::vector<int> dims;
+  int window = 1;                  // Embedding: words per window, tables' vocabularies and dims
+  std::vector<int> vocab, edim;
 };
 
 enum OpKind { OP_PACK, OP_GEMM, OP_LRN, OP_POOL, OP_SOFTMAX, OP_LRNPOOL };
@@ -74,6 +76,9 @@ struct Op {
   // by xf (= conv stride), 2 kx-unroll of a stride-1 kernel of width xf
   int xform = 0, xf = 1, xs = 1;  // xs: kx-unroll x step (packed pixel j starts at input x = j*xs)
   Shape orig_in;                // the layer's input before the transform
+  // SENNA window lookup in place of the pack (embed = 1): see EmbedGeom (kernels.h)
+  int embed = 0;
+  EmbedGeom eg{};
   int orig_k = 0;               // original kernel size
   // lrn
   int lrn_size = 5;

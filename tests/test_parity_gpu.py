@@ -8,7 +8,7 @@ import paper_conf_isca_hauswaldklclmdm15_b200 as dj
 from datagen import recipes
 
 from parity import (FP32_PROB_TOL, REL_LOGIT_TOL, TOP1_MIN, blob, compare_16bit, compare_fp32,
-                    oracle_rows)
+                    oracle_net, oracle_rows)
 
 pytestmark = pytest.mark.gpu
 
@@ -152,3 +152,58 @@ def test_concurrent_streams_share_read_only_weights():
     dj.djinn_sync(net.handle, s2.cuda_stream)
     net.close()
     assert torch.equal(o1, ref) and torch.equal(o2, ref)
+
+
+# ---------------------------------------------------------------- SENNA lookup
+ID_APPS = ["pos_ids", "chk_ids", "ner_ids"]
+
+
+@pytest.mark.parametrize("prec", ["fp32", "bf16", "fp16"])
+@pytest.mark.parametrize("app", ID_APPS)
+def test_token_id_nets_match_oracle(app, prec):
+    n = 1000
+    x = recipes.gen_input_rows(app, 0, n, prec)
+    lg_ref, pr_ref = oracle_rows(app, x, prec)
+    net = dj.DjinnNet(dj.net_description(app), blob(app, prec), prec, n)
+    xt = torch.from_numpy(x).cuda()
+    lg = net.forward(xt, dj.DJINN_OUT_LOGITS).cpu().numpy()
+    pr = net.forward(xt, dj.DJINN_OUT_PROB).cpu().numpy()
+    net.close()
+    if prec == "fp32":
+        r = compare_fp32(pr, pr_ref, lg, lg_ref)
+        assert r["prob_max_abs"] <= FP32_PROB_TOL, r
+    else:
+        r = compare_16bit(lg, lg_ref)
+        assert r["rel_max"] <= REL_LOGIT_TOL and r["top1_decidable"] >= TOP1_MIN, r
+    print(app, prec, r)
+
+
+@pytest.mark.parametrize("app", ID_APPS)
+def test_token_id_net_equals_base_net_on_gathered_windows(app):
+    """Lookup + MLP on the GPU == the base app's GPU path fed the oracle-gathered window
+    vectors, bitwise: the lookup is exact and the MLP kernels see the same operands."""
+    from oracle import ops
+    prec, n = "bf16", 777
+    x = recipes.gen_input_rows(app, 0, n, prec)
+    W = recipes.gen_weights(app, prec)
+    L = oracle_net(app).layers[1]
+    win = ops.embedding(x, W[0]["w"], L["window"], L["vocab"], L["dims"]).astype(np.float32)
+    a = dj.DjinnNet(dj.net_description(app), blob(app, prec), prec, n)
+    b = dj.DjinnNet(dj.net_description(app[:3]), blob(app[:3], prec), prec, n)
+    la = a.forward(torch.from_numpy(x).cuda(), dj.DJINN_OUT_LOGITS).cpu()
+    lb = b.forward(torch.from_numpy(win).cuda(), dj.DJINN_OUT_LOGITS).cpu()
+    a.close()
+    b.close()
+    assert torch.equal(la, lb)
+
+
+def test_token_id_invalid_indices_select_zero_vectors():
+    app, prec, n = "pos_ids", "bf16", 300
+    x = recipes.gen_input_rows(app, 0, n, prec)
+    x[::7, 0] = -1.0            # word index below range
+    x[1::7, 3] = 130000.0       # word index == vocab
+    x[2::7, 5] = 2.5            # non-integer suffix index
+    lg_ref, _ = oracle_rows(app, x, prec)
+    lg = run_gpu(app, prec, x)
+    r = compare_16bit(lg, lg_ref)
+    assert r["rel_max"] <= REL_LOGIT_TOL, r

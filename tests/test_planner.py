@@ -10,7 +10,7 @@ import paper_conf_isca_hauswaldklclmdm15_b200 as dj
 from oracle import OracleNet
 from oracle.calibrate import net_text
 
-APPS = ["imc", "dig", "face", "asr", "pos", "chk", "ner"]
+APPS = ["imc", "dig", "face", "asr", "pos", "chk", "ner"] + ["pos_ids", "chk_ids", "ner_ids"]
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -88,3 +88,16 @@ def test_describe_argument_errors():
     with pytest.raises(dj.DjinnError) as e:
         dj.djinn_describe(dj.net_description("pos"), dj.DJINN_BF16, 0)
     assert e.value.code == dj.DJINN_E_INVAL
+
+
+def test_embedding_plan_and_errors():
+    plan = dj.djinn_describe(dj.net_description("ner_ids"), dj.DJINN_BF16, 64)[0]
+    assert "[embedding window 5 tables 6 D 75]" in plan and "375x1x1/p384" in plan
+    bad = dj.net_description("pos_ids").replace("dim: 15", "dim: 16")
+    with pytest.raises(dj.DjinnError) as e:
+        dj.djinn_describe(bad, dj.DJINN_BF16, 64)
+    assert e.value.code == dj.DJINN_E_SHAPE
+    bad = dj.net_description("pos_ids").replace("vocab: 455 dim: 5", "vocab: 455")
+    with pytest.raises(dj.DjinnError) as e:
+        dj.djinn_describe(bad, dj.DJINN_BF16, 64)
+    assert e.value.code == dj.DJINN_E_PARSE
