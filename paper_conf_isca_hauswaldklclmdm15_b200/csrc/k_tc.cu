@@ -491,7 +491,7 @@ __device__ __forceinline__ int num_m_tiles(const GemmGeom& g, int cg = 1) {
 }
 
 // ---------------------------------------------------------------- the kernel
-template <int BN, bool BF16, int CG, bool SLAB>
+template <int BN, bool BF16, int CG, bool SLAB, int KSUB = BK / 16>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const GemmGeom g, const float* __restrict__ bias, void* __restrict__ Y) {
@@ -887,8 +887,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 const uint64_t ad = a_hi | (uint64_t)(abase + (e & 0x3FFFFFu));
                 const uint64_t bd = b_hi | (uint64_t)(bstage + (uint32_t)i * (C::B_BYTES >> 4));
                 const uint32_t acc0 = (e >> 22) & 1u ? 0u : 1u;
+                // KSUB = 3: the K block's last 16 channels are zero padding (g.kv16)
 #pragma unroll
-                for (int k = 0; k < (kDbgNoMma ? 0 : BK / 16); ++k) {
+                for (int k = 0; k < (kDbgNoMma ? 0 : KSUB); ++k) {
                   if (CG == 2) mma_f16_2sm(d, ad + 2 * k, bd + 2 * k, idesc, k ? 1u : acc0);
                   else mma_f16(d, ad + 2 * k, bd + 2 * k, idesc, k ? 1u : acc0);
                 }
@@ -1208,12 +1209,12 @@ int slab_smem(const GemmGeom& g, int stages) {
   return 1024 + ring + 2 * slab + (2 * stages + 12) * 8 + 16;
 }
 
-template <int BN, bool BF16, int CG, bool SLAB>
+template <int BN, bool BF16, int CG, bool SLAB, int KSUB = BK / 16>
 cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtensorMap* tmB, const float* bias, void* Y,
                         cudaStream_t st) {
   using C = Cfg<BN, CG>;
   static int attr_set = 0;  // benign race: idempotent attribute set
-  auto kern = tc_gemm_kernel<BN, BF16, CG, SLAB>;
+  auto kern = tc_gemm_kernel<BN, BF16, CG, SLAB, KSUB>;
   const int smem = SLAB ? slab_smem<BN, CG>(g, g.stages) : C::SMEM;
   if (SLAB && (g.stages < 2 || smem > SLAB_SMEM_MAX)) return cudaErrorInvalidValue;
   if (attr_set < smem) {
@@ -1251,6 +1252,13 @@ cudaError_t launch_bn(const GemmGeom& g, int bn, const CUtensorMap* tmA, const C
                       void* Y, cudaStream_t st) {
   if (g.slab) {  // slab convolutions run on CTA pairs only
     if (g.cg != 2) return cudaErrorInvalidValue;
+    if (g.kv16 == 3) {
+      switch (bn) {
+        case 96: return launch_inst<96, BF16, 2, true, 3>(g, tmA, tmB, bias, Y, st);
+        case 128: return launch_inst<128, BF16, 2, true, 3>(g, tmA, tmB, bias, Y, st);
+        default: break;
+      }
+    }
     switch (bn) {
       case 96: return launch_inst<96, BF16, 2, true>(g, tmA, tmB, bias, Y, st);
       case 128: return launch_inst<128, BF16, 2, true>(g, tmA, tmB, bias, Y, st);

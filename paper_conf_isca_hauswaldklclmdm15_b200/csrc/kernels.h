@@ -93,6 +93,9 @@ struct GemmGeom {
   int slab, Hv, Wv;
   int slab_parts, slab_rows;  // the slab is loaded as slab_parts TMA boxes of slab_rows rows
   int stages;         // slab mode: B ring stages (runtime; set by tc_slab_config)
+  int kv16;           // slab mode, one 64-channel chunk per tap: 16-channel K sub-steps holding
+                      //   real channels (3 for 48 of 64: the 4th is zero padding and gets no MMA,
+                      //   a compile-time variant of the kernel); 4 otherwise
   int kps;            // slab mode: K blocks of B per ring stage (one MMA commit per stage)
   int tslots;         // TMEM accumulator slots: 0 = as many as fit (<= 4), 2 = two (DJINN_TSLOTS=2)
   int epi_wg;         // epilogue warpgroups draining tiles: 3 (3 slots) or 2 (up to 4 slots)

@@ -537,6 +537,7 @@ void Net::build(const std::string& desc) {
         throw Error(DJINN_E_UNSUPPORTED, L.name + ": input channel layout does not match the grouping");
       const bool grouped_layout = cur.gsz < cur.C;
       g.Cgp = (grp == 1) ? cur.Cp : (grouped_layout ? cur.gpitch : Cg);
+      int creal = (grp == 1) ? cur.C : Cg;  // real (unpadded) channels of a tap
       g.cin_goff = grouped_layout ? cur.gpitch : Cg;
       // First layer with few channels on the tensor-core path: repack the input so that K
       // is dense.  Strided kernels: space-to-depth by the stride (k x k / s  ->  ceil(k/s)^2
@@ -551,6 +552,7 @@ void Net::build(const std::string& desc) {
             pk.xf = o.xf = f;
             pk.out = Shape();
             pk.out.C = f * f * cur.C; pk.out.H = Hs; pk.out.W = Ws; pk.out.Cp = tap_pitch(f * f * cur.C);
+            creal = pk.out.C;
             g.H = Hs; g.W = Ws; g.Cp_in = g.Cgp = pk.out.Cp;
             g.KH = g.KW = ks;
             g.stride = 1;
@@ -672,6 +674,11 @@ void Net::build(const std::string& desc) {
           g.slab_parts = (R + 255) / 256;
           g.slab_rows = rup((R + g.slab_parts - 1) / g.slab_parts, 8);
           o.ohw = Hv * Wv;
+          // taps of 48 real channels in a 64-channel chunk (IMC conv1 after space-to-depth,
+          // conv2's groups): the 4th 16-channel K sub-step multiplies zero weights, so the
+          // kernel variant with 3 MMAs per K block skips it (DJINN_KSKIP=0: off)
+          const char* ks = getenv("DJINN_KSKIP");
+          g.kv16 = (g.Cgp == 64 && creal > 32 && creal <= 48 && g.kxs == 1 && g.xb <= 1 && !(ks && ks[0] == '0')) ? 3 : 4;
         }
       }
       if (!g.slab && o.in.bdr > 0) {  // a bordered input read by im2col: pad-0 conv over the stored grid
@@ -1248,7 +1255,8 @@ std::string Net::plan_string() const {
         << " act=" << o.g.act << " bn=" << o.bn << " cg=" << o.g.cg << " cw=" << o.g.cw << " zf=" << o.g.zf << " KHxKW=" << o.g.KH << "x"
         << o.g.KW << (o.g.xb > 1 ? " xblock=" + std::to_string(o.g.xb) : std::string())
         << (o.g.slab ? " slab=" + std::to_string(o.g.Hv) + "x" + std::to_string(o.g.Wv) + ":" + std::to_string(o.g.slab_parts) + "x" +
-                           std::to_string(o.g.slab_rows) + " stages=" + std::to_string(o.g.stages) + "x" + std::to_string(o.g.kps)
+                           std::to_string(o.g.slab_rows) + " stages=" + std::to_string(o.g.stages) + "x" + std::to_string(o.g.kps) +
+                           (o.g.kv16 == 3 ? std::string(" mma/kblock=3") : std::string())
                      : std::string())
         << (o.g.kxs > 1 ? " x-unrolled-input=" + std::to_string(o.g.kxs) : std::string())
         << (o.g.lcg > 1 ? " taps/row=" + std::to_string(o.g.lcg) : std::string())
