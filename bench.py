@@ -360,7 +360,7 @@ def main():
                         "roofline_ms": rl, "roofline_frac": rl / t}
 
     # ---- e2e: public API with pinned HOST buffers (H2D + D2H inside the timed region)
-    e2e = None
+    e2e = e2e16 = None
     if not args.no_e2e:
         hin = {a: inputs[a].cpu().pin_memory() for a in apps}
         hout = {a: torch.empty(BATCH_ROWS[a], nets[a].out_elems).pin_memory() for a in apps}
@@ -382,6 +382,23 @@ def main():
                 "queries_per_s": q * world / (t / 1e3), "ms_per_batch": t,
                 "bytes_per_query": byts / q, "pcie_gbs_achieved": byts / (t / 1e3) / 1e9,
                 "pcie_gbs_needed_at_device_rate": byts / (per_app[a]["ms_per_batch"] / 1e3) / 1e9}
+        # the same step with the inputs sent in the path's 16-bit type (djinn_forward16):
+        # lossless here (inputs are on the path's grid), half the H2D bytes
+        if grid != "fp32":
+            tdt = torch.bfloat16 if grid == "bf16" else torch.float16
+            hin16 = {a: inputs[a].to(tdt).cpu().pin_memory() for a in apps}
+
+            def step_host16():
+                for a in apps:
+                    dj.djinn_forward16(nets[a].handle, hin16[a], BATCH_ROWS[a], hout[a], dj.DJINN_OUT_PROB, sh)
+            for _ in range(2):
+                step_host16()
+            k = max(3, args.steps // 4)
+            t = timed(step_host16, k) / k
+            e2e16 = {"value": sum(BATCH_ROWS[a] / ROWS_PER_QUERY[a] for a in apps) * world / (t / 1e3),
+                     "unit": "queries/s", "ms_per_step": t,
+                     "h2d_bytes_per_step": int(sum(hin16[a].numel() * 2 for a in apps)),
+                     "d2h_bytes_per_step": int(sum(hout[a].numel() * 4 for a in apps))}
         k = max(3, args.steps // 4)
         t = timed(step_host, k) / k
         e2e = {"value": sum(BATCH_ROWS[a] / ROWS_PER_QUERY[a] for a in apps) * world / (t / 1e3), "unit": "queries/s",
@@ -451,7 +468,7 @@ def main():
                            "parallelism": f"replica x{world}, query shards, no per-step collective",
                            "services": "serial (one stream, PDL-chained); see concurrent_services",
                            "host_fed_pipe_chunks": os.environ.get("DJINN_PIPE_CHUNKS", "auto (<=4 by copy size)")},
-                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "concurrent_services": conc, "nlp_token_ids": ids,
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "e2e_16bit_inputs": e2e16, "concurrent_services": conc, "nlp_token_ids": ids,
                 "gpu_launches": int(launches),
                 "clocks": clk.summary(), "per_app": per_app,
                 "top_ops": [{k: o[k] for k in ("app", "op", "kind", "ms_total", "avg_us", "tflops", "gbs", "bound",

@@ -137,6 +137,20 @@ DJINN_API int djinn_load_net(const char* desc, size_t desc_len, const float* wei
 DJINN_API int djinn_forward(djinn_net* net, const float* input, int64_t rows, int in_mem,
                   void* output, int out_mem, int out_mode, void* stream);
 
+/*
+ * djinn_forward16 -- djinn_forward with the input rows already in the net's 16-bit
+ * storage type (bf16 for a DJINN_BF16 net, fp16 for DJINN_FP16): the values the first
+ * kernel would round fp32 inputs to, so results are bit-identical to djinn_forward on the
+ * widened rows, while a host-fed query moves half the bytes over PCIe (the bottleneck
+ * the paper measured for its services, L231-253).
+ *   input : uint16 [rows, in_elems_per_row], same row order as djinn_forward; host or
+ *           device (in_mem).  Other arguments, asynchrony and threading as djinn_forward.
+ * Errors: DJINN_E_UNSUPPORTED on a DJINN_FP32 net.  (Inputs that are not 16-bit floats,
+ * e.g. the Embedding layer's token indices, go through djinn_forward.)
+ */
+DJINN_API int djinn_forward16(djinn_net* net, const void* input, int64_t rows, int in_mem,
+                  void* output, int out_mem, int out_mode, void* stream);
+
 /* djinn_sync -- synchronise `stream` and surface asynchronous CUDA errors as
  * DJINN_E_CUDA. */
 DJINN_API int djinn_sync(djinn_net* net, void* stream);

@@ -25,7 +25,7 @@ DJINN_FP32, DJINN_BF16, DJINN_FP16 = 0, 1, 2
 DJINN_MEM_HOST, DJINN_MEM_DEVICE = 0, 1
 DJINN_OUT_PROB, DJINN_OUT_ARGMAX, DJINN_OUT_LOGITS = 0, 1, 2
 PRECISION = {"fp32": DJINN_FP32, "bf16": DJINN_BF16, "fp16": DJINN_FP16}
-EXPORTS = ["djinn_load_net", "djinn_forward", "djinn_sync", "djinn_free", "djinn_net_info",
+EXPORTS = ["djinn_load_net", "djinn_forward", "djinn_forward16", "djinn_sync", "djinn_free", "djinn_net_info",
            "djinn_weight_arena", "djinn_plan_info", "djinn_profile", "djinn_profile_read", "djinn_op_info",
            "djinn_describe", "djinn_last_error", "djinn_kernel_launches"]
 OP_KINDS = ["pack", "gemm", "lrn", "pool", "softmax", "lrn+pool"]
@@ -50,6 +50,7 @@ def lib() -> ctypes.CDLL:
         P, I, I64, SZ = ctypes.c_void_p, ctypes.c_int, ctypes.c_int64, ctypes.c_size_t
         L.djinn_load_net.argtypes = [ctypes.c_char_p, SZ, P, SZ, I, I, I, I64, ctypes.POINTER(P)]
         L.djinn_forward.argtypes = [P, P, I64, I, P, I, I, P]
+        L.djinn_forward16.argtypes = [P, P, I64, I, P, I, I, P]
         L.djinn_sync.argtypes = [P, P]
         L.djinn_free.argtypes = [P]
         L.djinn_net_info.argtypes = [P] + [ctypes.POINTER(I64)] * 4
@@ -104,6 +105,14 @@ def djinn_forward(net: int, inp, rows: int, out, out_mode: int, stream: Optional
     ip, imem = _ptr_mem(inp)
     op, omem = _ptr_mem(out)
     _check(lib().djinn_forward(net, ip, rows, imem, op, omem, out_mode, stream))
+
+
+def djinn_forward16(net: int, inp, rows: int, out, out_mode: int, stream: Optional[int] = None) -> None:
+    """Mirror of djinn_forward16: ``inp`` holds the rows in the net's 16-bit type (a torch
+    bfloat16 / float16 tensor or a numpy uint16 array of the raw bits)."""
+    ip, imem = _ptr_mem(inp)
+    op, omem = _ptr_mem(out)
+    _check(lib().djinn_forward16(net, ip, rows, imem, op, omem, out_mode, stream))
 
 
 def djinn_sync(net: int, stream: Optional[int] = None) -> None:

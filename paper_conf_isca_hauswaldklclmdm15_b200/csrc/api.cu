@@ -117,6 +117,23 @@ int djinn_forward(djinn_net* net, const float* input, int64_t rows, int in_mem, 
   });
 }
 
+int djinn_forward16(djinn_net* net, const void* input, int64_t rows, int in_mem, void* output, int out_mem,
+                    int out_mode, void* stream) {
+  return guarded([&]() -> int {
+    if (!net) return fail(DJINN_E_INVAL, "net is NULL");
+    if (rows < 0) return fail(DJINN_E_INVAL, "rows < 0");
+    if (net->impl.dt == djinn::DT_F32) return fail(DJINN_E_UNSUPPORTED, "16-bit input on an fp32 net");
+    if (rows == 0) return DJINN_OK;
+    if (!input || !output) return fail(DJINN_E_INVAL, "input/output is NULL");
+    if (in_mem != DJINN_MEM_HOST && in_mem != DJINN_MEM_DEVICE) return fail(DJINN_E_INVAL, "bad in_mem");
+    if (out_mem != DJINN_MEM_HOST && out_mem != DJINN_MEM_DEVICE) return fail(DJINN_E_INVAL, "bad out_mem");
+    if (out_mode < DJINN_OUT_PROB || out_mode > DJINN_OUT_LOGITS) return fail(DJINN_E_INVAL, "bad out_mode");
+    DeviceGuard dg(net->impl.device);
+    net->impl.forward((const float*)input, rows, in_mem, output, out_mem, out_mode, (cudaStream_t)stream, true);
+    return DJINN_OK;
+  });
+}
+
 int djinn_sync(djinn_net* net, void* stream) {
   return guarded([&]() -> int {
     if (!net) return fail(DJINN_E_INVAL, "net is NULL");

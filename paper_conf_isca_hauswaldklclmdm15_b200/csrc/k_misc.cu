@@ -207,6 +207,34 @@ cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int 
 }
 
 // ------------------------------------------------------------------------------------------
+// djinn_forward16: widen 16-bit input rows to fp32 (exact), 8 elements per thread when aligned.
+template <typename T>
+__global__ void widen16_kernel(const T* __restrict__ x, float* __restrict__ y, int64_t n) {
+  pdl_trigger();
+  pdl_wait();
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t n8 = ((reinterpret_cast<uintptr_t>(x) & 15) == 0) ? n / 8 : 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n8; i += stride) {
+    const uint4 v = __ldg(reinterpret_cast<const uint4*>(x) + i);
+    const T* h = reinterpret_cast<const T*>(&v);
+    float4 a, b;
+    a.x = ld(h + 0); a.y = ld(h + 1); a.z = ld(h + 2); a.w = ld(h + 3);
+    b.x = ld(h + 4); b.y = ld(h + 5); b.z = ld(h + 6); b.w = ld(h + 7);
+    reinterpret_cast<float4*>(y)[2 * i] = a;
+    reinterpret_cast<float4*>(y)[2 * i + 1] = b;
+  }
+  for (int64_t i = n8 * 8 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += stride) y[i] = ld(x + i);
+}
+
+cudaError_t launch_widen16(const void* x, float* y, int64_t n, int dt, cudaStream_t st) {
+  const int T = 256;
+  const int g = min(nblocks((n + 7) / 8, T), 148 * 16);
+  if (dt == DT_F16) launch_pdl(widen16_kernel<__half>, dim3(g), dim3(T), 0, st, (const __half*)x, y, n);
+  else launch_pdl(widen16_kernel<__nv_bfloat16>, dim3(g), dim3(T), 0, st, (const __nv_bfloat16*)x, y, n);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------
 // SENNA window lookup (kernels.h launch_embed).  One thread per output column: consecutive
 // threads copy consecutive elements of one table row, so each (word, table) lookup is one
 // coalesced read of dim[t] elements; the row's indices are L1-resident broadcasts.

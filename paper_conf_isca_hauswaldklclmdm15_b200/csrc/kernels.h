@@ -114,6 +114,9 @@ struct GemmGeom {
 cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f, int xs,
                               int Ho, int Wo, int Cp, int dt, cudaStream_t st);
 
+// --- djinn_forward16: 16-bit input rows (the path's type dt) -> fp32, exact ----------------
+cudaError_t launch_widen16(const void* x, float* y, int64_t n, int dt, cudaStream_t st);
+
 // --- SENNA window lookup (K0 variant) ------------------------------------
 // x: float32 [rows][window * T] feature indices, word-major (x[r][w*T + t]);
 // tables: the path's type, table t = [vocab[t]][dim[t]] at element offset toff[t];

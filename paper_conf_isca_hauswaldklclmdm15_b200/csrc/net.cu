@@ -1000,6 +1000,7 @@ void Net::load_weights(const float* w, size_t n, int mem) {
 Workspace::~Workspace() {
   for (void* p : buf) if (p) cudaFree(p);
   if (in_stage) cudaFree(in_stage);
+  if (in_stage16) cudaFree(in_stage16);
   if (out_stage) cudaFree(out_stage);
   for (int s = 0; s < 2; ++s)
     for (cudaEvent_t e : {in_ready[s], in_free[s], out_ready[s], out_free[s]})
@@ -1102,12 +1103,16 @@ static int pipe_chunks(size_t io_bytes) {
   return io_bytes >= (32u << 20) ? 2 : 1;   // measured on B200 (bench e2e): 2 >= 4 > 1
 }
 
-void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_mem, int mode, cudaStream_t st) {
+void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_mem, int mode, cudaStream_t st,
+                  bool in16) {
   if (poisoned) throw Error(DJINN_E_CUDA, "net is poisoned by an earlier CUDA error");
   Workspace* w = workspace(st);
   const bool hin = in_mem == DJINN_MEM_HOST, hout = out_mem == DJINN_MEM_HOST;
-  if (hin && !w->in_stage)
+  if ((hin || in16) && !w->in_stage)
     if (cudaMalloc(&w->in_stage, (size_t)max_rows * in_elems * 4) != cudaSuccess) throw Error(DJINN_E_NOMEM, "input staging");
+  if (hin && in16 && !w->in_stage16)
+    if (cudaMalloc(&w->in_stage16, (size_t)max_rows * in_elems * 2) != cudaSuccess) throw Error(DJINN_E_NOMEM, "input staging");
+  const size_t in_row_bytes = (size_t)in_elems * (in16 ? 2 : 4);
   if (hout && !w->out_stage)
     if (cudaMalloc(&w->out_stage, (size_t)max_rows * out_elems * 4) != cudaSuccess) throw Error(DJINN_E_NOMEM, "output staging");
   if ((hin || hout) && !w->cin) {
@@ -1124,7 +1129,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
   int slots = 1;
   if (hin || hout) {
     const int64_t nr = std::min<int64_t>(rows, max_rows);
-    const size_t io = (size_t)nr * ((hin ? in_elems * 4 : 0) + (hout ? out_row_bytes : 0));
+    const size_t io = (size_t)nr * ((hin ? in_row_bytes : 0) + (hout ? out_row_bytes : 0));
     const int P = pipe_chunks(io);
     cs = std::max<int64_t>(1, (nr + P - 1) / P);
     slots = 2 * cs <= max_rows ? 2 : 1;
@@ -1143,15 +1148,27 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
   for (int64_t r0 = 0, c = 0; r0 < rows; r0 += cs, ++c) {
     const int64_t n = std::min<int64_t>(cs, rows - r0);
     const int sl = (int)(c % slots);
-    const float* src = in + r0 * in_elems;
+    const float* src = in16 ? (const float*)((const uint16_t*)in + r0 * in_elems) : in + r0 * in_elems;
     if (hin) {
       // H2D into slot `sl` once the kernels of its previous chunk have consumed it
-      float* stage = w->in_stage + (size_t)sl * cs * in_elems;
+      void* stage = in16 ? (void*)(w->in_stage16 + (size_t)sl * cs * in_elems) : (void*)(w->in_stage + (size_t)sl * cs * in_elems);
       ck(cudaStreamWaitEvent(w->cin, w->in_free[sl], 0), "event wait");
-      ck(cudaMemcpyAsync(stage, src, (size_t)n * in_elems * 4, cudaMemcpyHostToDevice, w->cin), "input H2D");
+      ck(cudaMemcpyAsync(stage, src, (size_t)n * in_row_bytes, cudaMemcpyHostToDevice, w->cin), "input H2D");
       ck(cudaEventRecord(w->in_ready[sl], w->cin), "event record");
       ck(cudaStreamWaitEvent(st, w->in_ready[sl], 0), "event wait");
-      src = stage;
+      src = (const float*)stage;
+    }
+    if (in16) {
+      // 16-bit rows -> fp32 (exact) in the fp32 staging buffer; the pack then runs unchanged
+      float* wide = w->in_stage + (size_t)(hin ? sl * cs : 0) * in_elems;
+      cudaError_t e = launch_widen16(src, wide, n * in_elems, dt, st);
+      ++launch_counter();
+      if (e != cudaSuccess) {
+        poisoned = true;
+        throw Error(DJINN_E_CUDA, std::string("widen16: ") + cudaGetErrorString(e));
+      }
+      if (hin) ck(cudaEventRecord(w->in_free[sl], st), "event record");  // the 16-bit slot is consumed
+      src = wide;
     }
     if (hout) ck(cudaStreamWaitEvent(st, w->out_free[sl], 0), "event wait");  // slot's previous D2H done
     uint8_t* dst = hout ? (uint8_t*)w->out_stage + (size_t)sl * cs * out_row_bytes : (uint8_t*)out + r0 * out_row_bytes;
@@ -1221,7 +1238,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
         throw Error(DJINN_E_CUDA, o.name + ": " + cudaGetErrorString(e));
       }
       if (profile && pop == (int)i) ck(cudaEventRecord(prof_events[pbase + 1], st), "profile event");
-      if (i == 0 && hin) ck(cudaEventRecord(w->in_free[sl], st), "event record");  // pack has read the slot
+      if (i == 0 && hin && !in16) ck(cudaEventRecord(w->in_free[sl], st), "event record");  // pack has read the slot
     }
     if (profile && pop < 0) ck(cudaEventRecord(prof_events[pbase + ops.size()], st), "profile event");
     if (hout) {

@@ -98,6 +98,7 @@ struct ProfRec {  // one timed forward chunk: events[first .. first + n_ops]
 struct Workspace {
   std::vector<void*> buf;  // 0/1 ping-pong, 2 logits, 3.. dedicated bordered tensors (borders stay zero)
   float* in_stage = nullptr;
+  uint16_t* in_stage16 = nullptr;  // djinn_forward16 host rows (two slots like in_stage)
   void* out_stage = nullptr;
   // host-fed mode: H2D on `cin`, D2H on `cout`, compute on the caller's stream; two staging
   // slots, each with a "filled" and a "drained" event (Net::forward)
@@ -140,7 +141,7 @@ struct Net {
   void load_weights(const float* w, size_t n, int mem);         // pack into the arena
   Workspace* workspace(cudaStream_t st);
   void forward(const float* in, int64_t rows, int in_mem, void* out, int out_mem, int mode,
-               cudaStream_t st);
+               cudaStream_t st, bool in16 = false);
   std::string plan_string() const;
 };
 

@@ -207,3 +207,38 @@ def test_token_id_invalid_indices_select_zero_vectors():
     lg = run_gpu(app, prec, x)
     r = compare_16bit(lg, lg_ref)
     assert r["rel_max"] <= REL_LOGIT_TOL, r
+
+
+# ---------------------------------------------------------------- 16-bit wire inputs
+# (token-id nets are not listed: indices up to 130000 are not 16-bit floats; they use djinn_forward)
+@pytest.mark.parametrize("app,prec", [("imc", "bf16"), ("dig", "fp16"), ("asr", "bf16"), ("ner", "fp16")])
+@pytest.mark.parametrize("in_host", [True, False])
+def test_forward16_equals_fp32_input_bitwise(app, prec, in_host, monkeypatch):
+    """djinn_forward16 on the rows' 16-bit images == djinn_forward on the fp32 rows (they
+    are on the path's grid, so the first kernel's rounding is the identity), with host
+    rows pipelined over 1 / 2 / 3 chunks."""
+    n = {"imc": 5, "dig": 250, "asr": 300, "ner": 500}[app]
+    x = recipes.gen_input_rows(app, 0, n, prec)
+    tdt = torch.bfloat16 if prec == "bf16" else torch.float16
+    x16 = torch.from_numpy(x).to(tdt)
+    assert torch.equal(x16.float(), torch.from_numpy(x))
+    net = dj.DjinnNet(dj.net_description(app), blob(app, prec), prec, n)
+    ref = net.forward(torch.from_numpy(x).cuda(), dj.DJINN_OUT_LOGITS).cpu()
+    s = torch.cuda.Stream()
+    for chunks in (1, 2, 3):
+        monkeypatch.setenv("DJINN_PIPE_CHUNKS", str(chunks))
+        inp = x16.pin_memory() if in_host else x16.cuda()
+        out = torch.empty(n, net.out_elems).pin_memory()
+        dj.djinn_forward16(net.handle, inp, n, out, dj.DJINN_OUT_LOGITS, s.cuda_stream)
+        dj.djinn_sync(net.handle, s.cuda_stream)
+        assert torch.equal(out, ref), chunks
+    net.close()
+
+
+def test_forward16_rejected_on_fp32_net():
+    net = dj.DjinnNet(dj.net_description("pos"), blob("pos", "fp32"), "fp32", 8)
+    with pytest.raises(dj.DjinnError) as e:
+        dj.djinn_forward16(net.handle, torch.zeros(8, 300, dtype=torch.bfloat16, device="cuda"), 8,
+                           torch.empty(8, 45, device="cuda"), dj.DJINN_OUT_PROB)
+    assert e.value.code == dj.DJINN_E_UNSUPPORTED
+    net.close()
