@@ -882,6 +882,15 @@ void Net::choose_tiles() {
     g.M = (int)(max_rows * o.ohw);
     o.bn = tc_pick_bn(g);
     o.g.cg = tc_pick_cg(g, o.bn);
+    {
+      // experiment hook: cap the tile width of dense GEMMs (DJINN_DENSE_BN=64/128)
+      const char* e = getenv("DJINN_DENSE_BN");
+      const int cap = e ? atoi(e) : 0;
+      if (g.mode == GM_DENSE && cap >= 16 && o.bn > cap) {
+        o.bn = cap;
+        o.g.cg = tc_pick_cg(g, o.bn);
+      }
+    }
     if (o.g.slab && !tc_slab_config(o.g, o.bn)) {
       o.g.slab = 0;
       o.ohw = o.g.OH * o.g.OWb;
