@@ -4,6 +4,7 @@
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
 #include <float.h>
+#include <stdlib.h>
 
 #include <algorithm>
 
@@ -131,34 +132,55 @@ __global__ void pack_xform_kernel(const float* __restrict__ x, T* __restrict__ y
 template <typename T, int MODE, int C, int F, int CP, int XS>
 __global__ void pack_xform_fixed_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int H, int W,
                                         int Ho, int Wo) {
+  // Stores are staged per warp in shared memory: a thread's pixel is CP*2 contiguous bytes, so
+  // direct 16-byte stores from 32 lanes would touch 32 separate lines per instruction; after
+  // the (XOR-swizzled, bank-conflict-free) staging each store instruction writes 512
+  // consecutive bytes of the warp's 32 consecutive output pixels.
+  constexpr int CPC = CP / 8;  // 16-byte chunks per pixel (power of two)
+  __shared__ uint4 stage[4][32 * CPC];
   pdl_trigger();
   pdl_wait();
   const int per_row = Ho * Wo;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  uint4* st = stage[wid];
   for (int64_t r = blockIdx.y; r < rows; r += gridDim.y) {
     const float* src = x + r * C * (int64_t)H * W;
-    for (int pix = blockIdx.x * blockDim.x + threadIdx.x; pix < per_row; pix += gridDim.x * blockDim.x) {
-      const int yo = pix / Wo, xo = pix - (pix / Wo) * Wo;
-      T* dst = y + (r * per_row + pix) * (int64_t)CP;
-      const int y0 = MODE == 1 ? yo * F : yo, x0 = MODE == 1 ? xo * F : xo * XS;
-      const float* p0 = src + (int64_t)y0 * W + x0;
+    uint4* dst_row = reinterpret_cast<uint4*>(y + r * per_row * (int64_t)CP);
+    for (int base = blockIdx.x * blockDim.x + wid * 32; base < per_row; base += gridDim.x * blockDim.x) {
+      const int pix = base + lane;
+      if (pix < per_row) {
+        const int yo = pix / Wo, xo = pix - (pix / Wo) * Wo;
+        const int y0 = MODE == 1 ? yo * F : yo, x0 = MODE == 1 ? xo * F : xo * XS;
+        const float* p0 = src + (int64_t)y0 * W + x0;
 #pragma unroll
-      for (int ch = 0; ch < CP; ch += 8) {
-        __align__(16) T v[8];
+        for (int ch = 0; ch < CP; ch += 8) {
+          __align__(16) T v[8];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          const int cc = ch + j;
-          float val = 0.f;
-          if (MODE == 1) {
-            const int d = cc / C, c = cc % C, dy = d / F, dx = d % F;
-            if (d < F * F && y0 + dy < H && x0 + dx < W) val = __ldg(p0 + ((int64_t)c * H + dy) * W + dx);
-          } else {
-            const int kx = cc / C, c = cc % C;
-            if (kx < F && x0 + kx < W) val = __ldg(p0 + (int64_t)c * H * W + kx);
+          for (int j = 0; j < 8; ++j) {
+            const int cc = ch + j;
+            float val = 0.f;
+            if (MODE == 1) {
+              const int d = cc / C, c = cc % C, dy = d / F, dx = d % F;
+              if (d < F * F && y0 + dy < H && x0 + dx < W) val = __ldg(p0 + ((int64_t)c * H + dy) * W + dx);
+            } else {
+              const int kx = cc / C, c = cc % C;
+              if (kx < F && x0 + kx < W) val = __ldg(p0 + (int64_t)c * H * W + kx);
+            }
+            v[j] = cvt<T>(val);
           }
-          v[j] = cvt<T>(val);
+          st[lane * CPC + ((ch / 8) ^ (lane & (CPC - 1)))] = *reinterpret_cast<const uint4*>(v);
         }
-        *reinterpret_cast<uint4*>(dst + ch) = *reinterpret_cast<const uint4*>(v);
       }
+      __syncwarp();
+      const int nv = min(32, per_row - base) * CPC;
+      uint4* dst = dst_row + (int64_t)base * CPC;
+#pragma unroll
+      for (int i = 0; i < CPC; ++i) {
+        const int e = i * 32 + lane;
+        const int p = e / CPC, k = e % CPC;
+        if (e < nv) dst[e] = st[p * CPC + (k ^ (p & (CPC - 1)))];
+      }
+      __syncwarp();
     }
   }
 }
@@ -715,6 +737,66 @@ __global__ void pool_max_remap_kernel(const T* __restrict__ x, T* __restrict__ y
   }
 }
 
+// 3x3 / stride-2 / pad-0 MAX pooling (IMC pool1/pool2/pool5, FACE M2) with the same layout change
+// as pool_max_remap_kernel, but each thread walks a band of R output rows of one column: the
+// horizontal max of an input row is computed once and the row shared by output rows oy and oy+1
+// (input row 2oy+2) is carried over, so each output row costs 6 loads instead of 9.  Windows
+// clip to the image (Caffe ceil geometry); clipped taps re-read the last row/column (exact).
+template <typename T, int R>
+__global__ void pool_max_k3s2_band_kernel(const T* __restrict__ x, T* __restrict__ y, int C, int Cpi, int gsz_i,
+                                          int gpitch_i, int H, int W, int OH, int OW, int Cpo, int gsz_o,
+                                          int gpitch_o, int xu, int obd, int xblocks) {
+  pdl_trigger();
+  pdl_wait();
+  __shared__ int in_off[64];
+  const int P = Cpo / xu, chunks = P / 8;
+  if (threadIdx.y == 0 && threadIdx.x < chunks) {
+    const int pos = threadIdx.x * 8, grp = pos / gpitch_o, within = pos - grp * gpitch_o, c0 = grp * gsz_o + within;
+    in_off[threadIdx.x] = (within < gsz_o && c0 < C) ? (c0 / gsz_i) * gpitch_i + c0 % gsz_i : -1;
+  }
+  __syncthreads();
+  const int band = blockIdx.x / xblocks, xb = blockIdx.x - band * xblocks;
+  const int ox = xb * blockDim.y + threadIdx.y;
+  if (ox >= OW) return;
+  const int oy0 = band * R, oy1 = min(oy0 + R, OH);
+  const int64_t r = blockIdx.y;
+  const int off = in_off[threadIdx.x];
+  const int64_t orow = (int64_t)(OW + 2 * obd) * Cpo;
+  T* yo = y + ((r * (OH + 2 * obd) + oy0 + obd) * (OW + 2 * obd) + ox + obd) * (int64_t)Cpo + threadIdx.x * 8;
+  if (off < 0) {
+    for (int oy = oy0; oy < oy1; ++oy, yo += orow) {
+      *reinterpret_cast<uint4*>(yo) = make_uint4(0, 0, 0, 0);
+      for (int sl = 1; sl < xu; ++sl) {
+        if (ox - sl >= 0) *reinterpret_cast<uint4*>(yo - (int64_t)sl * Cpo + sl * P) = make_uint4(0, 0, 0, 0);
+        if (ox + sl >= OW) *reinterpret_cast<uint4*>(yo + sl * P) = make_uint4(0, 0, 0, 0);
+      }
+    }
+    return;
+  }
+  const T* base = x + r * (int64_t)H * W * Cpi + off;
+  const int ws = ox * 2, w1 = min(ws + 1, W - 1), w2 = min(ws + 2, W - 1);
+  auto hrow = [&](int h) {
+    const T* p = base + (int64_t)h * W * Cpi;
+    const uint4 a = __ldg(reinterpret_cast<const uint4*>(p + (int64_t)ws * Cpi));
+    const uint4 b = __ldg(reinterpret_cast<const uint4*>(p + (int64_t)w1 * Cpi));
+    const uint4 c = __ldg(reinterpret_cast<const uint4*>(p + (int64_t)w2 * Cpi));
+    return max8(max8(a, b, T()), c, T());
+  };
+  uint4 prev = hrow(2 * oy0);
+  for (int oy = oy0; oy < oy1; ++oy, yo += orow) {
+    const int hs = 2 * oy;
+    const uint4 m1 = hrow(min(hs + 1, H - 1));
+    const uint4 m2 = hrow(min(hs + 2, H - 1));
+    const uint4 ov = max8(max8(prev, m1, T()), m2, T());
+    prev = m2;
+    *reinterpret_cast<uint4*>(yo) = ov;
+    for (int sl = 1; sl < xu; ++sl) {
+      if (ox - sl >= 0) *reinterpret_cast<uint4*>(yo - (int64_t)sl * Cpo + sl * P) = ov;
+      if (ox + sl >= OW) *reinterpret_cast<uint4*>(yo + sl * P) = make_uint4(0, 0, 0, 0);
+    }
+  }
+}
+
 cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int Cpi, int gsz_i, int gpitch_i, int H,
                               int W, int OH, int OW, int kernel, int stride, int pad, int Cpo, int gsz_o, int gpitch_o,
                               int xu, int obd, int dt, cudaStream_t st) {
@@ -729,6 +811,28 @@ cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int C
     return cudaErrorInvalidValue;
   const int chunks = Cpo / xu / 8;
   if (chunks > 64) return cudaErrorInvalidValue;
+  static const bool band_on = [] {
+    const char* e = getenv("DJINN_POOL_BAND");
+    return !e || atoi(e) != 0;
+  }();
+  if (band_on && kernel == 3 && stride == 2 && pad == 0) {
+    constexpr int R = 4;
+    const int xblocks = (OW + 256 / chunks - 1) / (256 / chunks);
+    const int bpix = (OW + xblocks - 1) / xblocks;  // balanced column blocks
+    const int bands = (OH + R - 1) / R;
+    for (int64_t r0 = 0; r0 < rows; r0 += 65535) {
+      const int64_t nr = rows - r0 < 65535 ? rows - r0 : 65535;
+      dim3 blk(chunks, bpix), g(xblocks * bands, (unsigned)nr);
+      const size_t xo = (size_t)r0 * H * W * Cpi, yo = (size_t)r0 * (OH + 2 * obd) * (OW + 2 * obd) * Cpo;
+      if (dt == DT_F16)
+        launch_pdl(pool_max_k3s2_band_kernel<__half, R>, dim3(g), dim3(blk), 0, st, (const __half*)x + xo, (__half*)y + yo,
+                   C, Cpi, gsz_i, gpitch_i, H, W, OH, OW, Cpo, gsz_o, gpitch_o, xu, obd, xblocks);
+      else
+        launch_pdl(pool_max_k3s2_band_kernel<__nv_bfloat16, R>, dim3(g), dim3(blk), 0, st, (const __nv_bfloat16*)x + xo,
+                   (__nv_bfloat16*)y + yo, C, Cpi, gsz_i, gpitch_i, H, W, OH, OW, Cpo, gsz_o, gpitch_o, xu, obd, xblocks);
+    }
+    return cudaGetLastError();
+  }
   const int pix = 256 / chunks;
   for (int64_t r0 = 0; r0 < rows; r0 += 65535) {  // grid.z <= 65535 images per launch
     const int64_t nr = rows - r0 < 65535 ? rows - r0 : 65535;
