@@ -311,6 +311,23 @@ __device__ __forceinline__ float lg2_ftz(float x) {
   asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
   return r;
 }
+#ifdef DJINN_LRN_POLY
+// 2^y on the FMA pipe (see k_misc.cu exp2_fma): relative error <= 4.2e-5, half of the LRN's
+// transcendental work moved off the MUFU.
+__device__ __forceinline__ float ex2_lrn(float y) {
+  y = fmaxf(y, -126.f);
+  const float t = y + 12582912.f;
+  const float n = t - 12582912.f;
+  const float f = y - n;
+  float p = fmaf(0.0096181291f, f, 0.0555041087f);
+  p = fmaf(p, f, 0.2402265070f);
+  p = fmaf(p, f, 0.6931471806f);
+  p = fmaf(p, f, 1.0f);
+  return __int_as_float(__float_as_int(p) + ((__float_as_int(t) - 0x4B400000) << 23));
+}
+#else
+__device__ __forceinline__ float ex2_lrn(float y) { return ex2_ftz(y); }
+#endif
 __device__ __forceinline__ float rcp_ftz(float x) {
   float r;
   asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
@@ -332,20 +349,29 @@ __device__ __forceinline__ float act_fast(float v, int act) {
 // Bias + activation on a 16-vector: the switch is resolved once per vector, the loops are
 // branch-free (the per-element runtime switch cost ~17% of issue slots in branch resolution).
 __device__ __forceinline__ void bias_act16(float (&v)[16], const uint32_t (&r)[16], const float (&b)[16], int act) {
+  // bias add and the sigmoid's scalings on the packed fp32 pipe (FADD2/FMUL2, bitwise equal)
 #pragma unroll
-  for (int j = 0; j < 16; ++j) v[j] = __uint_as_float(r[j]) + b[j];
+  for (int j = 0; j < 16; j += 2) {
+    const float2 s = add2(make_float2(__uint_as_float(r[j]), __uint_as_float(r[j + 1])), make_float2(b[j], b[j + 1]));
+    v[j] = s.x;
+    v[j + 1] = s.y;
+  }
   switch (act) {
     case ACT_RELU:
 #pragma unroll
       for (int j = 0; j < 16; ++j) v[j] = fmaxf(v[j], 0.f);
       break;
     case ACT_SIGMOID:
-#pragma unroll
-      for (int j = 0; j < 16; ++j) v[j] = sigmoid_fast(v[j]);
-      break;
     case ACT_SIGMOID_C:
 #pragma unroll
-      for (int j = 0; j < 16; ++j) v[j] = sigmoid_fast(v[j]) - 0.5f;
+      for (int j = 0; j < 16; j += 2) {
+        const float2 e = mul2(make_float2(v[j], v[j + 1]), make_float2(-1.4426950408889634f, -1.4426950408889634f));
+        const float2 d = add2(make_float2(ex2_ftz(e.x), ex2_ftz(e.y)), make_float2(1.f, 1.f));
+        float2 o = make_float2(rcp_ftz(d.x), rcp_ftz(d.y));
+        if (act == ACT_SIGMOID_C) o = add2(o, make_float2(-0.5f, -0.5f));
+        v[j] = o.x;
+        v[j + 1] = o.y;
+      }
       break;
     case ACT_TANH:
 #pragma unroll
@@ -1068,24 +1094,44 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 #pragma unroll
             for (int j = 0; j < 16; ++j) nxt[j] = 0.f;
           }
+          // Channel pairs on the packed fp32 pipe (FMUL2/FADD2/FFMA2), same operation order as
+          // the scalar form s5 = (sq[j]+sq[j+1]) + (sq[j+2]+sq[j+3]) + sq[j+4]: bitwise equal.
           float sq[20];
           sq[0] = pm2;
           sq[1] = pm1;
 #pragma unroll
-          for (int j = 0; j < 16; ++j) sq[2 + j] = cur[j] * cur[j];
-          sq[18] = nxt[0] * nxt[0];
-          sq[19] = nxt[1] * nxt[1];
+          for (int j = 0; j < 8; ++j) {
+            const float2 c2 = make_float2(cur[2 * j], cur[2 * j + 1]);
+            const float2 s2 = mul2(c2, c2);
+            sq[2 + 2 * j] = s2.x;
+            sq[3 + 2 * j] = s2.y;
+          }
+          {
+            const float2 n2 = make_float2(nxt[0], nxt[1]);
+            const float2 s2 = mul2(n2, n2);
+            sq[18] = s2.x;
+            sq[19] = s2.y;
+          }
+          float q[18];  // q[j] = sq[j] + sq[j+1]
+#pragma unroll
+          for (int j = 0; j < 18; ++j) q[j] = sq[j] + sq[j + 1];
+          const float2 ka2 = make_float2(ka, ka), kk2 = make_float2(kk, kk), nb2 = make_float2(nb, nb);
           float o[16];
 #pragma unroll
-          for (int j = 0; j < 16; ++j) {
-            const float s5 = (sq[j] + sq[j + 1]) + (sq[j + 2] + sq[j + 3]) + sq[j + 4];  // window c-2 .. c+2
+          for (int j = 0; j < 16; j += 2) {
+            const float2 s5 = add2(add2(make_float2(q[j], q[j + 1]), make_float2(q[j + 2], q[j + 3])),
+                                   make_float2(sq[j + 4], sq[j + 5]));  // windows c-2 .. c+2
+            const float2 c2 = make_float2(cur[j], cur[j + 1]);
 #if defined(DJINN_DBG_LRN0)
-            o[j] = cur[j] * fmaf(ka, s5, kk);  // diagnostic: no MUFU
-#elif defined(DJINN_DBG_LRN1)
-            o[j] = cur[j] * rsqrtf(fmaf(ka, s5, kk));  // diagnostic: one MUFU
+            const float2 r = fma2(ka2, s5, kk2);  // diagnostic: no MUFU
 #else
-            o[j] = cur[j] * ex2_ftz(nb * lg2_ftz(fmaf(ka, s5, kk)));
+            const float2 t = fma2(ka2, s5, kk2);
+            const float2 l = mul2(nb2, make_float2(lg2_ftz(t.x), lg2_ftz(t.y)));
+            const float2 r = make_float2(ex2_lrn(l.x), ex2_lrn(l.y));
 #endif
+            const float2 ov = mul2(c2, r);
+            o[j] = ov.x;
+            o[j + 1] = ov.y;
           }
           pm2 = sq[16];
           pm1 = sq[17];
