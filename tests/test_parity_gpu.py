@@ -242,3 +242,38 @@ def test_forward16_rejected_on_fp32_net():
                            torch.empty(8, 45, device="cuda"), dj.DJINN_OUT_PROB)
     assert e.value.code == dj.DJINN_E_UNSUPPORTED
     net.close()
+
+
+# ---------------------------------------------------------------- pooling kernel variants
+_POOL_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+sys.path.insert(0, sys.argv[1] + "/tests")
+import paper_conf_isca_hauswaldklclmdm15_b200 as dj
+from datagen import recipes
+from parity import blob
+app, prec, n = sys.argv[2], sys.argv[3], int(sys.argv[4])
+x = recipes.gen_input_rows(app, 0, n, prec)
+net = dj.DjinnNet(dj.net_description(app), blob(app, prec), prec, n)
+np.save(sys.argv[5], net.forward(torch.from_numpy(x).cuda(), dj.DJINN_OUT_LOGITS).cpu().numpy())
+net.close()
+"""
+
+
+@pytest.mark.parametrize("app,prec,n", [("imc", "bf16", 7), ("face", "fp16", 5)])
+def test_band_pool_equals_per_pixel_pool_bitwise(app, prec, n, tmp_path):
+    """The 3x3/stride-2 band max pool (IMC pool1/pool5, FACE M2 with its clipped ceil-geometry
+    last window; 27/71/6 output rows are not multiples of the 4-row band) and the per-pixel
+    pool kernel (DJINN_POOL_BAND=0) give bitwise-equal logits: a max reorders nothing."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    outs = []
+    for band in ("1", "0"):
+        f = str(tmp_path / f"lg{band}.npy")
+        env = dict(os.environ, DJINN_POOL_BAND=band)
+        subprocess.run([sys.executable, "-c", _POOL_CHILD, root, app, prec, str(n), f], env=env, check=True,
+                       timeout=600)
+        outs.append(np.load(f))
+    assert np.array_equal(outs[0], outs[1])
