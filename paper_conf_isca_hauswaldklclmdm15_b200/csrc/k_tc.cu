@@ -424,6 +424,21 @@ constexpr bool kDbgNoMma = true;  // DJINN_DBG_NOMMA: operands stream, no MMA is
 constexpr bool kDbgNoMma = false;
 #endif
 
+// 16-byte epilogue store; DJINN_ST_HINT selects the cache policy (experiment hook:
+// 0 plain st.global, 1 .L1::no_allocate, 2 .cs streaming).
+#ifndef DJINN_ST_HINT
+#define DJINN_ST_HINT 0
+#endif
+__device__ __forceinline__ void st16(void* p, uint4 v) {
+#if DJINN_ST_HINT == 1
+  asm volatile("st.global.L1::no_allocate.v4.b32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+               : "memory");
+#elif DJINN_ST_HINT == 2
+  asm volatile("st.global.cs.v4.b32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+#else
+  *reinterpret_cast<uint4*>(p) = v;
+#endif
+}
 template <bool BF16>
 __device__ __forceinline__ void store16(const GemmGeom& g, void* Y, int64_t off, const float (&v)[16], int nvalid8) {
 #ifdef DJINN_DBG_NOSTORE
@@ -449,17 +464,17 @@ __device__ __forceinline__ void store16(const GemmGeom& g, void* Y, int64_t off,
 #pragma unroll
     for (int h = 0; h < 2; ++h)
       if (h < nvalid8)
-        *reinterpret_cast<uint4*>(yp + 8 * h) =
-            make_uint4(pack2<false>(v[8 * h], v[8 * h + 1]), pack2<false>(v[8 * h + 2], v[8 * h + 3]),
-                       pack2<false>(v[8 * h + 4], v[8 * h + 5]), pack2<false>(v[8 * h + 6], v[8 * h + 7]));
+        st16(yp + 8 * h,
+             make_uint4(pack2<false>(v[8 * h], v[8 * h + 1]), pack2<false>(v[8 * h + 2], v[8 * h + 3]),
+                        pack2<false>(v[8 * h + 4], v[8 * h + 5]), pack2<false>(v[8 * h + 6], v[8 * h + 7])));
   } else {
     uint16_t* yp = reinterpret_cast<uint16_t*>(Y) + off;
 #pragma unroll
     for (int h = 0; h < 2; ++h)
       if (h < nvalid8)
-        *reinterpret_cast<uint4*>(yp + 8 * h) =
-            make_uint4(pack2<BF16>(v[8 * h], v[8 * h + 1]), pack2<BF16>(v[8 * h + 2], v[8 * h + 3]),
-                       pack2<BF16>(v[8 * h + 4], v[8 * h + 5]), pack2<BF16>(v[8 * h + 6], v[8 * h + 7]));
+        st16(yp + 8 * h,
+             make_uint4(pack2<BF16>(v[8 * h], v[8 * h + 1]), pack2<BF16>(v[8 * h + 2], v[8 * h + 3]),
+                        pack2<BF16>(v[8 * h + 4], v[8 * h + 5]), pack2<BF16>(v[8 * h + 6], v[8 * h + 7])));
   }
 }
 
