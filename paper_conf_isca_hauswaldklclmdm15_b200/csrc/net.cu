@@ -883,9 +883,21 @@ void Net::choose_tiles() {
     o.bn = tc_pick_bn(g);
     o.g.cg = tc_pick_cg(g, o.bn);
     {
-      // experiment hook: cap the tile width of dense GEMMs (DJINN_DENSE_BN=64/128)
-      const char* e = getenv("DJINN_DENSE_BN");
-      const int cap = e ? atoi(e) : 0;
+      // Dense GEMMs that fill less than one wave of 148 SMs with their default tile get
+      // 64-wide tiles if that makes at most two waves (measured on B200: POS l1 16.4 -> 12.4 us,
+      // DIG ip1 21.2 -> 16.3, IMC fc8 34.8 -> 22.6, FACE F7 49.3 -> 34.9; IMC fc6/fc7 would
+      // become 512 tiles and run 2x slower, so they keep 256-wide pairs; ASR already fills the GPU).
+      // DJINN_DENSE_BN=0 disables the rule, =64/128 forces that cap on every dense GEMM.
+      static const int env_cap = [] {
+        const char* e = getenv("DJINN_DENSE_BN");
+        return e ? atoi(e) : -1;
+      }();
+      int cap = env_cap;
+      if (cap < 0) {
+        const int64_t mt = (g.M + 128LL * o.g.cg - 1) / (128LL * o.g.cg), nt = (g.N + o.bn - 1) / o.bn;
+        const int64_t t64 = ((g.M + 127) / 128) * ((g.N + 63) / 64) * g.Z;  // tiles after the cap (cg = 1)
+        cap = (mt * nt * g.Z < 148 && t64 <= 2 * 148) ? 64 : 0;
+      }
       if (g.mode == GM_DENSE && cap >= 16 && o.bn > cap) {
         o.bn = cap;
         o.g.cg = tc_pick_cg(g, o.bn);
