@@ -101,3 +101,29 @@ def test_embedding_plan_and_errors():
     with pytest.raises(dj.DjinnError) as e:
         dj.djinn_describe(bad, dj.DJINN_BF16, 64)
     assert e.value.code == dj.DJINN_E_PARSE
+
+
+def _tiles(app, rows):
+    plan = dj.djinn_describe(dj.net_description(app), dj.DJINN_BF16, rows)[0]
+    out = {}
+    for line in plan.splitlines():
+        if "[dense" in line:
+            name = line.split()[1]
+            f = dict(kv.split("=", 1) for kv in line[line.index("[") + 1:].split() if "=" in kv)
+            out[name] = (int(f["bn"]), int(f["cg"]))
+    return out
+
+
+def test_dense_tiles_at_the_bench_batches():
+    """Dense GEMMs under one wave of 148 SMs take 64-wide single-CTA tiles when that stays
+    within two waves (DESIGN.md sec 5 item 10); the others keep their widest CTA-pair tiles."""
+    imc = _tiles("imc", 1024)
+    assert imc["fc6"] == (256, 2) and imc["fc7"] == (256, 2)      # 64-wide would be 512 tiles
+    assert imc["fc8"] == (64, 1)                                   # 8 x 16 = 128 tiles
+    face = _tiles("face", 256)
+    assert face["F7"] == (64, 1) and face["F8"] == (64, 1)
+    asr = _tiles("asr", 8192)
+    assert all(v == (256, 2) for v in asr.values())                # already > one wave
+    assert _tiles("pos", 4096)["l1"] == (64, 1)                    # 32 x 5 = 160 tiles
+    dig = _tiles("dig", 1600)
+    assert dig["ip1"] == (64, 1) and dig["ip2"] == (16, 1)
