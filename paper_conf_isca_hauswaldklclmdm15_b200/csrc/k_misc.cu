@@ -816,7 +816,11 @@ cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int C
     return !e || atoi(e) != 0;
   }();
   if (band_on && kernel == 3 && stride == 2 && pad == 0) {
-    constexpr int R = 4;
+    static const int R = [] {  // output rows per band (DJINN_POOL_R = 2 / 4 / 8)
+      const char* e = getenv("DJINN_POOL_R");
+      const int r = e ? atoi(e) : 4;
+      return (r == 2 || r == 8) ? r : 4;
+    }();
     const int xblocks = (OW + 256 / chunks - 1) / (256 / chunks);
     const int bpix = (OW + xblocks - 1) / xblocks;  // balanced column blocks
     const int bands = (OH + R - 1) / R;
@@ -824,12 +828,19 @@ cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int C
       const int64_t nr = rows - r0 < 65535 ? rows - r0 : 65535;
       dim3 blk(chunks, bpix), g(xblocks * bands, (unsigned)nr);
       const size_t xo = (size_t)r0 * H * W * Cpi, yo = (size_t)r0 * (OH + 2 * obd) * (OW + 2 * obd) * Cpo;
-      if (dt == DT_F16)
-        launch_pdl(pool_max_k3s2_band_kernel<__half, R>, dim3(g), dim3(blk), 0, st, (const __half*)x + xo, (__half*)y + yo,
-                   C, Cpi, gsz_i, gpitch_i, H, W, OH, OW, Cpo, gsz_o, gpitch_o, xu, obd, xblocks);
-      else
-        launch_pdl(pool_max_k3s2_band_kernel<__nv_bfloat16, R>, dim3(g), dim3(blk), 0, st, (const __nv_bfloat16*)x + xo,
-                   (__nv_bfloat16*)y + yo, C, Cpi, gsz_i, gpitch_i, H, W, OH, OW, Cpo, gsz_o, gpitch_o, xu, obd, xblocks);
+#define DJ_BAND_LAUNCH(T, RR)                                                                                      \
+  launch_pdl(pool_max_k3s2_band_kernel<T, RR>, dim3(g), dim3(blk), 0, st, (const T*)x + xo, (T*)y + yo, C, Cpi, gsz_i, \
+             gpitch_i, H, W, OH, OW, Cpo, gsz_o, gpitch_o, xu, obd, xblocks)
+      if (dt == DT_F16) {
+        if (R == 2) DJ_BAND_LAUNCH(__half, 2);
+        else if (R == 8) DJ_BAND_LAUNCH(__half, 8);
+        else DJ_BAND_LAUNCH(__half, 4);
+      } else {
+        if (R == 2) DJ_BAND_LAUNCH(__nv_bfloat16, 2);
+        else if (R == 8) DJ_BAND_LAUNCH(__nv_bfloat16, 8);
+        else DJ_BAND_LAUNCH(__nv_bfloat16, 4);
+      }
+#undef DJ_BAND_LAUNCH
     }
     return cudaGetLastError();
   }
