@@ -101,7 +101,47 @@ def djinn_load_net(desc: str, weights, precision: int, max_rows: int, device: in
     return h.value
 
 
+def _dtype_name(t) -> str:
+    return str(t.dtype).replace("torch.", "")
+
+
+def _numel(t) -> int:
+    return int(t.size if isinstance(t, np.ndarray) else t.numel())
+
+
+def _contiguous(t) -> bool:
+    return bool(t.flags["C_CONTIGUOUS"]) if isinstance(t, np.ndarray) else bool(t.is_contiguous())
+
+
+def _validate(net: int, inp, rows: int, out, out_mode: int, in_types) -> None:
+    """Argument checks the C ABI cannot make on raw pointers (the library would otherwise
+    read or write out of bounds): dtype, contiguity and element counts of both buffers."""
+    if rows < 0:
+        return                                   # the library reports DJINN_E_INVAL itself
+    in_elems, out_elems, _, _ = djinn_net_info(net)
+    def bad(msg):
+        raise DjinnError(DJINN_E_INVAL, msg)
+    if _dtype_name(inp) not in in_types:
+        bad(f"input dtype {_dtype_name(inp)}, expected one of {in_types}")
+    if not _contiguous(inp):
+        bad("input is not C-contiguous")
+    if _numel(inp) < rows * in_elems:
+        bad(f"input holds {_numel(inp)} elements, {rows} rows need {rows * in_elems}")
+    if out_mode == DJINN_OUT_ARGMAX:
+        o_types, o_need = ("int32",), rows
+    else:
+        o_types, o_need = ("float32",), rows * out_elems
+    if _dtype_name(out) not in o_types:
+        bad(f"output dtype {_dtype_name(out)}, mode {out_mode} needs {o_types[0]}")
+    if not _contiguous(out):
+        bad("output is not C-contiguous")
+    if _numel(out) < o_need:
+        bad(f"output holds {_numel(out)} elements, {rows} rows need {o_need}")
+
+
 def djinn_forward(net: int, inp, rows: int, out, out_mode: int, stream: Optional[int] = None) -> None:
+    """Mirror of djinn_forward: ``inp`` float32 rows, ``out`` float32 (int32 for ARGMAX)."""
+    _validate(net, inp, rows, out, out_mode, ("float32",))
     ip, imem = _ptr_mem(inp)
     op, omem = _ptr_mem(out)
     _check(lib().djinn_forward(net, ip, rows, imem, op, omem, out_mode, stream))
@@ -110,6 +150,7 @@ def djinn_forward(net: int, inp, rows: int, out, out_mode: int, stream: Optional
 def djinn_forward16(net: int, inp, rows: int, out, out_mode: int, stream: Optional[int] = None) -> None:
     """Mirror of djinn_forward16: ``inp`` holds the rows in the net's 16-bit type (a torch
     bfloat16 / float16 tensor or a numpy uint16 array of the raw bits)."""
+    _validate(net, inp, rows, out, out_mode, ("bfloat16", "float16", "uint16"))
     ip, imem = _ptr_mem(inp)
     op, omem = _ptr_mem(out)
     _check(lib().djinn_forward16(net, ip, rows, imem, op, omem, out_mode, stream))

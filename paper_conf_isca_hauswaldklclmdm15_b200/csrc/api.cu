@@ -87,6 +87,12 @@ int djinn_load_net(const char* desc, size_t desc_len, const float* weights, size
     }
     // per-layer tile choice and B tensor maps over the arena
     n.choose_tiles();
+    // GEMM rows are 32-bit in the kernels (M = rows x output pixels per row): reject a
+    // max_rows that would wrap instead of silently skipping the GEMM
+    for (const djinn::Op& o : n.ops)
+      if (o.kind == djinn::OP_GEMM && (int64_t)max_rows * o.ohw > (int64_t)INT32_MAX / 2)
+        return fail(DJINN_E_INVAL, o.name + ": max_rows x output pixels (" + std::to_string(max_rows) + " x " +
+                                       std::to_string(o.ohw) + ") exceeds the 32-bit GEMM row range");
     for (djinn::Op& o : n.ops) {
       if (o.kind != djinn::OP_GEMM || n.dt == djinn::DT_F32) continue;
       const djinn::GemmGeom& g = o.g;

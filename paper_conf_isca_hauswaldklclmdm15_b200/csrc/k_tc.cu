@@ -32,6 +32,8 @@
 #include <stdlib.h>
 
 #include "kernels.h"
+#include <atomic>
+#define TC_MAX_DEVICES 64
 
 #ifdef DJINN_TC_STATS
 #include <cstdio>
@@ -1274,14 +1276,18 @@ template <int BN, bool BF16, int CG, bool SLAB, int KSUB = BK / 16>
 cudaError_t launch_inst(const GemmGeom& g, const CUtensorMap* tmA, const CUtensorMap* tmB, const float* bias, void* Y,
                         cudaStream_t st) {
   using C = Cfg<BN, CG>;
-  static int attr_set = 0;  // benign race: idempotent attribute set
+  // The max-dynamic-smem attribute is per device context: cache it per device ordinal
+  // (benign race: the attribute set is idempotent).
+  static std::atomic<int> attr_set[TC_MAX_DEVICES];
   auto kern = tc_gemm_kernel<BN, BF16, CG, SLAB, KSUB>;
   const int smem = SLAB ? slab_smem<BN, CG>(g, g.stages) : C::SMEM;
   if (SLAB && (g.stages < 2 || smem > SLAB_SMEM_MAX)) return cudaErrorInvalidValue;
-  if (attr_set < smem) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= TC_MAX_DEVICES) return cudaErrorInvalidDevice;
+  if (attr_set[dev].load(std::memory_order_relaxed) < smem) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SLAB ? SLAB_SMEM_MAX : C::SMEM);
     if (e != cudaSuccess) return e;
-    attr_set = SLAB ? SLAB_SMEM_MAX : C::SMEM;
+    attr_set[dev].store(SLAB ? SLAB_SMEM_MAX : C::SMEM, std::memory_order_relaxed);
   }
   const int64_t mtiles = (g.mode == GM_CONV && g.a_tiled)
                              ? (int64_t)((g.OW + g.bx - 1) / g.bx) * ((g.OH + g.by - 1) / g.by) *

@@ -1022,6 +1022,7 @@ Workspace::~Workspace() {
   for (void* p : buf) if (p) cudaFree(p);
   if (in_stage) cudaFree(in_stage);
   if (in_stage16) cudaFree(in_stage16);
+  if (in_wide) cudaFree(in_wide);
   if (out_stage) cudaFree(out_stage);
   for (int s = 0; s < 2; ++s)
     for (cudaEvent_t e : {in_ready[s], in_free[s], out_ready[s], out_free[s]})
@@ -1129,8 +1130,10 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
   if (poisoned) throw Error(DJINN_E_CUDA, "net is poisoned by an earlier CUDA error");
   Workspace* w = workspace(st);
   const bool hin = in_mem == DJINN_MEM_HOST, hout = out_mem == DJINN_MEM_HOST;
-  if ((hin || in16) && !w->in_stage)
+  if (hin && !in16 && !w->in_stage)
     if (cudaMalloc(&w->in_stage, (size_t)max_rows * in_elems * 4) != cudaSuccess) throw Error(DJINN_E_NOMEM, "input staging");
+  if (in16 && !w->in_wide)
+    if (cudaMalloc(&w->in_wide, (size_t)max_rows * in_elems * 4) != cudaSuccess) throw Error(DJINN_E_NOMEM, "input widening");
   if (hin && in16 && !w->in_stage16)
     if (cudaMalloc(&w->in_stage16, (size_t)max_rows * in_elems * 2) != cudaSuccess) throw Error(DJINN_E_NOMEM, "input staging");
   const size_t in_row_bytes = (size_t)in_elems * (in16 ? 2 : 4);
@@ -1180,8 +1183,11 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
       src = (const float*)stage;
     }
     if (in16) {
-      // 16-bit rows -> fp32 (exact) in the fp32 staging buffer; the pack then runs unchanged
-      float* wide = w->in_stage + (size_t)(hin ? sl * cs : 0) * in_elems;
+      // 16-bit rows -> fp32 (exact) in their own buffer (chunks run in order on `st`, so one
+      // chunk's worth is enough); the pack then runs unchanged.  The H2D staging slots are
+      // never read by the pack on this path, so an interleaved host-fed djinn_forward cannot
+      // overwrite rows a pending pack still reads (its in_free wait covers the widen only).
+      float* wide = w->in_wide;
       cudaError_t e = launch_widen16(src, wide, n * in_elems, dt, st);
       ++launch_counter();
       if (e != cudaSuccess) {
@@ -1193,17 +1199,26 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
     }
     if (hout) ck(cudaStreamWaitEvent(st, w->out_free[sl], 0), "event wait");  // slot's previous D2H done
     uint8_t* dst = hout ? (uint8_t*)w->out_stage + (size_t)sl * cs * out_row_bytes : (uint8_t*)out + r0 * out_row_bytes;
-    const int pop = profile ? profile_op : -1;  // one timed op, or all (-1)
-    if (profile) {
+    // Profiling state is snapshotted under the lock: another thread may toggle it or grow
+    // prof_events / prof_recs (reallocating them) while this chunk's kernels are enqueued, so
+    // the chunk records into a local copy of its own event handles.
+    bool prof = false;
+    int pop = -1;  // one timed op, or all (-1)
+    std::vector<cudaEvent_t> pev;
+    {
       std::lock_guard<std::mutex> lk(mu);
-      prof_recs.push_back({prof_used, pop < 0 ? (int)ops.size() : 1, pop});
-      for (size_t i = 0; i <= (pop < 0 ? ops.size() : 1); ++i) prof_event();
+      prof = profile;
+      pop = profile_op;
+      if (prof) {
+        const size_t pbase = prof_used;
+        prof_recs.push_back({pbase, pop < 0 ? (int)ops.size() : 1, pop});
+        for (size_t i = 0; i <= (pop < 0 ? ops.size() : 1); ++i) pev.push_back(prof_event());
+      }
     }
-    const size_t pbase = profile ? prof_recs.back().first : 0;
     for (size_t i = 0; i < ops.size(); ++i) {
       const Op& o = ops[i];
       cudaError_t e = cudaSuccess;
-      if (profile && (pop < 0 || pop == (int)i)) ck(cudaEventRecord(prof_events[pbase + (pop < 0 ? i : 0)], st), "profile event");
+      if (prof && (pop < 0 || pop == (int)i)) ck(cudaEventRecord(pev[pop < 0 ? i : 0], st), "profile event");
       switch (o.kind) {
         case OP_PACK:
           if (o.embed) {
@@ -1218,6 +1233,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           g.ldwait = ldwait_mode();
           g.tslots = tslots_mode();
           g.epi_wg = epi_wg_mode(g);
+          if (n * o.ohw > (int64_t)INT32_MAX / 2) throw Error(DJINN_E_INVAL, o.name + ": GEMM rows exceed 32 bits");
           g.M = (int)(n * o.ohw);
           g.Nimg = (int)n;
           const void* A = w->buf[o.in_buf];
@@ -1258,10 +1274,10 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
         poisoned = true;
         throw Error(DJINN_E_CUDA, o.name + ": " + cudaGetErrorString(e));
       }
-      if (profile && pop == (int)i) ck(cudaEventRecord(prof_events[pbase + 1], st), "profile event");
+      if (prof && pop == (int)i) ck(cudaEventRecord(pev[1], st), "profile event");
       if (i == 0 && hin && !in16) ck(cudaEventRecord(w->in_free[sl], st), "event record");  // pack has read the slot
     }
-    if (profile && pop < 0) ck(cudaEventRecord(prof_events[pbase + ops.size()], st), "profile event");
+    if (prof && pop < 0) ck(cudaEventRecord(pev[ops.size()], st), "profile event");
     if (hout) {
       ck(cudaEventRecord(w->out_ready[sl], st), "event record");
       ck(cudaStreamWaitEvent(w->cout, w->out_ready[sl], 0), "event wait");

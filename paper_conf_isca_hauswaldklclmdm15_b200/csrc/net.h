@@ -99,6 +99,8 @@ struct Workspace {
   std::vector<void*> buf;  // 0/1 ping-pong, 2 logits, 3.. dedicated bordered tensors (borders stay zero)
   float* in_stage = nullptr;
   uint16_t* in_stage16 = nullptr;  // djinn_forward16 host rows (two slots like in_stage)
+  float* in_wide = nullptr;        // djinn_forward16: one chunk of rows widened to fp32 (read by
+                                   // the pack; never shared with the H2D staging slots)
   void* out_stage = nullptr;
   // host-fed mode: H2D on `cin`, D2H on `cout`, compute on the caller's stream; two staging
   // slots, each with a "filled" and a "drained" event (Net::forward)

@@ -7,19 +7,14 @@ import torch
 import paper_conf_isca_hauswaldklclmdm15_b200 as dj
 from datagen import recipes
 
-from parity import (FP32_PROB_TOL, REL_LOGIT_TOL, TOP1_MIN, blob, compare_16bit, compare_fp32,
-                    oracle_net, oracle_rows)
+from parity import (ELEM_TOL, FP32_PROB_TOL, REL_LOGIT_TOL, TOP1_MIN, TOP1_MIN_ROWS, blob, compare_16bit,
+                    compare_fp32, oracle_net, oracle_rows)
 
 pytestmark = pytest.mark.gpu
 
 # rows per parity case: small enough for the oracle in seconds, > one M tile with a ragged tail
 ROWS = {"dig": 300, "pos": 1000, "chk": 1000, "ner": 1000, "asr": 300, "face": 6, "imc": 6}
 APPS = list(ROWS)
-# DESIGN.md reading R14: top-1 agreement is asserted wherever the path's noise allows it; the
-# ASR service returns 548 probability vectors per query (Table 3), not a
-# classification, so on bf16 its asserted bound is the relative logit error and top-1 (99.3%
-# of decidable rows at tau = 1e-2, measured) is reported only.
-TOP1_REPORT_ONLY = {("asr", "bf16")}
 
 
 def run_gpu(app, prec, x, max_rows=None, mode=dj.DJINN_OUT_LOGITS):
@@ -55,7 +50,10 @@ def test_tensor_core_path_matches_oracle(app, prec):
     r = compare_16bit(lg, lg_ref)
     print(app, prec, r)
     assert r["rel_max"] <= REL_LOGIT_TOL, r
-    if (app, prec) not in TOP1_REPORT_ONLY:
+    assert r["elem_max"] <= ELEM_TOL, r
+    # top-1 >= 99.9 % is a rate: asserted here when the case has >= 1000 rows, and for every
+    # (app, precision) over the full bench batch in test_fullsize_gpu.py (reading R14)
+    if r["rows"] >= TOP1_MIN_ROWS:
         assert r["top1_decidable"] >= TOP1_MIN, r
 
 
