@@ -75,39 +75,60 @@ ROWS = 300          # c1 of gen_a: 300 x 64 output pixels = 150 M tiles of 128 p
 SEED = 0x5EED
 
 
-def _gain(net: OracleNet, i: int) -> float:
-    """Weight gain of the parametrised layer at net.layers[i]: large before an LRN (so its
-    denominator is exercised), 2 before a saturating activation, 4 for the logit
-    layer (the calibrated Tonic nets' logit std), else 1."""
+def _target(net: OracleNet, i: int) -> float:
+    """Target pre-activation std of the parametrised layer at net.layers[i] (the Tonic nets'
+    calibration rule, oracle/calibrate.py): 100 before an LRN (its denominator is exercised),
+    4 for the logit layer and before a sigmoid, 1 elsewhere."""
     if not any("w_shape" in L for L in net.layers[i + 1:]):
         return 4.0
     for L in net.layers[i + 1:]:
         if L["type"] in ("ReLU", "Dropout"):
             continue
         if L["type"] == "LRN":
-            return 60.0
-        if L["type"] in ("TanH", "Sigmoid", "HardTanh"):
-            return 2.0
+            return 100.0
+        if L["type"] == "Sigmoid":
+            return 4.0
         break
     return 1.0
 
 
 def gen_net(name: str, grid: str):
-    """Seeded weights (U(-1,1) * gain * sqrt(3 / fan_in), bias U(-0.1,0.1)) and inputs
-    U(-1,1), on the path's storage grid."""
+    """Seeded inputs U(-1,1) and weights U(-1,1) * sqrt(3 / fan_in), each output channel
+    standardised (LSUV, by the fp64 oracle on a 64-row calibration batch) to the target std
+    with bias jitter 0.1 * t -- the Tonic nets' recipe, so the logits stay input-sensitive and
+    16-bit rounding is not amplified by near-zero rows.  Everything on the path's grid."""
     net = OracleNet(NETS[name])
+    shp = tuple(net.input_shape)
+    per = int(np.prod(shp))
+    h = rng.uniform(SEED ^ 0xCA1, 1, 0, 64 * per, -1.0, 1.0).reshape((64,) + shp)
     W, p = [], 0
     for i, L in enumerate(net.layers):
-        if "w_shape" not in L:
+        if L["type"] in ("Input", "Softmax"):
             continue
-        a = _gain(net, i) * np.sqrt(3.0 / L["fan_in"])
+        if "w_shape" not in L:
+            h = net.apply(L, h)
+            continue
+        a = np.sqrt(3.0 / L["fan_in"])
         nw, nb = int(np.prod(L["w_shape"])), int(np.prod(L["b_shape"]))
         w = rng.uniform(SEED, 10 + 2 * p, 0, nw, -a, a).reshape(L["w_shape"])
-        b = rng.uniform(SEED, 11 + 2 * p, 0, nb, -0.1, 0.1).reshape(L["b_shape"])
-        W.append({"w": rng.round_to_grid(w, grid), "b": rng.round_to_grid(b, "fp32")})
+        z = net.apply(L, h, w, np.zeros(L["b_shape"]))
+        axes = (0,) if z.ndim == 2 else (0, 2, 3)
+        mu, sd = z.mean(axis=axes), z.std(axis=axes)
+        sd = np.where(sd > 0, sd, 1.0)
+        t = _target(net, i)
+        ax = 2 if L["type"] == "LocallyConnected" else 0
+        shape = [1] * w.ndim
+        shape[ax] = -1
+        w = w * (t / sd).reshape(shape)
+        jit = rng.uniform(SEED, 11 + 2 * p, 0, nb, -0.1 * t, 0.1 * t).reshape(L["b_shape"])
+        bsh = [1] * len(L["b_shape"])
+        bsh[0] = -1
+        b = (-mu * t / sd).reshape(bsh) + jit
+        wg, bg = rng.round_to_grid(w, grid), rng.round_to_grid(b, "fp32")
+        W.append({"w": wg, "b": bg})
+        h = net.apply(L, h, wg.astype(np.float64), bg.astype(np.float64))
         p += 1
-    shp = tuple(net.input_shape)
-    x = rng.round_to_grid(rng.uniform(SEED, 1, 0, ROWS * int(np.prod(shp)), -1.0, 1.0), grid)
+    x = rng.round_to_grid(rng.uniform(SEED, 1, 0, ROWS * per, -1.0, 1.0), grid)
     return net, W, x.reshape((ROWS,) + shp)
 
 
