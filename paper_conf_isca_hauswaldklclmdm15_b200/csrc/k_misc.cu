@@ -686,8 +686,8 @@ __device__ __forceinline__ uint4 max8(uint4 a, uint4 b, __nv_bfloat16) {
 
 template <typename T, int K>
 __global__ void pool_max_remap_kernel(const T* __restrict__ x, T* __restrict__ y, int C, int Cpi, int gsz_i,
-                                      int gpitch_i, int H, int W, int OH, int OW, int kern, int stride, int pad,
-                                      int Cpo, int gsz_o, int gpitch_o, int xu, int obd) {
+                                      int gpitch_i, int H, int W, int Hst, int Wst, int OH, int OW, int kern, int stride,
+                                      int pad, int Cpo, int gsz_o, int gpitch_o, int xu, int obd) {
   pdl_trigger();
   pdl_wait();
   __shared__ int in_off[64];  // per output chunk: input channel offset, -1 = zero chunk
@@ -705,7 +705,7 @@ __global__ void pool_max_remap_kernel(const T* __restrict__ x, T* __restrict__ y
   T* yo = y + ((r * (OH + 2 * obd) + oy + obd) * (OW + 2 * obd) + ox + obd) * (int64_t)Cpo + threadIdx.x * 8;
   uint4 ov = make_uint4(0, 0, 0, 0);
   if (off >= 0) {
-    const T* base = x + r * (int64_t)H * W * Cpi + off;
+    const T* base = x + r * (int64_t)Hst * Wst * Cpi + off;
     int hs = oy * stride - pad, ws = ox * stride - pad;
     int he = min(hs + kern, H + pad), we = min(ws + kern, W + pad);
     hs = max(hs, 0); ws = max(ws, 0); he = min(he, H); we = min(we, W);
@@ -718,16 +718,16 @@ __global__ void pool_max_remap_kernel(const T* __restrict__ x, T* __restrict__ y
 #pragma unroll
         for (int b = 0; b < K; ++b) {
           const int h = min(hs + a, he - 1), w = min(ws + b, we - 1);
-          v[a * K + b] = __ldg(reinterpret_cast<const uint4*>(base + ((int64_t)h * W + w) * Cpi));
+          v[a * K + b] = __ldg(reinterpret_cast<const uint4*>(base + ((int64_t)h * Wst + w) * Cpi));
         }
       ov = v[0];
 #pragma unroll
       for (int j = 1; j < K * K; ++j) ov = max8(ov, v[j], T());
     } else {
-      ov = __ldg(reinterpret_cast<const uint4*>(base + ((int64_t)hs * W + ws) * Cpi));
+      ov = __ldg(reinterpret_cast<const uint4*>(base + ((int64_t)hs * Wst + ws) * Cpi));
       for (int h = hs; h < he; ++h)
         for (int w = ws; w < we; ++w)
-          ov = max8(ov, __ldg(reinterpret_cast<const uint4*>(base + ((int64_t)h * W + w) * Cpi)), T());
+          ov = max8(ov, __ldg(reinterpret_cast<const uint4*>(base + ((int64_t)h * Wst + w) * Cpi)), T());
     }
   }
   *reinterpret_cast<uint4*>(yo) = ov;
@@ -744,8 +744,8 @@ __global__ void pool_max_remap_kernel(const T* __restrict__ x, T* __restrict__ y
 // clip to the image (Caffe ceil geometry); clipped taps re-read the last row/column (exact).
 template <typename T, int R>
 __global__ void pool_max_k3s2_band_kernel(const T* __restrict__ x, T* __restrict__ y, int C, int Cpi, int gsz_i,
-                                          int gpitch_i, int H, int W, int OH, int OW, int Cpo, int gsz_o,
-                                          int gpitch_o, int xu, int obd, int xblocks) {
+                                          int gpitch_i, int H, int W, int Hst, int Wst, int OH, int OW, int Cpo,
+                                          int gsz_o, int gpitch_o, int xu, int obd, int xblocks) {
   pdl_trigger();
   pdl_wait();
   __shared__ int in_off[64];
@@ -773,10 +773,10 @@ __global__ void pool_max_k3s2_band_kernel(const T* __restrict__ x, T* __restrict
     }
     return;
   }
-  const T* base = x + r * (int64_t)H * W * Cpi + off;
+  const T* base = x + r * (int64_t)Hst * Wst * Cpi + off;
   const int ws = ox * 2, w1 = min(ws + 1, W - 1), w2 = min(ws + 2, W - 1);
   auto hrow = [&](int h) {
-    const T* p = base + (int64_t)h * W * Cpi;
+    const T* p = base + (int64_t)h * Wst * Cpi;
     const uint4 a = __ldg(reinterpret_cast<const uint4*>(p + (int64_t)ws * Cpi));
     const uint4 b = __ldg(reinterpret_cast<const uint4*>(p + (int64_t)w1 * Cpi));
     const uint4 c = __ldg(reinterpret_cast<const uint4*>(p + (int64_t)w2 * Cpi));
@@ -798,9 +798,9 @@ __global__ void pool_max_k3s2_band_kernel(const T* __restrict__ x, T* __restrict
 }
 
 cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int Cpi, int gsz_i, int gpitch_i, int H,
-                              int W, int OH, int OW, int kernel, int stride, int pad, int Cpo, int gsz_o, int gpitch_o,
-                              int xu, int obd, int dt, cudaStream_t st) {
-  if (xu < 1 || Cpo % xu || obd < 0 || (obd > 0 && xu > 1)) return cudaErrorInvalidValue;
+                              int W, int Hst, int Wst, int OH, int OW, int kernel, int stride, int pad, int Cpo, int gsz_o,
+                              int gpitch_o, int xu, int obd, int dt, cudaStream_t st) {
+  if (xu < 1 || Cpo % xu || obd < 0 || (obd > 0 && xu > 1) || Hst < H || Wst < W) return cudaErrorInvalidValue;
   // plain layouts: one group spanning every position (channel c at c; pads read as zeros)
   const bool gi = gsz_i < C, go = gsz_o < C;
   if (!gi) gsz_i = gpitch_i = 1 << 30;
@@ -827,10 +827,10 @@ cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int C
     for (int64_t r0 = 0; r0 < rows; r0 += 65535) {
       const int64_t nr = rows - r0 < 65535 ? rows - r0 : 65535;
       dim3 blk(chunks, bpix), g(xblocks * bands, (unsigned)nr);
-      const size_t xo = (size_t)r0 * H * W * Cpi, yo = (size_t)r0 * (OH + 2 * obd) * (OW + 2 * obd) * Cpo;
+      const size_t xo = (size_t)r0 * Hst * Wst * Cpi, yo = (size_t)r0 * (OH + 2 * obd) * (OW + 2 * obd) * Cpo;
 #define DJ_BAND_LAUNCH(T, RR)                                                                                      \
   launch_pdl(pool_max_k3s2_band_kernel<T, RR>, dim3(g), dim3(blk), 0, st, (const T*)x + xo, (T*)y + yo, C, Cpi, gsz_i, \
-             gpitch_i, H, W, OH, OW, Cpo, gsz_o, gpitch_o, xu, obd, xblocks)
+             gpitch_i, H, W, Hst, Wst, OH, OW, Cpo, gsz_o, gpitch_o, xu, obd, xblocks)
       if (dt == DT_F16) {
         if (R == 2) DJ_BAND_LAUNCH(__half, 2);
         else if (R == 8) DJ_BAND_LAUNCH(__half, 8);
@@ -848,9 +848,9 @@ cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int C
   for (int64_t r0 = 0; r0 < rows; r0 += 65535) {  // grid.z <= 65535 images per launch
     const int64_t nr = rows - r0 < 65535 ? rows - r0 : 65535;
     dim3 blk(chunks, pix), g((OH * OW + pix - 1) / pix, (unsigned)nr);
-    const size_t xo = (size_t)r0 * H * W * Cpi, yo = (size_t)r0 * (OH + 2 * obd) * (OW + 2 * obd) * Cpo;
+    const size_t xo = (size_t)r0 * Hst * Wst * Cpi, yo = (size_t)r0 * (OH + 2 * obd) * (OW + 2 * obd) * Cpo;
 #define DJ_POOL_LAUNCH(T, KK)                                                                                   \
-  launch_pdl(pool_max_remap_kernel<T, KK>, dim3(g), dim3(blk), 0, st, (const T*)x + xo, (T*)y + yo, C, Cpi, gsz_i, gpitch_i, H, W, OH, OW, \
+  launch_pdl(pool_max_remap_kernel<T, KK>, dim3(g), dim3(blk), 0, st, (const T*)x + xo, (T*)y + yo, C, Cpi, gsz_i, gpitch_i, H, W, Hst, Wst, OH, OW, \
                                                   kernel, stride, pad, Cpo, gsz_o, gpitch_o, xu, obd)
     if (dt == DT_F16) {
       if (kernel == 3) DJ_POOL_LAUNCH(__half, 3);

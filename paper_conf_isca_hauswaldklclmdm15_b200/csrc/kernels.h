@@ -174,6 +174,24 @@ bool tc_slab_config(GemmGeom& g, int bn);
 cudaError_t launch_tc_gemm(const GemmGeom& g, int bn, int dt, const CUtensorMap* tmA,
                            const CUtensorMap* tmB, const float* bias, void* Y, cudaStream_t st);
 
+// --- fused first layer (K0 + K2 [+ K4]): fp32 NCHW images -> strided conv (space-to-depth by
+// the stride F into an Hs x Ws grid, KS x KS stride-1 taps), bias + act [+ Caffe LRN], 16-bit
+// NHWC output [Nimg][OH][OW][N] written by TMA tensor stores (k_stem.cu).
+// tmB: as launch_tc_gemm (box {64, N/2, 1}); tmY0: 4D map {Cp, OW, OH, rows} of the output, box
+// {64, 32, 1, 1}, SWIZZLE_128B; tmY1: the same map with box {32, 32, 1, 1}, SWIZZLE_64B.
+struct StemGeom {
+  int Nimg;            // images in this launch
+  int H, W;            // fp32 input image (C0 channels)
+  int Hs, Ws;          // space-to-depth grid (virtual GEMM rows per image = Hs * Ws)
+  int OH, OW;          // valid output pixels
+  int N;               // output channels (= tile width, = output pitch)
+  int act, epi_lrn, out_half;
+  float lrn_alpha_over_n, lrn_beta, lrn_k;
+};
+bool stem_supported(int bn, int f, int c0, int ks, int out_pitch);
+cudaError_t launch_stem_conv(const StemGeom& g, int dt, const CUtensorMap* tmB, const CUtensorMap* tmY0,
+                             const CUtensorMap* tmY1, const float* x, const float* bias, cudaStream_t st);
+
 // --- LRN across channels (K4), NHWC ----------------------------------------------------------
 // Channel c of a pixel is stored at (c/gsz)*gpitch + c%gsz (grouped layouts); pads -> 0.
 cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, int gsz, int gpitch, int size,
@@ -182,9 +200,10 @@ cudaError_t launch_lrn(const void* x, void* y, int64_t pixels, int C, int Cp, in
 // --- MAX pooling with a channel-layout change (plain/grouped in, plain/grouped/x-unrolled out), 16-bit,
 // kernel <= stride + 1.  obd: zero border of the stored output ((OH+2obd) x (OW+2obd) pixels;
 // the border is never written).
+// The input is stored on an Hst x Wst grid (>= H x W; pixel (y, x) at y * Wst + x).
 cudaError_t launch_pool_remap(const void* x, void* y, int64_t rows, int C, int Cpi, int gsz_i, int gpitch_i, int H,
-                              int W, int OH, int OW, int kernel, int stride, int pad, int Cpo, int gsz_o, int gpitch_o,
-                              int xu, int obd, int dt, cudaStream_t st);
+                              int W, int Hst, int Wst, int OH, int OW, int kernel, int stride, int pad, int Cpo, int gsz_o,
+                              int gpitch_o, int xu, int obd, int dt, cudaStream_t st);
 
 // --- LRN + max pooling fused (K4+K5): fp16 NHWC input (pitch Cpi, C channels, pads zero),
 // Caffe LRN across channels in fp32, Caffe MAX pooling (kernel 3, stride 2, pad 0) of the LRN

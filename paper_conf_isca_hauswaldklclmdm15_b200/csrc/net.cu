@@ -822,6 +822,31 @@ void Net::build(const std::string& desc) {
       ops.push_back(lp);
     }
   }
+  // Fused first layer (k_stem.cu): a space-to-depth first conv whose output is a plain
+  // NHWC tensor reads the fp32 images itself; the pack op is then not launched.  Opt-in
+  // (DJINN_STEM=1): correct and bitwise equal to pack + slab GEMM, but measured slower on B200
+  // (IMC conv1+norm1 638 us vs pack 163 + conv1 397 us; its fp32 gather is the bottleneck,
+  // DESIGN.md sec 5).
+  {
+    const char* se = getenv("DJINN_STEM");
+    if (f16 && (se && se[0] == '1') && ops.size() > 1 && ops[0].kind == OP_PACK && ops[0].xform == 1 &&
+        ops[1].kind == OP_GEMM && ops[1].xform == 1) {
+      Op& c = ops[1];
+      const GemmGeom& g = c.g;
+      // its output is the whole virtual Hs x Ws grid (one TMA store per 32 pixels); the consumer
+      // must be a pool that reads the stored grid (the MAX pool with a layout change)
+      const bool pool_next = ops.size() > 2 && ops[2].kind == OP_POOL && ops[2].is_max && ops[2].kernel <= ops[2].stride + 1 &&
+                             ops[2].in_buf == c.out_buf;
+      if (pool_next && g.mode == GM_CONV && g.Z == 1 && g.zf == 1 && g.stride == 1 && g.pad == 0 && g.xb <= 1 &&
+          !g.out_f32 && !g.out_half && c.out.gsz >= c.out.C && c.out.bdr == 0 && c.out.Cp == g.N && g.KH == g.KW &&
+          g.H - g.OH >= 0 && g.W - g.OW >= 0 && stem_supported(g.N, c.xf, c.orig_in.C, g.KH, c.out.Cp)) {
+        c.stem = 1;
+        ops[0].fused = 1;
+        c.out.hx = ops[2].in.hx = g.H - g.OH;
+        c.out.wx = ops[2].in.wx = g.W - g.OW;
+      }
+    }
+  }
   out_elems = cur.C;
   arena_bytes = rupz(arena_off, 1024);
   // Centered sigmoid storage on 16-bit paths: a sigmoid layer feeding a dense layer stores
@@ -841,7 +866,7 @@ void Net::build(const std::string& desc) {
     switch (o.kind) {
       case OP_PACK:
         // lookup: indices in, window vector out, one table row read per (word, table)
-        o.bytes_row = o.embed ? in_e * 4 + 2.0 * out_e * es : in_e * 4 + in_e * es;
+        o.bytes_row = o.fused ? 0.0 : o.embed ? in_e * 4 + 2.0 * out_e * es : in_e * 4 + in_e * es;
         break;
       case OP_GEMM: {
         const GemmGeom& g = o.g;
@@ -850,7 +875,7 @@ void Net::build(const std::string& desc) {
         else if (g.mode == GM_LC) kreal = (double)o.orig_k * o.orig_k * oin.C;
         else kreal = (double)o.orig_k * o.orig_k * (oin.C / (g.zf > 1 ? g.zf : g.Z));
         o.flops_row = 2.0 * out_e * kreal;
-        o.bytes_row = in_e * es + out_e * (g.out_f32 ? 4.0 : es);
+        o.bytes_row = in_e * (o.stem ? 4.0 : es) + out_e * (g.out_f32 ? 4.0 : es);  // stem: reads the fp32 images
         const double nb = g.mode == GM_DENSE ? g.N : (double)g.Z * g.bias_zstride;
         o.weight_bytes = (g.mode == GM_LC ? (double)g.Z * g.N * kreal
                                           : (g.mode == GM_CONV ? (double)o.out.C * kreal : (double)g.N * kreal)) * es +
@@ -903,6 +928,7 @@ void Net::choose_tiles() {
         o.g.cg = tc_pick_cg(g, o.bn);
       }
     }
+    if (o.stem) o.g.cg = 2;  // the stem kernel loads B as two boxes of bn / 2 rows per K block
     if (o.g.slab && !tc_slab_config(o.g, o.bn)) {
       o.g.slab = 0;
       o.ohw = o.g.OH * o.g.OWb;
@@ -1063,6 +1089,19 @@ Workspace* Net::workspace(cudaStream_t st) {
     ck(cudaMemset(w->buf[b], 0, buf_bytes[b]), "workspace memset");
   }
   w->tmA.resize(ops.size());
+  w->tmY0.resize(ops.size());
+  w->tmY1.resize(ops.size());
+  for (size_t i = 0; i < ops.size(); ++i) {
+    const Op& o = ops[i];
+    if (!o.stem) continue;
+    // output: the virtual grid [rows * Hs * Ws][Cp]; boxes of 32 pixels x 64 / 32 channels
+    const int Cp = o.out.Cp, odt = o.g.out_half ? DT_F16 : dt;
+    uint64_t dims[2] = {(uint64_t)Cp, (uint64_t)max_rows * (o.out.H + o.out.hx) * (o.out.W + o.out.wx)};
+    uint64_t strides[1] = {(uint64_t)Cp * 2};
+    uint32_t box0[2] = {64, 32}, box1[2] = {32, 32};
+    encode_tmap(&w->tmY0[i], odt, w->buf[o.out_buf], 2, dims, strides, box0, 128);
+    encode_tmap(&w->tmY1[i], odt, w->buf[o.out_buf], 2, dims, strides, box1, 64);
+  }
   if (dt != DT_F32) {
     for (size_t i = 0; i < ops.size(); ++i) {
       const Op& o = ops[i];
@@ -1218,9 +1257,11 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
     for (size_t i = 0; i < ops.size(); ++i) {
       const Op& o = ops[i];
       cudaError_t e = cudaSuccess;
+      bool skipped = false;
       if (prof && (pop < 0 || pop == (int)i)) ck(cudaEventRecord(pev[pop < 0 ? i : 0], st), "profile event");
       switch (o.kind) {
         case OP_PACK:
+          if (o.fused) { skipped = true; break; }  // the stem GEMM reads the fp32 rows itself
           if (o.embed) {
             e = launch_embed(src, (const uint8_t*)arena + o.w_off, w->buf[0], n, o.eg, o.out.Cp, dt, st);
             break;
@@ -1239,7 +1280,17 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           const void* A = w->buf[o.in_buf];
           void* Y = w->buf[o.out_buf];
           const uint8_t* ar = (const uint8_t*)arena;
-          if (dt == DT_F32)
+          if (o.stem) {
+            StemGeom sg{};
+            sg.Nimg = (int)n;
+            sg.H = o.orig_in.H; sg.W = o.orig_in.W;
+            sg.Hs = g.H; sg.Ws = g.W;
+            sg.OH = g.OH; sg.OW = g.OW;
+            sg.N = g.N;
+            sg.act = g.act; sg.epi_lrn = g.epi_lrn; sg.out_half = g.out_half;
+            sg.lrn_alpha_over_n = g.lrn_alpha_over_n; sg.lrn_beta = g.lrn_beta; sg.lrn_k = g.lrn_k;
+            e = launch_stem_conv(sg, dt, &o.tmB, &w->tmY0[i], &w->tmY1[i], src, (const float*)(ar + o.b_off), st);
+          } else if (dt == DT_F32)
             e = launch_simt_gemm(g, (const float*)A, (const float*)(ar + o.w_off), (const float*)(ar + o.b_off),
                                  (float*)Y, st);
           else
@@ -1254,8 +1305,8 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
         case OP_POOL:
           if (dt != DT_F32 && o.is_max && o.kernel <= o.stride + 1)
             e = launch_pool_remap(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.gsz, o.in.gpitch,
-                                  o.in.H, o.in.W, o.out.H, o.out.W, o.kernel, o.stride, o.pad, o.out.Cp, o.out.gsz,
-                                  o.out.gpitch, o.out.xu, o.out.bdr, dt, st);
+                                  o.in.H, o.in.W, o.in.H + o.in.hx, o.in.W + o.in.wx, o.out.H, o.out.W, o.kernel,
+                                  o.stride, o.pad, o.out.Cp, o.out.gsz, o.out.gpitch, o.out.xu, o.out.bdr, dt, st);
           else
             e = launch_pool(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.H, o.in.W, o.out.H, o.out.W,
                             o.kernel, o.stride, o.pad, o.is_max, o.out.xu, dt, st);
@@ -1269,13 +1320,14 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           e = launch_softmax((const float*)w->buf[2], n, (int)out_elems, out_pitch, dst, mode, st);
           break;
       }
-      ++launches;
+      if (!skipped) ++launches;
       if (e != cudaSuccess) {
         poisoned = true;
         throw Error(DJINN_E_CUDA, o.name + ": " + cudaGetErrorString(e));
       }
       if (prof && pop == (int)i) ck(cudaEventRecord(pev[1], st), "profile event");
-      if (i == 0 && hin && !in16) ck(cudaEventRecord(w->in_free[sl], st), "event record");  // pack has read the slot
+      if (i == (ops[0].fused ? 1u : 0u) && hin && !in16)
+        ck(cudaEventRecord(w->in_free[sl], st), "event record");  // the pack (or the stem GEMM) has read the slot
     }
     if (prof && pop < 0) ck(cudaEventRecord(pev[ops.size()], st), "profile event");
     if (hout) {
@@ -1316,8 +1368,10 @@ std::string Net::plan_string() const {
         << (o.g.lcg > 1 ? " taps/row=" + std::to_string(o.g.lcg) : std::string())
         << (o.g.mode == GM_CONV && o.g.a_tiled ? " block=" + std::to_string(o.g.bx) + "x" + std::to_string(o.g.by) + "x" +
                                                   std::to_string(o.g.bn) : std::string())
+        << (o.stem ? " stem(fp32 input, fused pack, resident B, TMA-store epilogue)" : "")
         << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << (o.g.out_half ? " fp16-out" : "") << "]";
     if (o.kind == OP_PACK && o.embed) s << " [embedding window " << o.eg.window << " tables " << o.eg.T << " D " << o.eg.D << "]";
+    if (o.kind == OP_PACK && o.fused) s << " [fused into the next op]";
     if (o.kind == OP_PACK && o.xform) s << " [" << (o.xform == 1 ? "space-to-depth " : "kx-unroll ") << o.xf << (o.xs > 1 ? " step " + std::to_string(o.xs) : std::string()) << "]";
     s << "\n";
   }

@@ -56,7 +56,9 @@ struct Shape {
   int xu = 1, P = 0;  // x-unrolled layout: pixel x stores pixels x..x+xu-1, each at pitch P (Cp = xu*P)
   int bdr = 0;        // zero border: stored (H + 2 bdr) x (W + 2 bdr) pixels, pixel (y, x) at (y + bdr, x + bdr)
                       // (the input of a slab convolution: its zero padding is stored)
-  int64_t per_row() const { return (int64_t)(H + 2 * bdr) * (W + 2 * bdr) * Cp; }
+  int hx = 0, wx = 0; // extra stored rows / columns after the image (never read): the fused first
+                      // layer writes its whole virtual Hs x Ws grid (k_stem.cu), pixel (y, x) at (y, x)
+  int64_t per_row() const { return (int64_t)(H + 2 * bdr + hx) * (W + 2 * bdr + wx) * Cp; }
   int pos(int c) const { return (c / gsz) * gpitch + c % gsz; }
 };
 
@@ -76,6 +78,9 @@ struct Op {
   // by xf (= conv stride), 2 kx-unroll of a stride-1 kernel of width xf
   int xform = 0, xf = 1, xs = 1;  // xs: kx-unroll x step (packed pixel j starts at input x = j*xs)
   Shape orig_in;                // the layer's input before the transform
+  // fused first layer (k_stem.cu): the GEMM reads the fp32 input itself (stem = 1) and the
+  // pack op before it is not launched (fused = 1)
+  int stem = 0, fused = 0;
   // SENNA window lookup in place of the pack (embed = 1): see EmbedGeom (kernels.h)
   int embed = 0;
   EmbedGeom eg{};
@@ -108,6 +113,7 @@ struct Workspace {
   cudaEvent_t in_ready[2] = {}, in_free[2] = {}, out_ready[2] = {}, out_free[2] = {};
   int64_t pipe_cs = 0;  // chunk rows of the last host-fed call (slot offsets depend on it)
   std::vector<CUtensorMap> tmA;  // per op (dense gemm) over its input buffer
+  std::vector<CUtensorMap> tmY0, tmY1;  // per op (stem): TMA-store maps over its output buffer
   ~Workspace();
 };
 

@@ -275,3 +275,43 @@ def test_band_pool_equals_per_pixel_pool_bitwise(app, prec, n, tmp_path):
                        timeout=600)
         outs.append(np.load(f))
     assert np.array_equal(outs[0], outs[1])
+
+
+# ---------------------------------------------------------------- fused first layer (k_stem.cu)
+_STEM_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+sys.path.insert(0, sys.argv[1] + "/tests")
+import paper_conf_isca_hauswaldklclmdm15_b200 as dj
+from datagen import recipes
+from parity import blob
+app, prec, n, start = sys.argv[2], sys.argv[3], int(sys.argv[4]), int(sys.argv[6])
+x = recipes.gen_input_rows(app, start, n, prec)
+net = dj.DjinnNet(dj.net_description(app), blob(app, prec), prec, n)
+print(net.plan())
+np.save(sys.argv[5], net.forward(torch.from_numpy(x).cuda(), dj.DJINN_OUT_LOGITS).cpu().numpy())
+net.close()
+"""
+
+
+@pytest.mark.parametrize("prec,n,start", [("fp16", 7, 0), ("bf16", 3, 11), ("fp16", 130, 5)])
+def test_stem_conv_equals_pack_plus_slab_gemm_bitwise(prec, n, start, tmp_path):
+    """IMC conv1+norm1 as the fused first-layer kernel (fp32 images gathered into the
+    space-to-depth slab in shared memory, resident B, TMA-store epilogue) and as the separate
+    pack + slab GEMM (DJINN_STEM=0) give bitwise-equal logits: the same 16-bit operands reach
+    the same MMAs in the same order, and the epilogue arithmetic is the same.  n = 7 / 3 / 130
+    images: tiles that straddle image boundaries and a ragged last tile."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    outs, plans = [], []
+    for stem in ("1", "0"):
+        f = str(tmp_path / f"lg{stem}.npy")
+        env = dict(os.environ, DJINN_STEM=stem)
+        r = subprocess.run([sys.executable, "-c", _STEM_CHILD, root, "imc", prec, str(n), f, str(start)], env=env,
+                           check=True, timeout=600, capture_output=True, text=True)
+        plans.append(r.stdout)
+        outs.append(np.load(f))
+    assert "stem(" in plans[0] and "stem(" not in plans[1], plans
+    assert np.array_equal(outs[0], outs[1])
