@@ -174,11 +174,14 @@ bool tc_slab_config(GemmGeom& g, int bn);
 cudaError_t launch_tc_gemm(const GemmGeom& g, int bn, int dt, const CUtensorMap* tmA,
                            const CUtensorMap* tmB, const float* bias, void* Y, cudaStream_t st);
 
-// --- fused first layer (K0 + K2 [+ K4]): fp32 NCHW images -> strided conv (space-to-depth by
-// the stride F into an Hs x Ws grid, KS x KS stride-1 taps), bias + act [+ Caffe LRN], 16-bit
-// NHWC output [Nimg][OH][OW][N] written by TMA tensor stores (k_stem.cu).
-// tmB: as launch_tc_gemm (box {64, N/2, 1}); tmY0: 4D map {Cp, OW, OH, rows} of the output, box
-// {64, 32, 1, 1}, SWIZZLE_128B; tmY1: the same map with box {32, 32, 1, 1}, SWIZZLE_64B.
+// --- first-layer strided conv with a resident filter bank (K2 [+ K4], k_stem.cu): space-to-depth
+// by the stride F into an Hs x Ws grid, KS x KS stride-1 taps, bias + act [+ Caffe LRN], 16-bit
+// NHWC output over the whole virtual grid [Nimg * Hs * Ws][N] written by TMA tensor stores.
+// gather = 1: reads the fp32 NCHW images x itself (K0 fused); gather = 0: reads the packed
+// 16-bit space-to-depth tensor through tmA (2D {64, rows * Hs * Ws}, box {64, slab_rows}).
+// tmB: as launch_tc_gemm (box {64, N/2, 1}); tmY0: 2D map {Cp, rows * Hs * Ws} of the output,
+// box {64, 32}, SWIZZLE_128B; tmY1: the same map with box {32, 32}, SWIZZLE_64B (gather only;
+// otherwise channels past 64 are stored from registers into Y).
 struct StemGeom {
   int Nimg;            // images in this launch
   int H, W;            // fp32 input image (C0 channels)
@@ -186,11 +189,13 @@ struct StemGeom {
   int OH, OW;          // valid output pixels
   int N;               // output channels (= tile width, = output pitch)
   int act, epi_lrn, out_half;
+  int gather, slab_rows;
   float lrn_alpha_over_n, lrn_beta, lrn_k;
 };
 bool stem_supported(int bn, int f, int c0, int ks, int out_pitch);
-cudaError_t launch_stem_conv(const StemGeom& g, int dt, const CUtensorMap* tmB, const CUtensorMap* tmY0,
-                             const CUtensorMap* tmY1, const float* x, const float* bias, cudaStream_t st);
+cudaError_t launch_stem_conv(const StemGeom& g, int dt, const CUtensorMap* tmA, const CUtensorMap* tmB,
+                             const CUtensorMap* tmY0, const CUtensorMap* tmY1, const float* x, const float* bias, void* Y,
+                             cudaStream_t st);
 
 // --- LRN across channels (K4), NHWC ----------------------------------------------------------
 // Channel c of a pixel is stored at (c/gsz)*gpitch + c%gsz (grouped layouts); pads -> 0.

@@ -822,14 +822,15 @@ void Net::build(const std::string& desc) {
       ops.push_back(lp);
     }
   }
-  // Fused first layer (k_stem.cu): a space-to-depth first conv whose output is a plain
-  // NHWC tensor reads the fp32 images itself; the pack op is then not launched.  Opt-in
-  // (DJINN_STEM=1): correct and bitwise equal to pack + slab GEMM, but measured slower on B200
-  // (IMC conv1+norm1 638 us vs pack 163 + conv1 397 us; its fp32 gather is the bottleneck,
-  // DESIGN.md sec 5).
+  // First-layer kernel (k_stem.cu) for a space-to-depth first conv whose output is a plain NHWC
+  // tensor: resident filter bank, TMA-store epilogue, slab of the packed tensor by TMA (default,
+  // stem = 2).  DJINN_STEM=1: the kernel gathers the fp32 images itself and the pack op is not
+  // launched -- bitwise equal, but measured slower on B200 (its fp32 gather is the bottleneck,
+  // DESIGN.md sec 5).  DJINN_STEM=0: the generic slab GEMM.
   {
     const char* se = getenv("DJINN_STEM");
-    if (f16 && (se && se[0] == '1') && ops.size() > 1 && ops[0].kind == OP_PACK && ops[0].xform == 1 &&
+    const int smode = se ? atoi(se) : 2;
+    if (f16 && smode > 0 && ops.size() > 1 && ops[0].kind == OP_PACK && ops[0].xform == 1 &&
         ops[1].kind == OP_GEMM && ops[1].xform == 1) {
       Op& c = ops[1];
       const GemmGeom& g = c.g;
@@ -840,8 +841,8 @@ void Net::build(const std::string& desc) {
       if (pool_next && g.mode == GM_CONV && g.Z == 1 && g.zf == 1 && g.stride == 1 && g.pad == 0 && g.xb <= 1 &&
           !g.out_f32 && !g.out_half && c.out.gsz >= c.out.C && c.out.bdr == 0 && c.out.Cp == g.N && g.KH == g.KW &&
           g.H - g.OH >= 0 && g.W - g.OW >= 0 && stem_supported(g.N, c.xf, c.orig_in.C, g.KH, c.out.Cp)) {
-        c.stem = 1;
-        ops[0].fused = 1;
+        c.stem = smode == 1 ? 1 : 2;
+        ops[0].fused = smode == 1 ? 1 : 0;
         c.out.hx = ops[2].in.hx = g.H - g.OH;
         c.out.wx = ops[2].in.wx = g.W - g.OW;
       }
@@ -875,7 +876,7 @@ void Net::build(const std::string& desc) {
         else if (g.mode == GM_LC) kreal = (double)o.orig_k * o.orig_k * oin.C;
         else kreal = (double)o.orig_k * o.orig_k * (oin.C / (g.zf > 1 ? g.zf : g.Z));
         o.flops_row = 2.0 * out_e * kreal;
-        o.bytes_row = in_e * (o.stem ? 4.0 : es) + out_e * (g.out_f32 ? 4.0 : es);  // stem: reads the fp32 images
+        o.bytes_row = in_e * (o.stem == 1 ? 4.0 : es) + out_e * (g.out_f32 ? 4.0 : es);  // stem 1 reads the fp32 images
         const double nb = g.mode == GM_DENSE ? g.N : (double)g.Z * g.bias_zstride;
         o.weight_bytes = (g.mode == GM_LC ? (double)g.Z * g.N * kreal
                                           : (g.mode == GM_CONV ? (double)o.out.C * kreal : (double)g.N * kreal)) * es +
@@ -1289,7 +1290,10 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
             sg.N = g.N;
             sg.act = g.act; sg.epi_lrn = g.epi_lrn; sg.out_half = g.out_half;
             sg.lrn_alpha_over_n = g.lrn_alpha_over_n; sg.lrn_beta = g.lrn_beta; sg.lrn_k = g.lrn_k;
-            e = launch_stem_conv(sg, dt, &o.tmB, &w->tmY0[i], &w->tmY1[i], src, (const float*)(ar + o.b_off), st);
+            sg.gather = o.stem == 1;
+            sg.slab_rows = g.slab_rows;
+            e = launch_stem_conv(sg, dt, &w->tmA[i], &o.tmB, &w->tmY0[i], &w->tmY1[i], src, (const float*)(ar + o.b_off),
+                                 Y, st);
           } else if (dt == DT_F32)
             e = launch_simt_gemm(g, (const float*)A, (const float*)(ar + o.w_off), (const float*)(ar + o.b_off),
                                  (float*)Y, st);
@@ -1368,7 +1372,8 @@ std::string Net::plan_string() const {
         << (o.g.lcg > 1 ? " taps/row=" + std::to_string(o.g.lcg) : std::string())
         << (o.g.mode == GM_CONV && o.g.a_tiled ? " block=" + std::to_string(o.g.bx) + "x" + std::to_string(o.g.by) + "x" +
                                                   std::to_string(o.g.bn) : std::string())
-        << (o.stem ? " stem(fp32 input, fused pack, resident B, TMA-store epilogue)" : "")
+        << (o.stem == 1 ? " stem(fp32 input, fused pack, resident B, TMA-store epilogue)" : "")
+        << (o.stem == 2 ? " stem(TMA slab, resident B, TMA-store epilogue)" : "")
         << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << (o.g.out_half ? " fp16-out" : "") << "]";
     if (o.kind == OP_PACK && o.embed) s << " [embedding window " << o.eg.window << " tables " << o.eg.T << " D " << o.eg.D << "]";
     if (o.kind == OP_PACK && o.fused) s << " [fused into the next op]";

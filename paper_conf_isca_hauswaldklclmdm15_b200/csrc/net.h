@@ -78,8 +78,9 @@ struct Op {
   // by xf (= conv stride), 2 kx-unroll of a stride-1 kernel of width xf
   int xform = 0, xf = 1, xs = 1;  // xs: kx-unroll x step (packed pixel j starts at input x = j*xs)
   Shape orig_in;                // the layer's input before the transform
-  // fused first layer (k_stem.cu): the GEMM reads the fp32 input itself (stem = 1) and the
-  // pack op before it is not launched (fused = 1)
+  // first-layer kernel with a resident filter bank (k_stem.cu): stem = 2 reads the packed
+  // space-to-depth tensor by TMA; stem = 1 reads the fp32 input itself and the pack op before
+  // it is not launched (fused = 1)
   int stem = 0, fused = 0;
   // SENNA window lookup in place of the pack (embed = 1): see EmbedGeom (kernels.h)
   int embed = 0;

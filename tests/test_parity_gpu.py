@@ -294,19 +294,21 @@ net.close()
 """
 
 
+@pytest.mark.parametrize("mode", ["1", "2"])
 @pytest.mark.parametrize("prec,n,start", [("fp16", 7, 0), ("bf16", 3, 11), ("fp16", 130, 5)])
-def test_stem_conv_equals_pack_plus_slab_gemm_bitwise(prec, n, start, tmp_path):
-    """IMC conv1+norm1 as the fused first-layer kernel (fp32 images gathered into the
-    space-to-depth slab in shared memory, resident B, TMA-store epilogue) and as the separate
-    pack + slab GEMM (DJINN_STEM=0) give bitwise-equal logits: the same 16-bit operands reach
-    the same MMAs in the same order, and the epilogue arithmetic is the same.  n = 7 / 3 / 130
-    images: tiles that straddle image boundaries and a ragged last tile."""
+def test_stem_conv_equals_pack_plus_slab_gemm_bitwise(mode, prec, n, start, tmp_path):
+    """IMC conv1+norm1 as the first-layer kernel with a resident filter bank and a TMA-store
+    epilogue over the virtual grid -- its slab gathered from the fp32 images (DJINN_STEM=1) or
+    loaded from the packed tensor by TMA (2, the default) -- and as the generic slab GEMM
+    (DJINN_STEM=0) give bitwise-equal logits: the same 16-bit operands reach the same MMAs in
+    the same order, and the epilogue arithmetic is the same.  n = 7 / 3 / 130 images: tiles
+    that straddle image boundaries and a ragged last tile."""
     import os
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     outs, plans = [], []
-    for stem in ("1", "0"):
+    for stem in (mode, "0"):
         f = str(tmp_path / f"lg{stem}.npy")
         env = dict(os.environ, DJINN_STEM=stem)
         r = subprocess.run([sys.executable, "-c", _STEM_CHILD, root, "imc", prec, str(n), f, str(start)], env=env,
