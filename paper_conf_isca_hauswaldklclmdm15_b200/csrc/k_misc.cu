@@ -526,12 +526,12 @@ cudaError_t launch_lrn_pool(const void* x, void* y, int64_t rows, int C, int Cpi
   const float an = alpha / size;
   cudaError_t e;
   if (dt == DT_F16) {
-    e = cudaFuncSetAttribute(lrn_pool_kernel<__half>, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+    e = ensure_max_smem((const void*)lrn_pool_kernel<__half>, 100 * 1024);
     if (e == cudaSuccess)
       e = launch_pdl(lrn_pool_kernel<__half>, g, b, smem, st, (const __half*)x, (__half*)y, C, Cpi, H, W, OH, OW, bands,
                      out_gsz, out_gpitch, Cpo, obd, an, -beta, k);
   } else {
-    e = cudaFuncSetAttribute(lrn_pool_kernel<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+    e = ensure_max_smem((const void*)lrn_pool_kernel<__nv_bfloat16>, 100 * 1024);
     if (e == cudaSuccess)
       e = launch_pdl(lrn_pool_kernel<__nv_bfloat16>, g, b, smem, st, (const __half*)x, (__nv_bfloat16*)y, C, Cpi, H, W,
                      OH, OW, bands, out_gsz, out_gpitch, Cpo, obd, an, -beta, k);

@@ -1,0 +1,359 @@
+// The whole forward pass of a two-layer window MLP (the SENNA-style POS / CHK / NER services,
+// PAPER.md L104 and Table 1; SURVEY 8(a) a2 + a7 + a8) as ONE kernel:
+//     h = act1(x . W1^T + b1),   z = h . W2^T + b2,   p = softmax(z)   (or z / argmax z)
+// for a tile of 128 query rows per CTA.  These nets are launch- and latency-bound, not
+// bandwidth-bound (4096 windows are 5 MB of input: 0.8 us of HBM time): the unfused path is four
+// dependent kernels (pack, l1, l2, softmax) of a few microseconds each ("small
+// networks"; L173 on their low GPU occupancy).  Here every intermediate stays on chip:
+//   1. all 8 warps load the tile's fp32 rows (coalesced), convert them to 16-bit and write the
+//      128B-swizzled K-major A operand of layer 1 into shared memory (pad columns zero);
+//   2. one thread streams W1 through a 4-stage ring of 32-column K blocks (TMA, SWIZZLE_64B) and
+//      issues tcgen05.mma (M = 128, N = N1p split into 256 + the rest) into TMEM columns
+//      [0, N1p); W2 (all of it, K-major SWIZZLE_128B) arrives once at the start;
+//   3. all 8 warps drain layer 1 (bias + activation, 16-bit) straight into layer 2's A operand,
+//      which overwrites layer 1's (consumed) A in shared memory;
+//   4. one thread issues layer 2 into TMEM columns [N1c, N1c + N2p);
+//   5. warps 0-3 (one row per thread) read the logits, add the bias and write the probabilities
+//      (max-subtracted exp, then normalised), the logits or the argmax (ties -> lowest index).
+// Arithmetic per element is the unfused path's: fp32 accumulation of 16-bit products, bias +
+// activation in fp32 rounded once to 16 bits, fp32 logits, expf-based softmax.
+#include "tc_common.cuh"
+#include <cfloat>
+#include <cstdio>
+#ifdef DJINN_MLP_STATS
+#define MST(i) if (tid == 0) ts[i] = clock64()
+#else
+#define MST(i)
+#endif
+
+namespace djinn {
+namespace {
+
+constexpr int MLP_THREADS = 256;
+constexpr int MLP_WSTAGES = 4;            // W1 ring stages
+constexpr int MLP_WK = 32;                // K columns per W1 stage (SWIZZLE_64B rows)
+
+__device__ __forceinline__ uint32_t idesc_rt(int n, bool bf16) {  // kind::f16, D fp32, K-major A/B, M = 128
+  const uint32_t ab = bf16 ? 1u : 0u;
+  return (1u << 4) | (ab << 7) | (ab << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+}
+
+template <bool BF16>
+__global__ void __launch_bounds__(MLP_THREADS, 1)
+    mlp2_kernel(const __grid_constant__ CUtensorMap tmW1, const __grid_constant__ CUtensorMap tmW2, const MlpGeom g,
+                const float* __restrict__ x, const float* __restrict__ b1, const float* __restrict__ b2,
+                void* __restrict__ out) {
+  pdl_trigger();
+#ifdef DJINN_MLP_STATS
+  long long ts[12] = {0};
+  const int tid0 = threadIdx.x;
+  if (tid0 == 0) ts[0] = clock64();
+#endif
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int KB0 = g.K0p / 64, KB1 = g.K1p / 64;  // 64-column blocks of the two A operands
+  const int abytes = (KB0 > KB1 ? KB0 : KB1) * 128 * 128;
+  const int wstage = g.N1p * MLP_WK * 2;          // one W1 ring stage (N1p rows of 64 B)
+  uint8_t* sA = smem;                             // A1, then A2
+  uint8_t* sW = sA + abytes;                      // W1 ring
+  uint8_t* sW2 = sW + ((MLP_WSTAGES * wstage + 1023) & ~1023);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sW2 + KB1 * g.N2p * 128);
+  // bars: w2full, wfull[4], wempty[4], d1full, d2full
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 11);
+  __shared__ __align__(16) float sb1[512];
+  __shared__ __align__(16) float sb2[256];
+  const uint32_t w2full = smem_u32(bars), wfull0 = smem_u32(bars + 1), wempty0 = smem_u32(bars + 5);
+  const uint32_t d1full = smem_u32(bars + 9), d2full = smem_u32(bars + 10);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, tid = threadIdx.x;
+  const int64_t row0 = (int64_t)blockIdx.x * 128;
+  const int nrows = (int)(g.rows - row0 < 128 ? g.rows - row0 : 128);
+  const int nkw = g.K0p / MLP_WK;  // W1 ring blocks
+
+  if (tid == 0) {
+    mbar_init(w2full, 1);
+    for (int s = 0; s < MLP_WSTAGES; ++s) {
+      mbar_init(wfull0 + 8 * s, 1);
+      mbar_init(wempty0 + 8 * s, 1);
+    }
+    mbar_init(d1full, 1);
+    mbar_init(d2full, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    fence_proxy_async();
+  }
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)), "r"(512u)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  for (int c = tid; c < 512; c += MLP_THREADS) sb1[c] = c < g.N1 ? __ldg(b1 + c) : 0.f;
+  for (int c = tid; c < 256; c += MLP_THREADS) sb2[c] = c < g.N2 ? __ldg(b2 + c) : 0.f;
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  // weights: W2 whole, and the first ring stages of W1 (never written by earlier kernels)
+  auto load_w1 = [&](int kb) {
+    const int s = kb % MLP_WSTAGES;
+    const uint32_t dst = smem_u32(sW) + (uint32_t)(s * wstage);
+    mbar_arrive_expect_tx(wfull0 + 8 * s, (uint32_t)wstage);
+    const int half = g.N1p / 2;  // two boxes of N1p / 2 rows
+    tma_2d(dst, &tmW1, wfull0 + 8 * s, kb * MLP_WK, 0);
+    tma_2d(dst + (uint32_t)(half * MLP_WK * 2), &tmW1, wfull0 + 8 * s, kb * MLP_WK, half);
+  };
+  if (tid == 0) {
+    mbar_arrive_expect_tx(w2full, (uint32_t)(KB1 * g.N2p * 128));
+    for (int kb = 0; kb < KB1; ++kb) tma_2d(smem_u32(sW2) + (uint32_t)(kb * g.N2p * 128), &tmW2, w2full, kb * 64, 0);
+    for (int kb = 0; kb < MLP_WSTAGES && kb < nkw; ++kb) load_w1(kb);
+  }
+  MST(1);
+  pdl_wait();  // the input rows and the output buffer belong to earlier kernels of the stream
+  MST(2);
+
+  // ---- 1. fp32 rows -> 16-bit A1 (K-major, 128B swizzle: element (r, k) of block k / 64 at
+  // r * 128 + (((k % 64) / 8) ^ (r % 8)) * 16 + (k % 8) * 2); a warp reads one row's floats
+  // contiguously, so the global reads are coalesced
+  {
+    // 4 rows per warp iteration with all their loads in flight before any is used (a row at a
+    // time serialised ~80 L2 round trips per warp: 12.5 us of the kernel's 29 us, B200)
+    constexpr int RB = 4, KMAX = 384 / 64;  // rows per batch; lane pairs per row (K0p <= 384)
+    for (int rb = warp * RB; rb < 128; rb += (MLP_THREADS / 32) * RB) {
+      float v[RB][KMAX][2];
+#pragma unroll
+      for (int i = 0; i < RB; ++i) {
+        const int r = rb + i;
+        const float* xr = x + (row0 + r) * (int64_t)g.K0;
+#pragma unroll
+        for (int j = 0; j < KMAX; ++j) {
+          const int k = lane * 2 + 64 * j;
+          v[i][j][0] = (r < nrows && k < g.K0) ? __ldg(xr + k) : 0.f;
+          v[i][j][1] = (r < nrows && k + 1 < g.K0) ? __ldg(xr + k + 1) : 0.f;
+        }
+      }
+#pragma unroll
+      for (int i = 0; i < RB; ++i) {
+        const int r = rb + i;
+#pragma unroll
+        for (int j = 0; j < KMAX; ++j) {
+          const int k = lane * 2 + 64 * j;
+          if (k < g.K0p) {
+            const int kk = k & 63;
+            const uint32_t off = (uint32_t)((k >> 6) * (128 * 128) + r * 128 + (((kk >> 3) ^ (r & 7)) << 4) + (kk & 7) * 2);
+            *reinterpret_cast<uint32_t*>(sA + off) = pack2<BF16>(v[i][j][0], v[i][j][1]);
+          }
+        }
+      }
+    }
+  }
+  fence_proxy_async();
+  __syncthreads();
+  MST(3);
+
+  const uint64_t hi128 = sdesc(0, 128), hi64 = sdesc(0, 64);
+  const bool bf = BF16;
+  // ---- 2. layer 1 MMAs (thread 0): K steps of 16 over the W1 ring
+  if (tid == 0) {
+    const int na = g.N1p > 256 ? 256 : g.N1p, nb = g.N1p - na;
+    const uint32_t ida = idesc_rt(na, bf), idb = nb ? idesc_rt(nb, bf) : 0u;
+    const uint32_t a16 = (smem_u32(sA) & 0x3FFFFu) >> 4, w16 = (smem_u32(sW) & 0x3FFFFu) >> 4;
+    for (int kb = 0; kb < nkw; ++kb) {
+      const int s = kb % MLP_WSTAGES;
+      mbar_wait(wfull0 + 8 * s, (uint32_t)(kb / MLP_WSTAGES) & 1);
+      tc_fence_after();
+#pragma unroll
+      for (int k = 0; k < MLP_WK / 16; ++k) {
+        const int kk = kb * MLP_WK + k * 16;  // first K column of this step
+        const uint64_t ad = hi128 | (uint64_t)(a16 + (uint32_t)((kk >> 6) * (128 * 128 / 16) + ((kk & 63) * 2) / 16));
+        const uint32_t wb = w16 + (uint32_t)(s * (wstage >> 4)) + (uint32_t)(k * 2);
+        mma_f16(tmem, ad, hi64 | (uint64_t)wb, ida, (kb | k) != 0);
+        if (nb) mma_f16(tmem + (uint32_t)na, ad, hi64 | (uint64_t)(wb + (uint32_t)((na * 64) >> 4)), idb, (kb | k) != 0);
+      }
+      mma_commit(wempty0 + 8 * s);
+    }
+    mma_commit(d1full);
+  } else if (tid == 32) {
+    // W1 ring refills: stage kb % S is reloaded with block kb + S once its MMAs have completed
+    for (int kb = 0; kb + MLP_WSTAGES < nkw; ++kb) {
+      mbar_wait(wempty0 + 8 * (kb % MLP_WSTAGES), (uint32_t)(kb / MLP_WSTAGES) & 1);
+      load_w1(kb + MLP_WSTAGES);
+    }
+  }
+  MST(4);
+  __syncwarp();
+
+  // ---- 3. layer 1 epilogue -> A2 (overwrites A1; its MMAs have completed)
+  {
+    if (lane == 0) mbar_wait(d1full, 0);
+    __syncwarp();
+    tc_fence_after();
+    const int quarter = warp & 3, half = warp >> 2;
+    const int r = quarter * 32 + lane;
+    const uint32_t tb = tmem + ((uint32_t)(quarter * 32) << 16);
+    const int nch = g.N1p / 16, c0 = half ? (nch + 1) / 2 : 0, c1 = half ? nch : (nch + 1) / 2;
+    uint8_t* a2 = sA;
+    // chunk ci: bias + activation -> 16-bit -> A2 (two 16-byte pieces)
+    auto emit = [&](int ci, const uint32_t (&rq)[16]) {
+      float bq[16], v[16];
+      lds16(bq, sb1 + ci * 16);
+      bias_act16(v, rq, bq, g.act1);
+      const int k = ci * 16;
+#pragma unroll
+      for (int j = 0; j < 16; ++j) v[j] = k + j < g.N1 ? v[j] : 0.f;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int kk = (k + 8 * h) & 63;
+        const uint32_t off = (uint32_t)(((k + 8 * h) >> 6) * (128 * 128) + r * 128 + (((kk >> 3) ^ (r & 7)) << 4));
+        *reinterpret_cast<uint4*>(a2 + off) =
+            make_uint4(pack2<BF16>(v[8 * h], v[8 * h + 1]), pack2<BF16>(v[8 * h + 2], v[8 * h + 3]),
+                       pack2<BF16>(v[8 * h + 4], v[8 * h + 5]), pack2<BF16>(v[8 * h + 6], v[8 * h + 7]));
+      }
+    };
+    // two chunks per step: the second one's TMEM load is in flight while the first is converted
+    for (int ci = c0; ci < c1; ci += 2) {
+      uint32_t ra[16], rb2[16];
+      tmem_ld16(tb + (uint32_t)(ci * 16), ra);
+      if (ci + 1 < c1) tmem_ld16(tb + (uint32_t)((ci + 1) * 16), rb2);
+      tmem_wait_ld();
+      emit(ci, ra);
+      if (ci + 1 < c1) emit(ci + 1, rb2);
+    }
+    // zero K columns [N1p, K1p) of A2 (W2 is zero there too; 0 * garbage could be NaN)
+    for (int k = g.N1p + 8 * half; k < g.K1p; k += 16) {
+      const int kk = k & 63;
+      *reinterpret_cast<uint4*>(a2 + (k >> 6) * (128 * 128) + r * 128 + (((kk >> 3) ^ (r & 7)) << 4)) = make_uint4(0, 0, 0, 0);
+    }
+  }
+  tc_fence_before();
+  fence_proxy_async();
+  __syncthreads();
+  MST(5);
+
+  // ---- 4. layer 2 MMAs (thread 0) into columns [N1c, N1c + N2p)
+  const uint32_t d2 = tmem + (uint32_t)g.N1c;
+  if (tid == 0) {
+    tc_fence_after();
+    mbar_wait(w2full, 0);
+    const uint32_t id2 = idesc_rt(g.N2p, bf);
+    const uint32_t a16 = (smem_u32(sA) & 0x3FFFFu) >> 4, w16 = (smem_u32(sW2) & 0x3FFFFu) >> 4;
+    for (int k = 0; k < g.K1p; k += 16) {
+      const uint64_t ad = hi128 | (uint64_t)(a16 + (uint32_t)((k >> 6) * (128 * 128 / 16) + ((k & 63) * 2) / 16));
+      const uint64_t bd = hi128 | (uint64_t)(w16 + (uint32_t)((k >> 6) * (g.N2p * 128 / 16) + ((k & 63) * 2) / 16));
+      mma_f16(d2, ad, bd, id2, k != 0);
+    }
+    mma_commit(d2full);
+  }
+  MST(8);
+  __syncwarp();
+
+  // ---- 5. logits (+ bias) -> shared memory (warps 0-3 own the TMEM lanes: one row each), then
+  // every warp takes rows: lanes over the row's N2 <= 64 columns, max / sum by shuffles, and
+  // coalesced stores of the probabilities / logits; argmax ties -> lowest index
+  float* stg = reinterpret_cast<float*>(sA);  // A's space: layer 2's MMAs have completed
+  const int N2 = g.N2, sp = N2 + 1;           // odd pitch: conflict-free column writes
+  if (warp < 4) {
+    if (lane == 0) mbar_wait(d2full, 0);
+    __syncwarp();
+    MST(9);
+    tc_fence_after();
+    const int r = warp * 32 + lane;
+    const uint32_t tb = d2 + ((uint32_t)(warp * 32) << 16);
+    const int nch = g.N2p / 16;
+    uint32_t rq[4][16];
+#pragma unroll
+    for (int ci = 0; ci < 4; ++ci)
+      if (ci < nch) tmem_ld16(tb + (uint32_t)(ci * 16), rq[ci]);  // all chunks in flight, one wait
+    tmem_wait_ld();
+#pragma unroll
+    for (int ci = 0; ci < 4; ++ci)
+      if (ci < nch) {
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+          const int c = ci * 16 + j;
+          if (c < N2) stg[r * sp + c] = __uint_as_float(rq[ci][j]) + sb2[c];
+        }
+      }
+  }
+  __syncthreads();
+  MST(10);
+  // two threads per row (interleaved columns) for the max / exp / sum, in place in shared memory
+  {
+    const int r = tid >> 1, h = tid & 1;
+    float* zr = stg + r * sp;
+    float m = -FLT_MAX;
+    int mi = 0x7fffffff;
+    for (int c = h; c < N2; c += 2) {
+      const float v = zr[c];
+      if (v > m || (v == m && c < mi)) { m = v; mi = c; }
+    }
+    const float m2 = __shfl_xor_sync(0xffffffffu, m, 1);
+    const int i2 = __shfl_xor_sync(0xffffffffu, mi, 1);
+    if (m2 > m || (m2 == m && i2 < mi)) { m = m2; mi = i2; }
+    if (g.out_mode == 1) {
+      if (h == 0 && r < nrows) reinterpret_cast<int*>(out)[row0 + r] = mi;
+    } else if (g.out_mode == 0) {
+      float sum = 0.f;
+      for (int c = h; c < N2; c += 2) {
+        const float e = expf(zr[c] - m);
+        zr[c] = e;
+        sum += e;
+      }
+      sum += __shfl_xor_sync(0xffffffffu, sum, 1);
+      const float inv = 1.f / sum;
+      for (int c = h; c < N2; c += 2) zr[c] *= inv;
+    }
+  }
+  if (g.out_mode != 1) {
+    __syncthreads();
+    // coalesced stores: a warp writes whole rows (lanes over columns)
+    for (int r = warp; r < nrows; r += MLP_THREADS / 32) {
+      float* o = reinterpret_cast<float*>(out) + (row0 + r) * N2;
+      for (int c = lane; c < N2; c += 32) o[c] = stg[r * sp + c];
+    }
+  }
+  MST(6);
+  tc_fence_before();
+  __syncthreads();
+  MST(7);
+#ifdef DJINN_MLP_STATS
+  if (tid == 0 && blockIdx.x == 0)
+    printf("[mlp] prologue %lld pdlwait %lld load %lld l1mma %lld l1epi %lld l2issue %lld d2wait %lld logits %lld softmax %lld tail %lld\n",
+           ts[1] - ts[0], ts[2] - ts[1], ts[3] - ts[2], ts[4] - ts[3], ts[5] - ts[4], ts[8] - ts[5], ts[9] - ts[8],
+           ts[10] - ts[9], ts[6] - ts[10], ts[7] - ts[6]);
+#endif
+  if (warp == 0) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512u) : "memory");
+  }
+}
+
+}  // namespace
+
+int mlp2_smem(const MlpGeom& g) {
+  const int KB0 = g.K0p / 64, KB1 = g.K1p / 64;
+  const int abytes = (KB0 > KB1 ? KB0 : KB1) * 128 * 128;
+  return 1024 + abytes + ((MLP_WSTAGES * g.N1p * MLP_WK * 2 + 1023) & ~1023) + KB1 * g.N2p * 128 + 12 * 8 + 16;
+}
+
+bool mlp2_supported(const MlpGeom& g) {
+  return g.K0p % 64 == 0 && g.K1p % 64 == 0 && g.N1p % 16 == 0 && g.N1p >= g.N1 && g.N1p <= 512 &&
+         (g.N1p <= 256 || (g.N1p - 256) % 16 == 0) && g.N1p / 2 <= 256 && g.K1p >= g.N1p && g.N2p % 16 == 0 &&
+         g.N2p >= g.N2 && g.N2p <= 64 && g.N1c % 16 == 0 && g.N1c >= g.N1p && g.N1c + g.N2p <= 512 &&
+         mlp2_smem(g) <= 227 * 1024 - 3 * 1024;
+}
+
+cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const CUtensorMap* tmW2, const float* x,
+                        const float* b1, const float* b2, void* out, cudaStream_t st) {
+  if (g.rows <= 0) return cudaSuccess;
+  if (!mlp2_supported(g)) return cudaErrorInvalidValue;
+  const int smem = mlp2_smem(g);
+  const unsigned grid = (unsigned)((g.rows + 127) / 128);
+  // the max-dynamic-smem attribute is set once per (device, kernel): a cudaFuncSetAttribute per
+  // call was a measurable part of the ~10 us host cost of a small service's forward
+  cudaError_t e = ensure_max_smem(dt == DT_BF16 ? (const void*)mlp2_kernel<true> : (const void*)mlp2_kernel<false>,
+                                  227 * 1024 - 3 * 1024);
+  if (e != cudaSuccess) return e;
+  if (dt == DT_BF16)
+    return launch_pdl(mlp2_kernel<true>, dim3(grid), dim3(MLP_THREADS), smem, st, *tmW1, *tmW2, g, x, b1, b2, out);
+  return launch_pdl(mlp2_kernel<false>, dim3(grid), dim3(MLP_THREADS), smem, st, *tmW1, *tmW2, g, x, b1, b2, out);
+}
+
+}  // namespace djinn

@@ -423,7 +423,7 @@ cudaError_t launch_stem_inst(const StemGeom& g, const CUtensorMap* tmA, const CU
   auto kern = stem_conv_kernel<BN, BF16, F, C0, KS, GATHER>;
   constexpr int smem = stem_smem<BN, KS, GATHER>();
   static_assert(smem <= 227 * 1024 - BN * 4, "stem kernel shared memory");
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaError_t e = ensure_max_smem((const void*)kern, smem);
   if (e != cudaSuccess) return e;
   const int64_t tiles = ((int64_t)g.Nimg * g.Hs * g.Ws + 127) / 128;
   const int grid = (int)(tiles < tc_num_sms() ? tiles : tc_num_sms());

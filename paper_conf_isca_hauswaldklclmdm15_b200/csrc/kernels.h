@@ -42,6 +42,8 @@ __device__ __forceinline__ float2 add2(float2 a, float2 b) {
 }
 #endif
 bool pdl_enabled();
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize, bytes) once per (device, kernel, bytes)
+cudaError_t ensure_max_smem(const void* kernel, int bytes);
 template <typename... KArgs, typename... Args>
 cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args&&... args) {
   cudaLaunchConfig_t cfg = {};
@@ -196,6 +198,24 @@ bool stem_supported(int bn, int f, int c0, int ks, int out_pitch);
 cudaError_t launch_stem_conv(const StemGeom& g, int dt, const CUtensorMap* tmA, const CUtensorMap* tmB,
                              const CUtensorMap* tmY0, const CUtensorMap* tmY1, const float* x, const float* bias, void* Y,
                              cudaStream_t st);
+
+// --- fused two-layer MLP + softmax (k_mlp.cu; the SENNA window nets): fp32 rows x [rows][K0]
+// -> h = act1(x W1^T + b1) (N1) -> z = h W2^T + b2 (N2) -> out (mode 0 prob fp32 [rows][N2],
+// 1 argmax int32 [rows], 2 logits fp32 [rows][N2]).  W1 / W2 are the arena's [N][Kpad] 16-bit
+// matrices; tmW1: 2D {K0p, N1}, box {32, N1p / 2}, SWIZZLE_64B; tmW2: 2D {K1p, N2}, box {64, N2p},
+// SWIZZLE_128B.
+struct MlpGeom {
+  int64_t rows;
+  int K0, K0p;         // input row length, padded to 64 (W1's Kpad)
+  int N1, N1p, N1c;    // layer 1 outputs, padded to 16; TMEM column of layer 2's accumulator
+  int K1p;             // W2's Kpad (layer 1 outputs padded to 64)
+  int N2, N2p;         // logits, padded to 16 (<= 64)
+  int act1, out_mode;
+};
+int mlp2_smem(const MlpGeom& g);
+bool mlp2_supported(const MlpGeom& g);
+cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const CUtensorMap* tmW2, const float* x,
+                        const float* b1, const float* b2, void* out, cudaStream_t st);
 
 // --- LRN across channels (K4), NHWC ----------------------------------------------------------
 // Channel c of a pixel is stored at (c/gsz)*gpitch + c%gsz (grouped layouts); pads -> 0.

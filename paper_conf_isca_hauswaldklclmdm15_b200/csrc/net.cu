@@ -11,6 +11,8 @@
 
 #include <algorithm>
 #include <atomic>
+#include <chrono>
+#include <cstdio>
 #include <cctype>
 #include <sstream>
 
@@ -158,6 +160,51 @@ bool pdl_enabled() {
     return !(e && e[0] == '0');
   }();
   return on;
+}
+
+// DJINN_HOST_PROF=1: host-side microseconds spent enqueueing each op (printed at exit) -- the
+// small services are bound by the host's launch path, not the GPU (tools/host_overhead.py).
+bool host_prof_on() {
+  static const bool on = [] {
+    const char* e = getenv("DJINN_HOST_PROF");
+    return e && e[0] == '1';
+  }();
+  return on;
+}
+namespace {
+struct HostProf {
+  std::mutex mu;
+  std::map<std::string, std::pair<double, long>> acc;
+  ~HostProf() {
+    for (auto& kv : acc) fprintf(stderr, "[djinn host] %-28s %9.2f us/call over %ld calls\n", kv.first.c_str(),
+                                 kv.second.first / kv.second.second, kv.second.second);
+  }
+};
+HostProf& host_prof() {
+  static HostProf h;
+  return h;
+}
+}  // namespace
+void host_prof_add(const std::string& key, double us) {
+  HostProf& h = host_prof();
+  std::lock_guard<std::mutex> lk(h.mu);
+  auto& a = h.acc[key];
+  a.first += us;
+  a.second += 1;
+}
+
+cudaError_t ensure_max_smem(const void* kernel, int bytes) {
+  static std::mutex mu;
+  static std::map<std::pair<int, const void*>, int> done;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  std::lock_guard<std::mutex> lk(mu);
+  int& have = done[{dev, kernel}];
+  if (have >= bytes) return cudaSuccess;
+  e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e == cudaSuccess) have = bytes;
+  return e;
 }
 
 std::atomic<int64_t>& launch_counter() {
@@ -848,6 +895,30 @@ void Net::build(const std::string& desc) {
       }
     }
   }
+  // Two-layer window MLP nets (pack -> dense -> dense -> softmax: POS / CHK / NER) run as one
+  // kernel (k_mlp.cu).  DJINN_MLP=0 keeps the four separate kernels.
+  {
+    const char* me = getenv("DJINN_MLP");
+    if (f16 && !(me && me[0] == '0') && ops.size() == 4 && ops[0].kind == OP_PACK && !ops[0].embed && !ops[0].xform &&
+        ops[1].kind == OP_GEMM && ops[1].g.mode == GM_DENSE && ops[2].kind == OP_GEMM && ops[2].g.mode == GM_DENSE &&
+        ops[2].g.out_f32 && ops[3].kind == OP_SOFTMAX) {
+      MlpGeom m{};
+      m.K0 = ops[0].in.C * ops[0].in.H * ops[0].in.W;
+      m.K0p = ops[1].g.Kpad;
+      m.N1 = ops[1].g.N;
+      m.N1p = rup(m.N1, 16);
+      m.N1c = m.N1p;
+      m.K1p = ops[2].g.Kpad;
+      m.N2 = ops[2].g.N;
+      m.N2p = rup(m.N2, 16);
+      m.act1 = ops[1].g.act;
+      if (ops[0].out.Cp == ops[1].g.K && m.K0 <= ops[0].out.Cp && ops[1].out.Cp <= m.K1p && mlp2_supported(m)) {
+        ops[1].mlp = 1;
+        ops[1].mg = m;
+        ops[0].fused = ops[2].fused = ops[3].fused = 1;
+      }
+    }
+  }
   out_elems = cur.C;
   arena_bytes = rupz(arena_off, 1024);
   // Centered sigmoid storage on 16-bit paths: a sigmoid layer feeding a dense layer stores
@@ -1260,6 +1331,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
       cudaError_t e = cudaSuccess;
       bool skipped = false;
       if (prof && (pop < 0 || pop == (int)i)) ck(cudaEventRecord(pev[pop < 0 ? i : 0], st), "profile event");
+      const auto th0 = host_prof_on() ? std::chrono::steady_clock::now() : std::chrono::steady_clock::time_point();
       switch (o.kind) {
         case OP_PACK:
           if (o.fused) { skipped = true; break; }  // the stem GEMM reads the fp32 rows itself
@@ -1271,6 +1343,16 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
                                 dt, st);
           break;
         case OP_GEMM: {
+          if (o.fused) { skipped = true; break; }
+          if (o.mlp) {
+            MlpGeom mg = o.mg;
+            mg.rows = n;
+            mg.out_mode = mode;
+            const uint8_t* ar = (const uint8_t*)arena;
+            e = launch_mlp2(mg, dt, &o.tmW1, &o.tmW2, src, (const float*)(ar + o.b_off), (const float*)(ar + ops[i + 1].b_off),
+                            dst, st);
+            break;
+          }
           GemmGeom g = o.g;
           g.ldwait = ldwait_mode();
           g.tslots = tslots_mode();
@@ -1321,9 +1403,12 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
                               o.beta, o.lrn_k, dt, st);
           break;
         case OP_SOFTMAX:
+          if (o.fused) { skipped = true; break; }
           e = launch_softmax((const float*)w->buf[2], n, (int)out_elems, out_pitch, dst, mode, st);
           break;
       }
+      if (host_prof_on())
+        host_prof_add(name + "/" + o.name, std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - th0).count());
       if (!skipped) ++launches;
       if (e != cudaSuccess) {
         poisoned = true;
@@ -1376,7 +1461,9 @@ std::string Net::plan_string() const {
         << (o.stem == 2 ? " stem(TMA slab, resident B, TMA-store epilogue)" : "")
         << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << (o.g.out_half ? " fp16-out" : "") << "]";
     if (o.kind == OP_PACK && o.embed) s << " [embedding window " << o.eg.window << " tables " << o.eg.T << " D " << o.eg.D << "]";
-    if (o.kind == OP_PACK && o.fused) s << " [fused into the next op]";
+    if (o.kind != OP_GEMM && o.fused) s << " [fused]";
+    if (o.kind == OP_GEMM && o.fused) s << " [fused into the MLP kernel]";
+    if (o.mlp) s << " [MLP kernel: whole net in one launch, N1p=" << o.mg.N1p << " K0p=" << o.mg.K0p << " N2p=" << o.mg.N2p << "]";
     if (o.kind == OP_PACK && o.xform) s << " [" << (o.xform == 1 ? "space-to-depth " : "kx-unroll ") << o.xf << (o.xs > 1 ? " step " + std::to_string(o.xs) : std::string()) << "]";
     s << "\n";
   }

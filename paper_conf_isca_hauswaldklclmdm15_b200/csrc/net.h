@@ -82,6 +82,11 @@ struct Op {
   // space-to-depth tensor by TMA; stem = 1 reads the fp32 input itself and the pack op before
   // it is not launched (fused = 1)
   int stem = 0, fused = 0;
+  // fused two-layer MLP + softmax (k_mlp.cu): this GEMM op runs the whole net (mlp = 1); the
+  // pack, the second GEMM and the softmax ops are not launched (fused = 1)
+  int mlp = 0;
+  MlpGeom mg{};
+  CUtensorMap tmW1{}, tmW2{};
   // SENNA window lookup in place of the pack (embed = 1): see EmbedGeom (kernels.h)
   int embed = 0;
   EmbedGeom eg{};
@@ -155,6 +160,8 @@ struct Net {
 };
 
 std::atomic<int64_t>& launch_counter();
+bool host_prof_on();
+void host_prof_add(const std::string& key, double us);
 void encode_tmap(CUtensorMap* m, int dt, const void* base, int rank, const uint64_t* dims,
                  const uint64_t* strides_bytes, const uint32_t* box, int swizzle_bytes = 128,
                  const uint32_t* elem_strides = nullptr);

@@ -317,3 +317,46 @@ def test_stem_conv_equals_pack_plus_slab_gemm_bitwise(mode, prec, n, start, tmp_
         outs.append(np.load(f))
     assert "stem(" in plans[0] and "stem(" not in plans[1], plans
     assert np.array_equal(outs[0], outs[1])
+
+
+# ---------------------------------------------------------------- fused window MLP (k_mlp.cu)
+_MLP_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+sys.path.insert(0, sys.argv[1] + "/tests")
+import paper_conf_isca_hauswaldklclmdm15_b200 as dj
+from datagen import recipes
+from parity import blob
+app, prec, n = sys.argv[2], sys.argv[3], int(sys.argv[4])
+x = torch.from_numpy(recipes.gen_input_rows(app, 0, n, prec)).cuda()
+net = dj.DjinnNet(dj.net_description(app), blob(app, prec), prec, n)
+print(net.plan())
+outs = [net.forward(x, m).cpu().numpy() for m in (dj.DJINN_OUT_LOGITS, dj.DJINN_OUT_PROB, dj.DJINN_OUT_ARGMAX)]
+np.savez(sys.argv[5], lg=outs[0], pr=outs[1], am=outs[2])
+net.close()
+"""
+
+
+@pytest.mark.parametrize("app,prec,n", [("pos", "fp16", 1000), ("chk", "bf16", 4096), ("ner", "fp16", 129),
+                                        ("ner", "bf16", 3000)])
+def test_mlp_kernel_equals_unfused_path(app, prec, n, tmp_path):
+    """The one-launch window-MLP kernel (pack + l1 + HardTanh + l2 + softmax on chip) and the four
+    separate kernels (DJINN_MLP=0) give bitwise-equal logits and argmax -- the same 16-bit
+    operands reach the MMAs in the same K order and the epilogues round the same way -- and
+    probabilities equal to the last ulps (the softmax sums in a different order)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    res, plans = [], []
+    for mlp in ("1", "0"):
+        f = str(tmp_path / f"o{mlp}.npz")
+        env = dict(os.environ, DJINN_MLP=mlp)
+        r = subprocess.run([sys.executable, "-c", _MLP_CHILD, root, app, prec, str(n), f], env=env, check=True,
+                           timeout=600, capture_output=True, text=True)
+        plans.append(r.stdout)
+        res.append(np.load(f))
+    assert "MLP kernel" in plans[0] and "MLP kernel" not in plans[1], plans
+    assert np.array_equal(res[0]["lg"], res[1]["lg"])
+    assert np.array_equal(res[0]["am"], res[1]["am"])
+    np.testing.assert_allclose(res[0]["pr"], res[1]["pr"], rtol=2e-6, atol=1e-7)
