@@ -542,6 +542,66 @@ def main():
                     "dtype": "f32"}
         n2.close()
 
+    # ---- serving curves (Figs. 7-9):
+    # (1) the native query batcher under closed-loop load -- clients = 2 x the batch size in
+    #     queries, each submitting one query and waiting for it -- per maximum batch size:
+    #     throughput and query latency p50 / p99 (the latency-vs-batch trade-off of Fig. 7c);
+    # (2) concurrent services: T host threads, each with its own stream, each running the
+    #     mixed step -- aggregate q/s and per-step device latency vs T (Figs. 8-9).
+    serving = None
+    if not args.no_sweep:
+        serving = {"batcher": {}, "concurrency": []}
+        for app, qbatches in (("imc", [1, 16, 64, 256]), ("pos", [1, 16, 64, 146])):
+            if app not in apps:
+                continue
+            rpq = ROWS_PER_QUERY[app]
+            pool = inputs[app][: min(BATCH_ROWS[app], 256 * rpq)].cpu().numpy().reshape(-1, nets[app].in_elems)
+            res = []
+            for qb in qbatches:
+                n2 = clone_net(app, qb * rpq)
+                bt = dj.DjinnBatcher(n2, qb * rpq, max_wait_us=200)
+                r = bt.drive(pool, rpq, clients=min(2 * qb, 512), seconds=0.4)
+                st_ = bt.stats()
+                bt.close()
+                n2.close()
+                res.append({"max_batch_queries": qb, "clients": min(2 * qb, 512), **r,
+                            "mean_batch_queries": st_["queries"] / max(1, st_["batches"])})
+            serving["batcher"][app] = res
+        import threading
+        for T in (1, 2, 4):
+            streams = [torch.cuda.Stream() for _ in range(T)]
+            outs_t = [{a: torch.empty_like(outputs[a]) for a in apps} for _ in range(T)]
+            ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(3)]
+                  for _ in range(T)]
+
+            def service_thread(t):
+                for k in range(3):
+                    ev[t][k][0].record(streams[t])
+                    for a in apps:
+                        dj.djinn_forward(nets[a].handle, inputs[a], BATCH_ROWS[a], outs_t[t][a], dj.DJINN_OUT_PROB,
+                                         streams[t].cuda_stream)
+                    ev[t][k][1].record(streams[t])
+            for t in range(T):  # warm the per-stream workspaces
+                for a in apps:
+                    dj.djinn_forward(nets[a].handle, inputs[a], BATCH_ROWS[a], outs_t[t][a], dj.DJINN_OUT_PROB,
+                                     streams[t].cuda_stream)
+            torch.cuda.synchronize()
+            gate = torch.cuda.Event(enable_timing=True)
+            gate.record(stream)  # every service stream starts after this event
+            for t in range(T):
+                streams[t].wait_event(gate)
+            th = [threading.Thread(target=service_thread, args=(t,)) for t in range(T)]
+            for x_ in th:
+                x_.start()
+            for x_ in th:
+                x_.join()
+            torch.cuda.synchronize()
+            span = max(gate.elapsed_time(ev[t][2][1]) for t in range(T))
+            lat = [ev[t][k][0].elapsed_time(ev[t][k][1]) for t in range(T) for k in range(3)]
+            q = sum(BATCH_ROWS[a] / ROWS_PER_QUERY[a] for a in apps)
+            serving["concurrency"].append({"threads": T, "queries_per_s": T * 3 * q / (span / 1e3),
+                                           "step_latency_ms_mean": sum(lat) / len(lat), "step_latency_ms_max": max(lat)})
+
     # ---- e2e: public API with pinned HOST buffers (H2D + D2H inside the timed region)
     e2e = e2e16 = None
     if not args.no_e2e:
@@ -653,7 +713,7 @@ def main():
                            "services": "serial (one stream, PDL-chained); see concurrent_services",
                            "host_fed_pipe_chunks": os.environ.get("DJINN_PIPE_CHUNKS", "auto (<=4 by copy size)")},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "table3": table3, "sweep": sweep,
-                "face_strong": face_strong, "dig_fp32": dig_fp32, "e2e_16bit_inputs": e2e16, "concurrent_services": conc, "nlp_token_ids": ids,
+                "face_strong": face_strong, "dig_fp32": dig_fp32, "serving": serving, "e2e_16bit_inputs": e2e16, "concurrent_services": conc, "nlp_token_ids": ids,
                 "gpu_launches": int(launches),
                 "clocks": clk.summary(), "per_app": per_app,
                 "top_ops": [{k: o[k] for k in ("app", "op", "kind", "ms_total", "avg_us", "tflops", "gbs", "bound",

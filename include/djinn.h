@@ -216,6 +216,46 @@ DJINN_API const char* djinn_last_error(void);
  * since load (for the bench's gpu_launches claim). */
 DJINN_API int64_t djinn_kernel_launches(void);
 
+/* ------------------------------------------------------------------ query batcher
+ * The service's batching (sec 5.1: "stacking multiple inputs into a larger
+ * matrix ... increases the dimensions of the matrix multiplication"; Table 3 L153-161 batches
+ * queries of an application): a per-net queue in front of djinn_forward.  Clients submit whole
+ * queries (any number of rows) from any thread; a worker thread stacks pending queries into one
+ * batch of at most max_batch_rows rows and runs it as one djinn_forward (pinned host staging,
+ * the library's own stream) when the batch is full or its oldest query has waited max_wait_us,
+ * then copies each query's output rows back.  While one batch runs on the GPU the next one
+ * fills (two staging buffers).
+ *
+ * Ownership: `input` is copied at submit; `output` (host memory of rows x the out_mode's row
+ * size, see djinn_forward) must stay valid until the query's djinn_batcher_wait returned.  The
+ * net must outlive the batcher; the batcher uses its own CUDA stream of the net's device.
+ * Tickets are positive and complete in submission order.  A forward error fails every query
+ * of that batch (their wait returns the error) and the batcher stays usable. */
+typedef struct djinn_batcher djinn_batcher;
+
+/* max_batch_rows in [1, the net's max_rows]; max_wait_us >= 0 (0: run whatever is pending as
+ * soon as the worker is free). */
+DJINN_API int djinn_batcher_create(djinn_net* net, int64_t max_batch_rows, int64_t max_wait_us, int out_mode,
+                                   djinn_batcher** out);
+/* Queue one query of `rows` rows (1 <= rows <= max_batch_rows) of fp32 host input; blocks only
+ * while both staging buffers are busy.  *ticket receives the query's ticket. */
+DJINN_API int djinn_batcher_submit(djinn_batcher* b, const float* input, int64_t rows, void* output, int64_t* ticket);
+/* Wait until the query `ticket` has its output (timeout_us < 0: no limit).  Returns DJINN_OK,
+ * DJINN_E_INVAL on timeout / unknown ticket, or the error of its batch's forward. */
+DJINN_API int djinn_batcher_wait(djinn_batcher* b, int64_t ticket, int64_t timeout_us);
+/* Statistics since create: batches run, rows run, queries completed, and query latency
+ * (submit -> output written) percentiles p50 / p99 in microseconds (any pointer may be NULL). */
+DJINN_API int djinn_batcher_stats(djinn_batcher* b, int64_t* batches, int64_t* rows, int64_t* queries, double* p50_us,
+                                  double* p99_us);
+/* Closed-loop load generator for the serving measurements: `clients` native threads, each
+ * repeatedly submitting the next query of `queries` (n_queries x rows_per_query fp32 rows, used
+ * round robin) and waiting for it, for `seconds`.  Reports completed queries per second and the
+ * p50 / p99 latency of the queries of that run. */
+DJINN_API int djinn_batcher_drive(djinn_batcher* b, const float* queries, int64_t n_queries, int64_t rows_per_query,
+                                  int clients, double seconds, double* queries_per_s, double* p50_us, double* p99_us);
+/* Drain pending queries, stop the worker, free the staging buffers. */
+DJINN_API int djinn_batcher_destroy(djinn_batcher* b);
+
 #ifdef __cplusplus
 }
 #endif

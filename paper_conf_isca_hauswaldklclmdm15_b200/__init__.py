@@ -27,7 +27,9 @@ DJINN_OUT_PROB, DJINN_OUT_ARGMAX, DJINN_OUT_LOGITS = 0, 1, 2
 PRECISION = {"fp32": DJINN_FP32, "bf16": DJINN_BF16, "fp16": DJINN_FP16}
 EXPORTS = ["djinn_load_net", "djinn_forward", "djinn_forward16", "djinn_sync", "djinn_free", "djinn_net_info",
            "djinn_weight_arena", "djinn_plan_info", "djinn_profile", "djinn_profile_read", "djinn_op_info",
-           "djinn_describe", "djinn_last_error", "djinn_kernel_launches"]
+           "djinn_describe", "djinn_batcher_create", "djinn_batcher_submit", "djinn_batcher_wait",
+           "djinn_batcher_stats", "djinn_batcher_drive", "djinn_batcher_destroy", "djinn_last_error",
+           "djinn_kernel_launches"]
 OP_KINDS = ["pack", "gemm", "lrn", "pool", "softmax", "lrn+pool"]
 
 
@@ -62,12 +64,19 @@ def lib() -> ctypes.CDLL:
         L.djinn_op_info.argtypes = [P, I, ctypes.c_char_p, SZ, ctypes.POINTER(I), ctypes.POINTER(D),
                                     ctypes.POINTER(D), ctypes.POINTER(D)]
         L.djinn_describe.argtypes = [ctypes.c_char_p, SZ, I, I64, ctypes.c_char_p, SZ] + [ctypes.POINTER(I64)] * 4
+        L.djinn_batcher_create.argtypes = [P, I64, I64, I, ctypes.POINTER(P)]
+        L.djinn_batcher_submit.argtypes = [P, P, I64, P, ctypes.POINTER(I64)]
+        L.djinn_batcher_wait.argtypes = [P, I64, I64]
+        L.djinn_batcher_stats.argtypes = [P] + [ctypes.POINTER(I64)] * 3 + [ctypes.POINTER(D)] * 2
+        L.djinn_batcher_drive.argtypes = [P, P, I64, I64, I, D, ctypes.POINTER(D), ctypes.POINTER(D), ctypes.POINTER(D)]
+        L.djinn_batcher_destroy.argtypes = [P]
         L.djinn_last_error.restype = ctypes.c_char_p
         L.djinn_last_error.argtypes = []
         L.djinn_kernel_launches.restype = I64
         L.djinn_kernel_launches.argtypes = []
         for f in EXPORTS[:-2]:
             getattr(L, f).restype = I
+        L.djinn_batcher_destroy.restype = I
         _lib = L
     return _lib
 
@@ -219,6 +228,61 @@ def djinn_describe(desc: str, precision: int, max_rows: int):
 
 def djinn_kernel_launches() -> int:
     return int(lib().djinn_kernel_launches())
+
+
+# ----------------------------------------------------------------- query batcher
+class DjinnBatcher:
+    """Mirror of the djinn_batcher_* calls: stacks queries submitted from any thread into
+    batches of at most ``max_batch_rows`` rows run by a native worker."""
+
+    def __init__(self, net: "DjinnNet", max_batch_rows: int, max_wait_us: int = 200, out_mode: int = DJINN_OUT_PROB):
+        h = ctypes.c_void_p()
+        _check(lib().djinn_batcher_create(net.handle, max_batch_rows, max_wait_us, out_mode, ctypes.byref(h)))
+        self.handle = h.value
+        self.net = net
+        self.out_mode = out_mode
+
+    def submit(self, rows: np.ndarray, out: np.ndarray) -> int:
+        """Queue one query (float32 C-contiguous host rows); ``out`` (host, float32 rows x
+        out_elems, or int32 rows for ARGMAX) must stay alive until wait() returns."""
+        if rows.dtype != np.float32 or not rows.flags["C_CONTIGUOUS"]:
+            raise DjinnError(DJINN_E_INVAL, "query rows must be C-contiguous float32")
+        n = rows.shape[0]
+        want = (np.int32, n) if self.out_mode == DJINN_OUT_ARGMAX else (np.float32, n * self.net.out_elems)
+        if out.dtype != want[0] or not out.flags["C_CONTIGUOUS"] or out.size < want[1] or \
+                rows.size != n * self.net.in_elems:
+            raise DjinnError(DJINN_E_INVAL, "query / output buffer shape or dtype")
+        t = ctypes.c_int64()
+        _check(lib().djinn_batcher_submit(self.handle, rows.ctypes.data, n, out.ctypes.data, ctypes.byref(t)))
+        return t.value
+
+    def wait(self, ticket: int, timeout_us: int = -1) -> None:
+        _check(lib().djinn_batcher_wait(self.handle, ticket, timeout_us))
+
+    def stats(self) -> dict:
+        v = [ctypes.c_int64() for _ in range(3)] + [ctypes.c_double() for _ in range(2)]
+        _check(lib().djinn_batcher_stats(self.handle, *[ctypes.byref(x) for x in v]))
+        return dict(zip(("batches", "rows", "queries", "p50_us", "p99_us"), (x.value for x in v)))
+
+    def drive(self, queries: np.ndarray, rows_per_query: int, clients: int, seconds: float) -> dict:
+        """Native closed-loop load: ``clients`` threads submit-and-wait queries for ``seconds``."""
+        q = np.ascontiguousarray(queries, dtype=np.float32)
+        n = q.shape[0] // rows_per_query
+        qps, p50, p99 = ctypes.c_double(), ctypes.c_double(), ctypes.c_double()
+        _check(lib().djinn_batcher_drive(self.handle, q.ctypes.data, n, rows_per_query, clients, seconds,
+                                         ctypes.byref(qps), ctypes.byref(p50), ctypes.byref(p99)))
+        return {"queries_per_s": qps.value, "p50_us": p50.value, "p99_us": p99.value}
+
+    def close(self) -> None:
+        if self.handle:
+            _check(lib().djinn_batcher_destroy(self.handle))
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 # ----------------------------------------------------------------- convenience

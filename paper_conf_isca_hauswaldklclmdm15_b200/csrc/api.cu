@@ -7,9 +7,6 @@
 #include "../../include/djinn.h"
 #include "net.h"
 
-struct djinn_net {
-  djinn::Net impl;
-};
 
 namespace {
 thread_local std::string g_err;
@@ -47,6 +44,10 @@ int guarded(F&& f) {
   }
 }
 }  // namespace
+
+namespace djinn {
+void set_last_error(const std::string& msg) { g_err = msg; }
+}  // namespace djinn
 
 extern "C" {
 

@@ -161,6 +161,7 @@ struct Net {
 
 std::atomic<int64_t>& launch_counter();
 bool host_prof_on();
+void set_last_error(const std::string& msg);  // djinn_last_error() of the calling thread (api.cu)
 void host_prof_add(const std::string& key, double us);
 void encode_tmap(CUtensorMap* m, int dt, const void* base, int rank, const uint64_t* dims,
                  const uint64_t* strides_bytes, const uint32_t* box, int swizzle_bytes = 128,
@@ -169,3 +170,8 @@ void encode_im2col(CUtensorMap* m, int dt, const void* base, const uint64_t* dim
                    const int* lower_wh, const int* upper_wh, int channels, int pixels, const uint32_t* elem_strides);
 
 }  // namespace djinn
+
+// The C ABI's opaque handle (include/djinn.h).
+struct djinn_net {
+  djinn::Net impl;
+};
