@@ -284,6 +284,9 @@ def main():
     ap.add_argument("--precision", default=os.environ.get("DJINN_BENCH_PRECISION", "fp16"),
                     choices=["bf16", "fp16", "fp32"])
     ap.add_argument("--no-sweep", action="store_true", help="skip the per-app batch sweep (SURVEY 8(d))")
+    ap.add_argument("--headline-only", action="store_true",
+                    help="only the timed mixed step (for ncu launch lists): no sweep, serving, strong FACE, "
+                         "DIG fp32, e2e, token ids, concurrent services or CPU baseline")
     ap.add_argument("--dry-run", action="store_true",
                     help="launch/rendezvous/timing plumbing only (gloo on CPU; used by the CPU tests)")
     ap.add_argument("--oracle-leg", action="store_true", help=argparse.SUPPRESS)
@@ -306,6 +309,8 @@ def main():
         return reference_arm(args)
     if args.dry_run:
         return dry_run(args)
+    if args.headline_only:
+        args.no_sweep = args.no_e2e = args.no_ids = args.no_concurrent = args.no_cpu_baseline = True
     assert args.warmup >= 3 or os.environ.get("DJINN_BENCH_ALLOW_SHORT"), "W >= 3 warm-up steps required"
 
     import torch
@@ -518,7 +523,7 @@ def main():
     # ---- strong-scaled FACE (BASELINE configs[4]: "batch 256, sharded over 8xB200"): the
     # 256-image batch split into whole queries over the N ranks; q/s = 256 / max-over-ranks time
     face_strong = None
-    if "face" in apps:
+    if "face" in apps and not args.headline_only:
         q0, nr = parallel.query_shard(BATCH_ROWS["face"], 1, world, rank)
         n2 = clone_net("face", max(1, nr))
         xi = inputs["face"][:nr].contiguous()
@@ -530,7 +535,7 @@ def main():
 
     # ---- BASELINE configs[0]: DIG LeNet, 16 queries (1600 images), fp32 (SIMT FFMA path)
     dig_fp32 = None
-    if "dig" in apps:
+    if "dig" in apps and not args.headline_only:
         w32 = recipes.flat_blob(recipes.gen_weights("dig", "fp32"))
         n2 = dj.DjinnNet(dj.net_description("dig"), w32, "fp32", BATCH_ROWS["dig"], local)
         r0, nr = parallel.weak_shard(BATCH_ROWS["dig"], rank)
