@@ -999,6 +999,16 @@ void Net::choose_tiles() {
         o.bn = cap;
         o.g.cg = tc_pick_cg(g, o.bn);
       }
+      // Wave quantisation of large dense GEMMs on CTA pairs: a tile's MMA time grows with its
+      // width, so pick the width (192 or 256) with the fewer waves x width over the 74 pairs.
+      // Measured on B200 (DJINN_DENSE_BN=192 for all): ASR a1-a5 (8192 x 2048 x 2048, 4 waves
+      // of 256 vs 5 of 192) 57.3 -> 54.7 us each; ASR out (N = 8000) and IMC fc6 / fc7 slower at
+      // 192, as the model predicts.
+      if (env_cap < 0 && g.mode == GM_DENSE && o.g.cg == 2 && o.bn == 256) {
+        const int64_t pairs = tc_num_sms() / 2, mt = (g.M + 255) / 256;
+        auto cost = [&](int bn) { return ((mt * ((g.N + bn - 1) / bn) + pairs - 1) / pairs) * bn; };
+        if (cost(192) < cost(256)) o.bn = 192;
+      }
     }
     if (o.stem) o.g.cg = 2;  // the stem kernel loads B as two boxes of bn / 2 rows per K block
     if (o.g.slab && !tc_slab_config(o.g, o.bn)) {

@@ -123,7 +123,10 @@ def test_dense_tiles_at_the_bench_batches():
     face = _tiles("face", 256)
     assert face["F7"] == (64, 1) and face["F8"] == (64, 1)
     asr = _tiles("asr", 8192)
-    assert all(v == (256, 2) for v in asr.values())                # already > one wave
+    # > one wave: CTA pairs; the 2048-wide layers take 192-wide tiles (5 waves of 192 beat 4 of
+    # 256 over 74 pairs: wave quantisation), the 8000-wide output layer keeps 256
+    assert asr["out"] == (256, 2)
+    assert all(v == (192, 2) for k, v in asr.items() if k != "out")
     assert _tiles("pos", 4096)["l1"] == (64, 1)                    # 32 x 5 = 160 tiles
     dig = _tiles("dig", 1600)
     assert dig["ip1"] == (64, 1) and dig["ip2"] == (16, 1)
