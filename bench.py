@@ -630,6 +630,11 @@ def main():
                 "queries_per_s": q * world / (t / 1e3), "ms_per_batch": t,
                 "bytes_per_query": byts / q, "pcie_gbs_achieved": byts / (t / 1e3) / 1e9,
                 "pcie_gbs_needed_at_device_rate": byts / (per_app[a]["ms_per_batch"] / 1e3) / 1e9}
+            # Fig. 13: host bandwidth a server needs to keep G GPUs at their
+            # device-resident rate (weak scaling: G x one GPU's bytes/s), next to what this host
+            # delivered to one GPU
+            need1 = per_app[a]["host_fed"]["pcie_gbs_needed_at_device_rate"]
+            per_app[a]["host_fed"]["gbs_needed_vs_gpus"] = {str(G): G * need1 for G in (1, 2, 4, 8)}
         # the same step with the inputs sent in the path's 16-bit type (djinn_forward16):
         # lossless here (inputs are on the path's grid), half the H2D bytes
         if grid != "fp32":
