@@ -130,13 +130,16 @@ __device__ __forceinline__ void store16(const GemmGeom& g, void* Y, int64_t off,
         reinterpret_cast<float4*>(yp + 8 * h)[1] = make_float4(v[8 * h + 4], v[8 * h + 5], v[8 * h + 6], v[8 * h + 7]);
       }
   } else if (BF16 && g.out_half) {
+    // a bf16 net's conv output read only by the lrn+pool kernel is kept in fp16 (3 more mantissa
+    // bits than bf16; the plan says "fp16-out"), saturated to the fp16 range: a value beyond
+    // 65504 becomes +-65504, never inf (then NaN after LRN)
     uint16_t* yp = reinterpret_cast<uint16_t*>(Y) + off;
 #pragma unroll
     for (int h = 0; h < 2; ++h)
       if (h < nvalid8)
         st16(yp + 8 * h,
-             make_uint4(pack2<false>(v[8 * h], v[8 * h + 1]), pack2<false>(v[8 * h + 2], v[8 * h + 3]),
-                        pack2<false>(v[8 * h + 4], v[8 * h + 5]), pack2<false>(v[8 * h + 6], v[8 * h + 7])));
+             make_uint4(pack2_f16_sat(v[8 * h], v[8 * h + 1]), pack2_f16_sat(v[8 * h + 2], v[8 * h + 3]),
+                        pack2_f16_sat(v[8 * h + 4], v[8 * h + 5]), pack2_f16_sat(v[8 * h + 6], v[8 * h + 7])));
   } else {
     uint16_t* yp = reinterpret_cast<uint16_t*>(Y) + off;
 #pragma unroll

@@ -336,6 +336,10 @@ __device__ __forceinline__ void lds16(float (&b)[16], const float* s) {
 #pragma unroll
   for (int q = 0; q < 4; ++q) *reinterpret_cast<float4*>(b + 4 * q) = reinterpret_cast<const float4*>(s)[q];
 }
+__device__ __forceinline__ uint32_t pack2_f16_sat(float a, float b) {  // fp16 pair, clamped to +-65504
+  __half2 h = __floats2half2_rn(fminf(fmaxf(a, -65504.f), 65504.f), fminf(fmaxf(b, -65504.f), 65504.f));
+  return *reinterpret_cast<uint32_t*>(&h);
+}
 template <bool BF16>
 __device__ __forceinline__ uint32_t pack2(float a, float b) {
   if (BF16) {

@@ -275,3 +275,29 @@ def test_binding_rejects_unsafe_buffers():
     dj.djinn_forward(net.handle, x, 64, out, dj.DJINN_OUT_PROB)                        # the valid call works
     dj.djinn_sync(net.handle)
     net.close()
+
+
+_SAT_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1]); sys.path.insert(0, sys.argv[1] + "/tests")
+import test_layers_gpu as t
+from datagen import recipes
+import paper_conf_isca_hauswaldklclmdm15_b200 as dj
+net, W, x = t.gen_net("gen_c", "bf16")
+W[0]["w"] = W[0]["w"] * 4096.0          # conv1 outputs far beyond the fp16 range (65504)
+W[0]["b"] = W[0]["b"] * 4096.0
+n = dj.DjinnNet(t.GEN_C, recipes.flat_blob(W), "bf16", x.shape[0])
+print(n.plan())
+np.save(sys.argv[2], n.forward(torch.from_numpy(x).cuda(), dj.DJINN_OUT_LOGITS).cpu().numpy())
+"""
+
+
+def test_bf16_fp16_intermediate_saturates_instead_of_overflowing(tmp_path):
+    """a bf16 net's conv output read only by the lrn+pool kernel is kept in fp16
+    ("fp16-out" in the plan); values beyond 65504 must saturate, never become inf / NaN."""
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    f = str(tmp_path / "lg.npy")
+    r = subprocess.run([sys.executable, "-c", _SAT_CHILD, root, f], env=dict(os.environ, DJINN_LRN_POOL="1"),
+                       check=True, timeout=600, capture_output=True, text=True)
+    assert "fp16-out" in r.stdout, r.stdout
+    assert np.isfinite(np.load(f)).all()
