@@ -34,6 +34,8 @@
 #include "kernels.h"
 #include "tc_common.cuh"
 #include <atomic>
+#include <algorithm>
+#include <type_traits>
 #define TC_MAX_DEVICES 64
 
 #ifdef DJINN_TC_STATS
@@ -240,7 +242,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   const uint32_t sfull0 = smem_u32(bars + 2 * NST + 8), sempty0 = smem_u32(bars + 2 * NST + 10);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int num_kb = g.Kpad / BK;
+  const int num_kb = g.ksplit > 1 ? g.kpb : g.Kpad / BK;  // K blocks per tile (split-K: per split)
 #ifdef DJINN_TC_STATS
   unsigned long long st_prod_wait = 0, st_prod_issue = 0, st_mma_full = 0, st_mma_tempty = 0, st_mma_issue = 0, st_epi_wait = 0,
                      st_epi_work = 0;
@@ -322,6 +324,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     int s = 0, qo = 0;  // ring slot; owner of the current stage (q % nown)
     uint32_t ph = 0;
     auto load_b = [&](uint32_t fb, int kb, int n0, int z) {
+      // split-K (dense): z is the K split, B has one z slice
+      if (g.ksplit > 1) { kb += z * g.kpb; z = 0; }
       if (!kDbgNoB) tma_a3<CG>(sB0 + (uint32_t)s * C::B_BYTES, &tmB, fb, kb * BK, n0 * BN + bn_off, z);
     };
     auto next_stage = [&]() {
@@ -491,7 +495,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           const uint32_t a_dst = sA0 + (uint32_t)s * C::A_BYTES;
           const bool iss = mine && leader;
           if (mode == GM_DENSE) {
-            if (iss) tma_a2<CG>(a_dst, &tmA, fb, kb * BK, my_m0);
+            if (iss) tma_a2<CG>(a_dst, &tmA, fb, (kb + (g.ksplit > 1 ? z * g.kpb : 0)) * BK, my_m0);
           } else {
             for (int j = 0; j < chunks_per_kb; ++j, ++q) {
               // past the valid K: a channel coordinate beyond the extent -> TMA zero-fills
@@ -718,7 +722,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             if (co < g.Co) b = __ldg(g.mode == GM_LC ? bias + (int64_t)tc.z0 * g.bias_zstride + dx * g.Co + co : bias + co);
           } else {
             const int zi = c / BN, nb = tc.n0 * BN + (c - zi * BN);
-            if (nb < g.N) b = __ldg(bias + (int64_t)(tc.z0 * g.zf + zi) * g.bias_zstride + nb);
+            if (nb < g.N && g.ksplit <= 1) b = __ldg(bias + (int64_t)(tc.z0 * g.zf + zi) * g.bias_zstride + nb);
           }
           sb[c] = b;
         }
@@ -867,7 +871,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       } else {
         for (int zi = 0; zi < g.zf; ++zi) {
           const int z = tc.z0 * g.zf + zi;
-          const int64_t pix = (g.mode == GM_LC) ? (int64_t)m * g.OH * g.OW + z : (g.mode == GM_CONV ? opix : (int64_t)m);
+          const int64_t pix = (g.mode == GM_LC) ? (int64_t)m * g.OH * g.OW + z
+                              : (g.mode == GM_CONV ? opix : (int64_t)m + (g.ksplit > 1 ? (int64_t)z * g.M : 0));
           const int goff = (g.mode == GM_CONV) ? z * g.cout_goff : 0;
           const int nb0 = tc.n0 * BN;
 #pragma unroll 1
@@ -1027,6 +1032,63 @@ cudaError_t launch_bn(const GemmGeom& g, int bn, const CUtensorMap* tmA, const C
 }
 
 }  // namespace
+
+namespace {
+// split-K reduction: 8 columns per thread, partial sums added in split order
+template <typename T>
+__global__ void splitk_reduce_kernel(const float* __restrict__ part, int S, int64_t rows, int N, int ppitch,
+                                     const float* __restrict__ bias, int act, T* __restrict__ y, float* __restrict__ yf,
+                                     int out_pitch, int write_cols) {
+  pdl_trigger();
+  pdl_wait();
+  const int c8 = (write_cols + 7) / 8;
+  const int64_t total = rows * c8, split = rows * (int64_t)ppitch;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t m = i / c8;
+    const int n0 = (int)(i - m * c8) * 8;
+    float v[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) v[j] = 0.f;
+    if (n0 < N) {
+      const float* p = part + m * ppitch + n0;
+      for (int sidx = 0; sidx < S; ++sidx, p += split) {
+        const float4 a = __ldg(reinterpret_cast<const float4*>(p)), b = __ldg(reinterpret_cast<const float4*>(p + 4));
+        v[0] += a.x; v[1] += a.y; v[2] += a.z; v[3] += a.w; v[4] += b.x; v[5] += b.y; v[6] += b.z; v[7] += b.w;
+      }
+#pragma unroll
+      for (int j = 0; j < 8; ++j) v[j] = n0 + j < N ? act_fast(v[j] + __ldg(bias + n0 + j), act) : 0.f;
+    }
+    if (yf) {
+      float* o = yf + m * out_pitch + n0;
+#pragma unroll
+      for (int j = 0; j < 8; ++j)
+        if (n0 + j < write_cols) o[j] = v[j];
+    } else {
+      *reinterpret_cast<uint4*>(y + m * out_pitch + n0) =
+          make_uint4(pack2<sizeof(T) == 2 && !std::is_same<T, __half>::value>(v[0], v[1]),
+                     pack2<sizeof(T) == 2 && !std::is_same<T, __half>::value>(v[2], v[3]),
+                     pack2<sizeof(T) == 2 && !std::is_same<T, __half>::value>(v[4], v[5]),
+                     pack2<sizeof(T) == 2 && !std::is_same<T, __half>::value>(v[6], v[7]));
+    }
+  }
+}
+}  // namespace
+
+cudaError_t launch_splitk_reduce(const float* part, int S, int64_t rows, int N, int ppitch, const float* bias, int act,
+                                 void* y, int out_pitch, int write_cols, int out_f32, int dt, cudaStream_t st) {
+  if (rows <= 0) return cudaSuccess;
+  if (ppitch % 8 || (!out_f32 && (out_pitch % 8 || write_cols % 8))) return cudaErrorInvalidValue;
+  const int64_t total = rows * ((write_cols + 7) / 8);
+  const int grid = (int)std::min<int64_t>((total + 255) / 256, 148 * 16);
+  if (out_f32)
+    return launch_pdl(splitk_reduce_kernel<__half>, dim3(grid), dim3(256), 0, st, part, S, rows, N, ppitch, bias, act,
+                      (__half*)nullptr, (float*)y, out_pitch, write_cols);
+  if (dt == DT_BF16)
+    return launch_pdl(splitk_reduce_kernel<__nv_bfloat16>, dim3(grid), dim3(256), 0, st, part, S, rows, N, ppitch, bias,
+                      act, (__nv_bfloat16*)y, (float*)nullptr, out_pitch, write_cols);
+  return launch_pdl(splitk_reduce_kernel<__half>, dim3(grid), dim3(256), 0, st, part, S, rows, N, ppitch, bias, act,
+                    (__half*)y, (float*)nullptr, out_pitch, write_cols);
+}
 
 int tc_num_sms() {
   if (!g_num_sms) {

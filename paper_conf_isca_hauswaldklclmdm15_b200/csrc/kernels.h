@@ -126,6 +126,8 @@ struct GemmGeom {
   int epi_wg;         // epilogue warpgroups draining tiles: 3 (3 slots) or 2 (up to 4 slots)
   int ldwait;         // slab mode: B-loader stage wait (0 spin, 1 poll + nanosleep back-off, 2 suspend hint)
   int obd;            // conv output: zero border of the stored output tensor (its consumer's pad)
+  int ksplit, kpb;    // dense split-K: z = K split (ksplit > 1), kpb K blocks each; the launch writes
+                      // fp32 partial sums [ksplit][M][out_pitch] with no bias / activation
   int lrn_size;
   float lrn_alpha_over_n, lrn_beta, lrn_k;
 };
@@ -216,6 +218,12 @@ int mlp2_smem(const MlpGeom& g);
 bool mlp2_supported(const MlpGeom& g);
 cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const CUtensorMap* tmW2, const float* x,
                         const float* b1, const float* b2, void* out, cudaStream_t st);
+
+// --- split-K reduction: y[m][n] = act(bias[n] + sum_s part[s][m][n]) for n < N, 0 for
+// N <= n < write_cols; part fp32 [S][rows][ppitch]; y 16-bit (dt) or fp32 (out_f32) with row
+// pitch out_pitch.  The partial sums are added in split order (deterministic).
+cudaError_t launch_splitk_reduce(const float* part, int S, int64_t rows, int N, int ppitch, const float* bias, int act,
+                                 void* y, int out_pitch, int write_cols, int out_f32, int dt, cudaStream_t st);
 
 // --- LRN across channels (K4), NHWC ----------------------------------------------------------
 // Channel c of a pixel is stored at (c/gsz)*gpitch + c%gsz (grouped layouts); pads -> 0.

@@ -1010,6 +1010,27 @@ void Net::choose_tiles() {
         if (cost(192) < cost(256)) o.bn = 192;
       }
     }
+    // Split-K for dense GEMMs that cannot fill the GPU with output tiles but have a long K (FACE
+    // F8: 4 tiles of 64 K blocks; the FC layers at the Table 3 batches, e.g. IMC fc6 at 16
+    // images): K is cut into S ranges so S x tiles CTAs stream it; the fp32 partials are added
+    // in split order by a reduction that applies bias + activation.  DJINN_SPLITK=0 disables.
+    {
+      static const bool sk_on = [] {
+        const char* e = getenv("DJINN_SPLITK");
+        return !(e && e[0] == '0');
+      }();
+      const int nkb = g.Kpad / 64;
+      const int64_t tiles = ((g.M + 127) / 128) * ((g.N + o.bn - 1) / o.bn);
+      o.ksplit = 1;
+      if (sk_on && !o.mlp && g.mode == GM_DENSE && o.g.cg == 1 && nkb >= 32 && tiles <= 74) {
+        const int S = (int)std::min<int64_t>(nkb / 8, 148 / tiles);
+        if (S >= 2) {
+          o.ksplit = S;
+          o.kpb = (nkb + S - 1) / S;
+          o.npart = rup(g.N, 8);
+        }
+      }
+    }
     if (o.stem) o.g.cg = 2;  // the stem kernel loads B as two boxes of bn / 2 rows per K block
     if (o.g.slab && !tc_slab_config(o.g, o.bn)) {
       o.g.slab = 0;
@@ -1131,6 +1152,7 @@ Workspace::~Workspace() {
   if (in_stage) cudaFree(in_stage);
   if (in_stage16) cudaFree(in_stage16);
   if (in_wide) cudaFree(in_wide);
+  if (part) cudaFree(part);
   if (out_stage) cudaFree(out_stage);
   for (int s = 0; s < 2; ++s)
     for (cudaEvent_t e : {in_ready[s], in_free[s], out_ready[s], out_free[s]})
@@ -1169,6 +1191,12 @@ Workspace* Net::workspace(cudaStream_t st) {
     if (!buf_bytes[b]) continue;
     if (cudaMalloc(&w->buf[b], buf_bytes[b]) != cudaSuccess) throw Error(DJINN_E_NOMEM, "workspace allocation");
     ck(cudaMemset(w->buf[b], 0, buf_bytes[b]), "workspace memset");
+  }
+  {
+    size_t pb = 0;
+    for (const Op& o : ops)
+      if (o.ksplit > 1) pb = std::max(pb, (size_t)o.ksplit * max_rows * o.npart * 4);
+    if (pb && cudaMalloc(&w->part, pb) != cudaSuccess) throw Error(DJINN_E_NOMEM, "split-K workspace");
   }
   w->tmA.resize(ops.size());
   w->tmY0.resize(ops.size());
@@ -1389,7 +1417,23 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           } else if (dt == DT_F32)
             e = launch_simt_gemm(g, (const float*)A, (const float*)(ar + o.w_off), (const float*)(ar + o.b_off),
                                  (float*)Y, st);
-          else
+          else if (o.ksplit > 1) {
+            GemmGeom gp = g;  // fp32 partials over o.ksplit K ranges, no bias / activation
+            gp.Z = gp.ksplit = o.ksplit;
+            gp.kpb = o.kpb;
+            gp.act = ACT_NONE;
+            gp.out_f32 = 1;
+            gp.out_half = 0;
+            gp.out_pitch = gp.write_cols = o.npart;
+            gp.out_gsz = gp.out_gpitch = 1 << 30;
+            gp.bias_zstride = 0;
+            e = launch_tc_gemm(gp, o.bn, dt, &w->tmA[i], &o.tmB, (const float*)(ar + o.b_off), w->part, st);
+            if (e == cudaSuccess) {
+              ++launches;
+              e = launch_splitk_reduce(w->part, o.ksplit, n, g.N, o.npart, (const float*)(ar + o.b_off), g.act, Y,
+                                       g.out_pitch, g.write_cols, g.out_f32, dt, st);
+            }
+          } else
             e = launch_tc_gemm(g, o.bn, dt, &w->tmA[i], &o.tmB, (const float*)(ar + o.b_off), Y, st);
           break;
         }
@@ -1467,6 +1511,7 @@ std::string Net::plan_string() const {
         << (o.g.lcg > 1 ? " taps/row=" + std::to_string(o.g.lcg) : std::string())
         << (o.g.mode == GM_CONV && o.g.a_tiled ? " block=" + std::to_string(o.g.bx) + "x" + std::to_string(o.g.by) + "x" +
                                                   std::to_string(o.g.bn) : std::string())
+        << (o.ksplit > 1 ? " split-K=" + std::to_string(o.ksplit) + "x" + std::to_string(o.kpb) : std::string())
         << (o.stem == 1 ? " stem(fp32 input, fused pack, resident B, TMA-store epilogue)" : "")
         << (o.stem == 2 ? " stem(TMA slab, resident B, TMA-store epilogue)" : "")
         << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << (o.g.out_half ? " fp16-out" : "") << "]";

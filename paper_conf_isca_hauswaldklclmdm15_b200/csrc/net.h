@@ -85,6 +85,9 @@ struct Op {
   // fused two-layer MLP + softmax (k_mlp.cu): this GEMM op runs the whole net (mlp = 1); the
   // pack, the second GEMM and the softmax ops are not launched (fused = 1)
   int mlp = 0;
+  // dense split-K (ksplit > 1): the GEMM writes fp32 partials over ksplit K ranges of kpb
+  // K blocks into the workspace's part buffer (pitch npart), a reduction adds bias + act
+  int ksplit = 1, kpb = 0, npart = 0;
   MlpGeom mg{};
   CUtensorMap tmW1{}, tmW2{};
   // SENNA window lookup in place of the pack (embed = 1): see EmbedGeom (kernels.h)
@@ -120,6 +123,7 @@ struct Workspace {
   int64_t pipe_cs = 0;  // chunk rows of the last host-fed call (slot offsets depend on it)
   std::vector<CUtensorMap> tmA;  // per op (dense gemm) over its input buffer
   std::vector<CUtensorMap> tmY0, tmY1;  // per op (stem): TMA-store maps over its output buffer
+  float* part = nullptr;                 // split-K partial sums (the largest need of any op)
   ~Workspace();
 };
 

@@ -360,3 +360,30 @@ def test_mlp_kernel_equals_unfused_path(app, prec, n, tmp_path):
     assert np.array_equal(res[0]["lg"], res[1]["lg"])
     assert np.array_equal(res[0]["am"], res[1]["am"])
     np.testing.assert_allclose(res[0]["pr"], res[1]["pr"], rtol=2e-6, atol=1e-7)
+
+
+@pytest.mark.parametrize("app,prec,n", [("imc", "fp16", 16), ("face", "bf16", 2), ("face", "fp16", 256)])
+def test_split_k_dense_layers_match_oracle_and_unsplit(app, prec, n, tmp_path):
+    """Dense layers with few output tiles and a long K run split-K (fp32 partials added in
+    split order by a reduction that applies bias + activation): IMC fc6/fc7/fc8 at the Table 3
+    batch of 16 images, FACE F7/F8 at 2 and F8 at 256 images.  Against the oracle (contract
+    tolerance) and against the unsplit kernels (DJINN_SPLITK=0: only fp32 summation order
+    differs, so the logits agree to a few 16-bit roundings)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    x = recipes.gen_input_rows(app, 0, n, prec)
+    lg_ref, _ = oracle_rows(app, x, prec)
+    outs = []
+    for v in ("1", "0"):
+        f = str(tmp_path / f"lg{v}.npy")
+        env = dict(os.environ, DJINN_SPLITK=v)
+        r = subprocess.run([sys.executable, "-c", _STEM_CHILD, root, app, prec, str(n), f, "0"], env=env, check=True,
+                           timeout=600, capture_output=True, text=True)
+        assert ("split-K" in r.stdout) == (v == "1"), r.stdout
+        outs.append(np.load(f))
+    r = compare_16bit(outs[0], lg_ref)
+    assert r["rel_max"] <= REL_LOGIT_TOL and r["elem_max"] <= ELEM_TOL, r
+    d = compare_16bit(outs[0], outs[1].astype(np.float64))
+    assert d["rel_max"] <= 5e-3, d
