@@ -689,9 +689,17 @@ void Net::build(const std::string& desc) {
         g.cw = 64;
         const int P = o.out.Cp;
         int XB = 1;
+        // cap on the LC x-block: 8 (N = 128, CTA pairs) pays at a full 256-image batch (FACE L4
+        // 79 us vs 101 at 4), 4 below one 128-row tile (FACE 2 / 32 images: 214 -> 192 us, 227 ->
+        // 199 us per batch on B200).  DJINN_LC_XB overrides.
+        static const int lc_xb_env = [] {
+          const char* e = getenv("DJINN_LC_XB");
+          return e ? atoi(e) : 0;
+        }();
+        const int lc_xb_cap = lc_xb_env > 0 ? lc_xb_env : (max_rows <= 128 ? 4 : 8);
         if (o.out.gsz >= o.out.C && P <= 64)
           for (int xbc = 8; xbc >= 2; xbc /= 2)
-            if (xbc * P <= 256 && (xbc - 1) * g.stride + g.KW <= 32) { XB = xbc; break; }
+            if (xbc <= lc_xb_cap && xbc * P <= 256 && (xbc - 1) * g.stride + g.KW <= 32) { XB = xbc; break; }
         g.kwp = rup((XB - 1) * g.stride + g.KW, g.lcg);
         g.K = g.KH * g.kwp * g.Cgp;
         if (XB > 1) {
