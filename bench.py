@@ -486,10 +486,24 @@ def main():
         k = int(min(200, max(5, target_ms / max(t1, 1e-3))))
         return timed(f, k) / k
 
+    blob_cache = {}
+
     def clone_net(app, rows, prec=None):
+        # the arena layout can depend on max_rows (e.g. the LC x-block below one 128-row tile):
+        # copy the loaded arena when the layouts agree, else pack the weights again
+        import re
+
+        def layout(n):  # what the weight packing depends on: each GEMM's Z x N x Kpad and x-block
+            return re.findall(r"N=\d+ Z=\d+ K=\d+ Kpad=\d+|xblock=\d+", n.plan())
         n2 = dj.DjinnNet(dj.net_description(app), None, prec or grid, rows, local)
-        parallel.arena_tensor(n2).copy_(parallel.arena_tensor(nets[app]))
-        return n2
+        a2, a1 = parallel.arena_tensor(n2), parallel.arena_tensor(nets[app])
+        if a2.numel() == a1.numel() and layout(n2) == layout(nets[app]):
+            a2.copy_(a1)
+            return n2
+        n2.close()
+        if app not in blob_cache:
+            blob_cache[app] = recipes.flat_blob(recipes.gen_weights(app, prec or grid))
+        return dj.DjinnNet(dj.net_description(app), blob_cache[app], prec or grid, rows, local)
 
     def tiled(x, rows):
         reps = (rows + x.shape[0] - 1) // x.shape[0]
