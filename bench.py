@@ -84,22 +84,49 @@ def queries_per_step(world: int = 1) -> float:
 
 # ------------------------------------------------------------------ clocks sampler
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled every 50 ms in a background process; only
-    samples whose host timestamp falls inside [mark_start, mark_end] (the timed region) are
-    summarised (B200_PROFILING.md "clocks DURING the timed region")."""
+    """SM clock, power and clock-event (throttle) reasons sampled DURING the timed region
+    (B200_PROFILING.md "clocks DURING the timed region"): an NVML thread polls every 2 ms between
+    mark_start and mark_end (the timed region of the default run is ~70 ms, too short for
+    nvidia-smi's 50 ms loop to catch reliably); nvidia-smi every 50 ms is the fallback."""
     Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
     NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+    NVML_BITS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40, "sw_power_cap": 0x4}
 
     def __init__(self, device: int):
         self.device = device
         self.rows = []
         self.proc = None
+        self.nv = None
+        self.active = False
+        self.stop = False
         self.t0 = self.t1 = None
+        self.src = None
+
+    def _nvml_handle(self):
+        import pynvml
+        pynvml.nvmlInit()
+        try:
+            import torch
+            bus = torch.cuda.get_device_properties(self.device).pci_bus_id
+            dom = torch.cuda.get_device_properties(self.device).pci_domain_id
+            dev = torch.cuda.get_device_properties(self.device).pci_device_id
+            return pynvml, pynvml.nvmlDeviceGetHandleByPciBusId(f"{dom:08x}:{bus:02x}:{dev:02x}.0")
+        except Exception:
+            return pynvml, pynvml.nvmlDeviceGetHandleByIndex(self.device)
 
     def __enter__(self):
         try:
+            self.nv = self._nvml_handle()
+            self.src = "nvml 2 ms"
+            self.t = threading.Thread(target=self._poll, daemon=True)
+            self.t.start()
+            return self
+        except Exception:
+            self.nv = None
+        try:
+            self.src = "nvidia-smi 50 ms"
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}",
                                           "--format=csv,noheader,nounits", "-lms", "50"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
@@ -110,18 +137,39 @@ class ClockSampler:
             self.proc = None
         return self
 
+    def _poll(self):
+        pm, h = self.nv
+        mx = pm.nvmlDeviceGetMaxClockInfo(h, pm.NVML_CLOCK_SM)
+        while not self.stop:
+            if self.active:
+                try:
+                    sm = pm.nvmlDeviceGetClockInfo(h, pm.NVML_CLOCK_SM)
+                    pw = pm.nvmlDeviceGetPowerUsage(h) / 1000.0
+                    rs = pm.nvmlDeviceGetCurrentClocksEventReasons(h)
+                    act = ["Active" if rs & self.NVML_BITS[n] else "Not Active" for n in self.NAMES]
+                    self.rows.append((time.time(), [str(sm), str(mx), f"{pw:.1f}"] + act))
+                except Exception:
+                    pass
+                time.sleep(0.002)
+            else:
+                time.sleep(0.0005)
+
     def _read(self):
         for line in self.proc.stdout:
             self.rows.append((time.time(), [x.strip() for x in line.split(",")]))
 
     def mark_start(self):
         self.t0 = time.time()
+        self.active = True
 
     def mark_end(self):
+        self.active = False
         self.t1 = time.time()
-        time.sleep(0.1)
+        if self.proc:
+            time.sleep(0.1)
 
     def __exit__(self, *a):
+        self.stop = True
         if self.proc:
             self.proc.terminate()
             try:
@@ -137,7 +185,7 @@ class ClockSampler:
         pw = [float(r[2]) for r in rows if len(r) > 2 and num(r[2])]
         reasons = sorted({self.NAMES[i] for r in rows for i in range(4) if len(r) > 3 + i and r[3 + i] == "Active"})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(rows), "power_w_max": max(pw) if pw else None}
+                "reasons": reasons, "samples": len(rows), "power_w_max": max(pw) if pw else None, "source": self.src}
 
 
 # ------------------------------------------------------------------ CPU oracle leg
