@@ -36,6 +36,17 @@
 //   SLAB: warps 0-11 epilogue (3 warpgroups, 3 TMEM slots: the LRN epilogue is the long pole),
 //     warp 12 slab TMA producer, warp 13 MMA.  Staging holds the 64-channel box of each warp;
 //     the remaining BN - 64 channels are stored from registers.
+//   POOL (SLAB + K5 fused, the default for IMC conv1 + norm1 + pool1): the following 3 x 3 /
+//     stride-2 MAX pool runs in the epilogue, so the conv output (IMC: 595 MB) never reaches HBM
+//     -- only the pooled tensor (4.2x smaller) is written, in the consumer's layout.  A tile is
+//     two output rows of one image (2 * Ws <= 128 GEMM rows, starting at row 2r): pool row r
+//     takes conv rows 2r, 2r + 1, 2r + 2, so tile r computes the partial max of its rows 2r and
+//     2r + 1 (handed to the next tile's warpgroup through shared memory, mbarrier-ordered) and
+//     completes pool row r - 1 with its row 2r.  A CTA walks whole bands of pool rows of one
+//     image in order (bands split an image only when there are fewer images than SMs).  The
+//     epilogue stages each half of the LRN'd channels (16-bit, exactly the values the unfused
+//     path stores) in shared memory, pools them, and writes the pooled pixels with coalesced
+//     16-byte stores.
 #include "tc_common.cuh"
 #include <cstdio>
 
@@ -79,13 +90,46 @@ template <int BN, bool GATHER>
 __host__ __device__ constexpr int stem_stage_bytes() {  // staging bytes per epilogue warp
   return GATHER ? 32 * BN * 2 : (BN / 64) * 4096;
 }
-template <int BN, int KS, bool GATHER>
+// POOL: per warpgroup, one half of the tile's channels staged per pixel at an odd number of
+// 16-byte pieces (conflict-free for 8 consecutive pixels); two hand-off buffers of the partial
+// pool row, [2 halves][POW_MAX][HP pieces]
+constexpr int POW_MAX = 28;
+template <int BN>
+__host__ __device__ constexpr int pool_pstr() { return ((BN / 2) / 8 + 1) * 16; }
+template <int BN>
+__host__ __device__ constexpr int pool_hand_bytes() { return 2 * POW_MAX * ((BN / 2) / 8) * 16; }
+template <int BN, int KS, bool GATHER, bool POOL>
 __host__ __device__ constexpr int stem_smem() {
   return 1024 + ((KS * KS * BN * 128 + 1023) & ~1023) + 2 * ST_SLAB_BYTES +
-         StemCfg<GATHER>::EPI_WARPS * stem_stage_bytes<BN, GATHER>() + 16 * 8 + 16;
+         (POOL ? StemCfg<GATHER>::NWG * 128 * pool_pstr<BN>() + 2 * pool_hand_bytes<BN>()
+               : StemCfg<GATHER>::EPI_WARPS * stem_stage_bytes<BN, GATHER>()) +
+         32 * 8 + 16;
+}
+__device__ __forceinline__ uint4 lds128(uint32_t addr) {
+  uint4 v;
+  asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr) : "memory");
+  return v;
+}
+template <bool BF16>
+__device__ __forceinline__ uint4 hmax8(uint4 a, uint4 b) {  // packed 16-bit max (exact)
+  uint4 r;
+  if (BF16) {
+    const __nv_bfloat162* x = reinterpret_cast<const __nv_bfloat162*>(&a);
+    const __nv_bfloat162* y = reinterpret_cast<const __nv_bfloat162*>(&b);
+    __nv_bfloat162* z = reinterpret_cast<__nv_bfloat162*>(&r);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) z[j] = __hmax2(x[j], y[j]);
+  } else {
+    const __half2* x = reinterpret_cast<const __half2*>(&a);
+    const __half2* y = reinterpret_cast<const __half2*>(&b);
+    __half2* z = reinterpret_cast<__half2*>(&r);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) z[j] = __hmax2(x[j], y[j]);
+  }
+  return r;
 }
 
-template <int BN, bool BF16, int F, int C0, int KS, bool GATHER>
+template <int BN, bool BF16, int F, int C0, int KS, bool GATHER, bool POOL>
 __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
     stem_conv_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                      const __grid_constant__ CUtensorMap tmY0, const __grid_constant__ CUtensorMap tmY1,
@@ -110,17 +154,37 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
   uint8_t* sB = smem;
   uint8_t* sSlab = sB + ((KB * B_BLK + 1023) & ~1023);
   uint8_t* sOut = sSlab + 2 * ST_SLAB_BYTES;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sOut + SC::EPI_WARPS * STG);
-  // bars: bfull, sfull[2], sempty[2], tfull[4], tempty[4]
+  uint8_t* sHand = sOut + (POOL ? NWG * 128 * pool_pstr<BN>() : SC::EPI_WARPS * STG);  // POOL: partial pool rows
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sHand + (POOL ? 2 * pool_hand_bytes<BN>() : 0));
+  // bars: bfull, sfull[2], sempty[2], tfull[4], tempty[4], (tmem slot), POOL: hfull[2][2] at 16, hempty[2][2] at 20
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 13);
   __shared__ __align__(16) float sbias[BN];
   const uint32_t bfull = smem_u32(bars), sfull0 = smem_u32(bars + 1), sempty0 = smem_u32(bars + 3);
   const uint32_t tfull0 = smem_u32(bars + 5), tempty0 = smem_u32(bars + 9);
+  const uint32_t hfull0 = smem_u32(bars + 16), hempty0 = smem_u32(bars + 20);
+  static_assert(!POOL || !GATHER, "the fused pool runs on the TMA-slab variant");
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int HW = g.Hs * g.Ws;
   const int64_t M = (int64_t)g.Nimg * HW;
   const int tiles = (int)((M + 127) / 128);
+  // This CTA's tile sequence, walked identically by the producer, the MMA warp and the
+  // epilogue: fn(local tile lt, first GEMM row, image, pool-row index r, first / last tile of a
+  // band).  POOL: units (image, band of pool rows [pr0, pr1)), tile r = conv rows 2r, 2r + 1
+  // for r = pr0 .. pr1; otherwise 128 consecutive virtual pixels, strided over the grid.
+  auto for_each_tile = [&](auto&& fn) {
+    int lt = 0;
+    if (POOL) {
+      const int units = g.Nimg * g.bands;
+      for (int u = cid; u < units; u += ncl) {
+        const int img = u / g.bands, b = u - img * g.bands;
+        const int pr0 = b * g.POH / g.bands, pr1 = (b + 1) * g.POH / g.bands;
+        for (int r = pr0; r <= pr1; ++r, ++lt) fn(lt, img * HW + 2 * r * g.Ws, img, r, r == pr0, r == pr1);
+      }
+    } else {
+      for (int t = cid; t < tiles; t += ncl, ++lt) fn(lt, t * 128, 0, 0, false, false);
+    }
+  };
 
   if (warp == SC::PROD_WARP && lane == 0) {
     mbar_init(bfull, 1);
@@ -132,6 +196,11 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
       mbar_init(tfull0 + 8 * s, 1);
       mbar_init(tempty0 + 8 * s, 4);  // the draining warpgroup
     }
+    if (POOL)
+      for (int s = 0; s < 4; ++s) {
+        mbar_init(hfull0 + 8 * s, 1);   // writer warpgroup, per (buffer, half)
+        mbar_init(hempty0 + 8 * s, 1);  // reader warpgroup, per (buffer, half)
+      }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");  // (cluster of one)
     fence_proxy_async();
     if (!GATHER) asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmA) : "memory");
@@ -240,21 +309,150 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
   } else if (!GATHER && warp == SC::PROD_WARP) {
     // ---- slab producer: one TMA box {64 channels, slab rows} of the packed tensor per tile
     if (elect_one()) {
-      int lt = 0;
-      for (int t = cid; t < tiles; t += ncl, ++lt) {
+      for_each_tile([&](int lt, int row0, int, int, bool, bool) {
         const int sb = lt & 1;
         mbar_wait_sleep(sempty0 + 8 * sb, ((uint32_t)(lt >> 1) & 1) ^ 1);
         mbar_arrive_expect_tx(sfull0 + 8 * sb, (uint32_t)g.slab_rows * 128u);
-        tma_2d(smem_u32(sSlab) + (uint32_t)sb * ST_SLAB_BYTES, &tmA, sfull0 + 8 * sb, 0, t * 128);
-      }
+        tma_2d(smem_u32(sSlab) + (uint32_t)sb * ST_SLAB_BYTES, &tmA, sfull0 + 8 * sb, 0, row0);
+      });
     }
     __syncwarp();
   } else if (!GATHER && warp == SC::MMA_WARP) {
     mbar_wait(bfull, 0);
     tc_fence_after();
-    int lt = 0;
-    for (int t = cid; t < tiles; t += ncl, ++lt) issue_tile(lt);
-  } else if (warp < SC::EPI_WARPS) {
+    for_each_tile([&](int lt, int, int, int, bool, bool) { issue_tile(lt); });
+  } else if (POOL && warp < SC::EPI_WARPS) {
+    // ---- epilogue with the fused 3 x 3 / stride-2 MAX pool (POOL): thread = tile row m
+    constexpr int HALF = BN / 2, HP = HALF / 8, PSTR = pool_pstr<BN>(), HB = pool_hand_bytes<BN>();
+    constexpr int HHALF = POW_MAX * HP * 16;  // bytes of one half of a hand-off buffer
+    static_assert(HALF % 16 == 0, "a staged half is whole 16-column accumulator chunks");
+    const int quarter = warp & 3, wg = warp >> 2;
+    const int m = quarter * 32 + lane;
+    const uint32_t lane_base = (uint32_t)(quarter * 32) << 16;
+    const uint32_t stg = smem_u32(sOut) + (uint32_t)(wg * 128 * PSTR);
+    const uint32_t my_row = stg + (uint32_t)(m * PSTR);
+    const uint32_t hand = smem_u32(sHand);
+    const int PJ = g.pool_gp / 8;  // output pieces per half (grouped: the group pitch, pads written 0)
+    const int OPH = g.POH + 2 * g.obd, OPW = g.POW + 2 * g.obd;
+    uint16_t* Yp = reinterpret_cast<uint16_t*>(Y);
+    const float ka = g.lrn_alpha_over_n, kk = g.lrn_k, nb = -g.lrn_beta;
+    for_each_tile([&](int lt, int, int img, int r, bool first, bool last) {
+      if (lt % NWG != wg) return;
+      const int slot = lt % NSLOT, k = lt & 1, kp = k ^ 1;
+      if (lane == 0) mbar_wait_sleep(tfull0 + 8 * slot, (uint32_t)(lt / NSLOT) & 1);
+      __syncwarp();
+      tc_fence_after();
+      const uint32_t tbase = tmem + lane_base + (uint32_t)(slot * 128);
+      // pool the staged half h of the tile's channels.  Hand-off buffer k carries this tile's
+      // partial pool row r (max of conv rows 2r, 2r + 1) to tile lt + 1; each (buffer, half) is
+      // rewritten only after its previous reader (tile lt - 1, same half) has released it and
+      // is published with one arrival, so no barrier phase can run two uses ahead, and the
+      // chain between consecutive tiles is one pool step, not a whole epilogue.  Waits sleep in
+      // lane 0 (spinning warps would take issue slots from the other warpgroups' LRN math).
+      auto pool_half = [&](int h) {
+        asm volatile("bar.sync %0, 128;" ::"r"(1 + wg) : "memory");  // half h staged by the warpgroup
+        if (lane == 0) {
+          mbar_wait_sleep(hempty0 + 8 * (2 * k + h), ((uint32_t)(lt >> 1) & 1) ^ 1);
+          if (lt > 0) mbar_wait_sleep(hfull0 + 8 * (2 * kp + h), (uint32_t)((lt - 1) >> 1) & 1);
+        }
+        __syncwarp();
+        const uint32_t hw = hand + (uint32_t)(k * HB + h * HHALF), hr = hand + (uint32_t)(kp * HB + h * HHALF);
+        const int64_t orow = ((int64_t)img * OPH + (r - 1) + g.obd) * OPW + g.obd;  // pool row r - 1, column 0
+        for (int q = m; q < g.POW * PJ; q += 128) {
+          const int pc = q / PJ, j = q - pc * PJ;
+          uint4 res = make_uint4(0u, 0u, 0u, 0u);
+          if (j < HP) {
+            const uint32_t a = stg + (uint32_t)(2 * pc * PSTR + j * 16);
+            const uint4 va = hmax8<BF16>(hmax8<BF16>(lds128(a), lds128(a + PSTR)), lds128(a + 2 * PSTR));
+            const uint32_t b = a + (uint32_t)(g.Ws * PSTR);
+            const uint4 vb = hmax8<BF16>(hmax8<BF16>(lds128(b), lds128(b + PSTR)), lds128(b + 2 * PSTR));
+            if (!last) sts128(hw + (uint32_t)((pc * HP + j) * 16), hmax8<BF16>(va, vb));
+            if (!first) res = hmax8<BF16>(lds128(hr + (uint32_t)((pc * HP + j) * 16)), va);
+          }
+          if (!first) *reinterpret_cast<uint4*>(Yp + (orow + pc) * g.Cpo + h * g.pool_gp + 8 * j) = res;
+        }
+        asm volatile("bar.sync %0, 128;" ::"r"(1 + wg) : "memory");  // staging read, hand-off half written
+        if (m == 0) {
+          mbar_arrive(hfull0 + 8 * (2 * k + h));
+          if (lt > 0) mbar_arrive(hempty0 + 8 * (2 * kp + h));
+        }
+      };
+      auto put_chunk = [&](int i, const float (&o)[16]) {  // 16-bit LRN output -> staged half
+        const int p0 = 2 * (i % (HALF / 16));
+#pragma unroll
+        for (int hh = 0; hh < 2; ++hh)
+          sts128(my_row + (uint32_t)((p0 + hh) * 16),
+                 make_uint4(pack2<BF16>(o[8 * hh], o[8 * hh + 1]), pack2<BF16>(o[8 * hh + 2], o[8 * hh + 3]),
+                            pack2<BF16>(o[8 * hh + 4], o[8 * hh + 5]), pack2<BF16>(o[8 * hh + 6], o[8 * hh + 7])));
+      };
+      // Caffe LRN across the pixel's N channels (the same arithmetic, in the same order, as the
+      // unfused epilogue below and k_tc.cu)
+      const int N = g.N;
+      float bq[16], cur[16], nxt[16];
+      uint32_t rq[16];
+      tmem_ld16(tbase, rq);
+      tmem_wait_ld();
+      lds16(bq, sbias);
+      bias_act16(cur, rq, bq, g.act);
+      if (NCH > 1) tmem_ld16(tbase + 16, rq);
+      float pm2 = 0.f, pm1 = 0.f;
+#pragma unroll 1
+      for (int i = 0; i < NCH; ++i) {
+        if (i + 1 < NCH) {
+          tmem_wait_ld();
+          lds16(bq, sbias + 16 * (i + 1));
+          bias_act16(nxt, rq, bq, g.act);
+          if (16 * (i + 1) + 16 > N) {
+#pragma unroll
+            for (int j = 0; j < 16; ++j) nxt[j] = 16 * (i + 1) + j < N ? nxt[j] : 0.f;
+          }
+          if (i + 2 < NCH) tmem_ld16(tbase + (uint32_t)(16 * (i + 2)), rq);
+        } else {
+#pragma unroll
+          for (int j = 0; j < 16; ++j) nxt[j] = 0.f;
+          // every accumulator column has been read: hand the slot back to the MMA
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive_relaxed(tempty0 + 8 * slot);
+        }
+        float sq[20];
+        sq[0] = pm2;
+        sq[1] = pm1;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const float2 s2 = mul2(make_float2(cur[2 * j], cur[2 * j + 1]), make_float2(cur[2 * j], cur[2 * j + 1]));
+          sq[2 + 2 * j] = s2.x;
+          sq[3 + 2 * j] = s2.y;
+        }
+        {
+          const float2 s2 = mul2(make_float2(nxt[0], nxt[1]), make_float2(nxt[0], nxt[1]));
+          sq[18] = s2.x;
+          sq[19] = s2.y;
+        }
+        float q[18];
+#pragma unroll
+        for (int j = 0; j < 18; ++j) q[j] = sq[j] + sq[j + 1];
+        const float2 ka2 = make_float2(ka, ka), kk2 = make_float2(kk, kk), nb2 = make_float2(nb, nb);
+        float o[16];
+#pragma unroll
+        for (int j = 0; j < 16; j += 2) {
+          const float2 s5 = add2(add2(make_float2(q[j], q[j + 1]), make_float2(q[j + 2], q[j + 3])),
+                                 make_float2(sq[j + 4], sq[j + 5]));
+          const float2 t2 = fma2(ka2, s5, kk2);
+          const float2 l = mul2(nb2, make_float2(lg2_ftz(t2.x), lg2_ftz(t2.y)));
+          const float2 ov = mul2(make_float2(cur[j], cur[j + 1]), make_float2(ex2_ftz(l.x), ex2_ftz(l.y)));
+          o[j] = ov.x;
+          o[j + 1] = ov.y;
+        }
+        pm2 = sq[16];
+        pm1 = sq[17];
+        put_chunk(i, o);
+        if (i % (HALF / 16) == HALF / 16 - 1) pool_half(i / (HALF / 16));
+#pragma unroll
+        for (int j = 0; j < 16; ++j) cur[j] = nxt[j];
+      }
+    });
+  } else if (!POOL && warp < SC::EPI_WARPS) {
     // ---- epilogue: warpgroup wg drains local tiles lt with lt % NWG == wg; thread = one pixel
     const int quarter = warp & 3, wg = warp >> 2;
     const uint32_t lane_base = (uint32_t)(quarter * 32) << 16;
@@ -417,16 +615,16 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
   }
 }
 
-template <int BN, bool BF16, int F, int C0, int KS, bool GATHER>
+template <int BN, bool BF16, int F, int C0, int KS, bool GATHER, bool POOL>
 cudaError_t launch_stem_inst(const StemGeom& g, const CUtensorMap* tmA, const CUtensorMap* tmB, const CUtensorMap* tmY0,
                              const CUtensorMap* tmY1, const float* x, const float* bias, void* Y, cudaStream_t st) {
-  auto kern = stem_conv_kernel<BN, BF16, F, C0, KS, GATHER>;
-  constexpr int smem = stem_smem<BN, KS, GATHER>();
+  auto kern = stem_conv_kernel<BN, BF16, F, C0, KS, GATHER, POOL>;
+  constexpr int smem = stem_smem<BN, KS, GATHER, POOL>();
   static_assert(smem <= 227 * 1024 - BN * 4, "stem kernel shared memory");
   cudaError_t e = ensure_max_smem((const void*)kern, smem);
   if (e != cudaSuccess) return e;
-  const int64_t tiles = ((int64_t)g.Nimg * g.Hs * g.Ws + 127) / 128;
-  const int grid = (int)(tiles < tc_num_sms() ? tiles : tc_num_sms());
+  const int64_t work = POOL ? (int64_t)g.Nimg * g.bands : ((int64_t)g.Nimg * g.Hs * g.Ws + 127) / 128;
+  const int grid = (int)(work < tc_num_sms() ? work : tc_num_sms());
   return launch_pdl(kern, dim3(grid), dim3(StemCfg<GATHER>::THREADS), smem, st, *tmA, *tmB, *tmY0, *tmY1, g, x, bias, Y);
 }
 
@@ -436,18 +634,49 @@ bool stem_supported(int bn, int f, int c0, int ks, int out_pitch) {
   return bn == 96 && out_pitch == 96 && f == 4 && c0 == 3 && ks == 3;
 }
 
+bool stem_pool_supported(int n, int ws, int oh, int ow, int kernel, int stride, int pad, int cpo, int gsz, int gpitch,
+                         int xu) {
+  // tile = two conv rows; pool rows exactly cover the conv rows (no clipped ceil window);
+  // output plain at pitch n, or two groups of n / 2 channels at a group pitch (pads written 0)
+  if (kernel != 3 || stride != 2 || pad != 0 || xu != 1 || 2 * ws > 128 || oh < 3 || ow < 3) return false;
+  if ((oh - 3) % 2 || (ow - 3) % 2 || (ow - 3) / 2 + 1 > POW_MAX || ow > ws) return false;
+  const bool plain = cpo == n && gsz >= n;
+  const bool grouped = gsz == n / 2 && gpitch >= gsz && gpitch % 8 == 0 && cpo == 2 * gpitch;
+  return n == 96 && (plain || grouped);
+}
+
+int stem_pool_bands(int nimg, int poh) {
+  // bands of pool rows per image: minimise the busiest CTA's tiles, ceil(units / SMs) x
+  // (rows per band + 1); ties -> fewer bands (fewer extra tiles)
+  const int sms = tc_num_sms();
+  int best = 1;
+  int64_t best_cost = -1;
+  for (int b = 1; b <= poh; ++b) {
+    const int64_t units = (int64_t)nimg * b;
+    const int64_t cost = ((units + sms - 1) / sms) * ((poh + b - 1) / b + 1);
+    if (best_cost < 0 || cost < best_cost) { best = b; best_cost = cost; }
+  }
+  return best;
+}
+
 cudaError_t launch_stem_conv(const StemGeom& g, int dt, const CUtensorMap* tmA, const CUtensorMap* tmB,
                              const CUtensorMap* tmY0, const CUtensorMap* tmY1, const float* x, const float* bias, void* Y,
                              cudaStream_t st) {
   if (g.Nimg <= 0) return cudaSuccess;
   if (g.N != 96 || (!g.gather && (g.slab_rows < 128 + 2 * g.Ws + 2 || g.slab_rows > ST_SLAB_ROWS)))
     return cudaErrorInvalidValue;
-  if (g.gather) {
-    if (dt == DT_BF16) return launch_stem_inst<96, true, 4, 3, 3, true>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
-    return launch_stem_inst<96, false, 4, 3, 3, true>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
+  if (g.pool) {
+    if (g.gather || g.out_half || !g.epi_lrn || g.bands < 1 || g.bands > g.POH || g.POW > POW_MAX || 2 * g.Ws > 128)
+      return cudaErrorInvalidValue;
+    if (dt == DT_BF16) return launch_stem_inst<96, true, 4, 3, 3, false, true>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
+    return launch_stem_inst<96, false, 4, 3, 3, false, true>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
   }
-  if (dt == DT_BF16) return launch_stem_inst<96, true, 4, 3, 3, false>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
-  return launch_stem_inst<96, false, 4, 3, 3, false>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
+  if (g.gather) {
+    if (dt == DT_BF16) return launch_stem_inst<96, true, 4, 3, 3, true, false>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
+    return launch_stem_inst<96, false, 4, 3, 3, true, false>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
+  }
+  if (dt == DT_BF16) return launch_stem_inst<96, true, 4, 3, 3, false, false>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
+  return launch_stem_inst<96, false, 4, 3, 3, false, false>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
 }
 
 }  // namespace djinn

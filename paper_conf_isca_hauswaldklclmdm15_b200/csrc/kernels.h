@@ -195,8 +195,16 @@ struct StemGeom {
   int act, epi_lrn, out_half;
   int gather, slab_rows;
   float lrn_alpha_over_n, lrn_beta, lrn_k;
+  // pool = 1: the following 3 x 3 / stride-2 MAX pool is fused (requires epi_lrn, !gather,
+  // !out_half): Y is the pooled tensor [Nimg][POH + 2 obd][POW + 2 obd][Cpo] (the border is
+  // never written), channel c of half h = c / (N / 2) at h * pool_gp + c % (N / 2), the rest of
+  // each half's pool_gp channels written 0; bands = pool-row bands per image (stem_pool_bands)
+  int pool, POH, POW, bands, Cpo, pool_gp, obd;
 };
 bool stem_supported(int bn, int f, int c0, int ks, int out_pitch);
+bool stem_pool_supported(int n, int ws, int oh, int ow, int kernel, int stride, int pad, int cpo, int gsz, int gpitch,
+                         int xu);
+int stem_pool_bands(int nimg, int poh);
 cudaError_t launch_stem_conv(const StemGeom& g, int dt, const CUtensorMap* tmA, const CUtensorMap* tmB,
                              const CUtensorMap* tmY0, const CUtensorMap* tmY1, const float* x, const float* bias, void* Y,
                              cudaStream_t st);

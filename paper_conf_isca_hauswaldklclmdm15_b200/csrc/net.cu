@@ -884,7 +884,7 @@ void Net::build(const std::string& desc) {
   // DESIGN.md sec 5).  DJINN_STEM=0: the generic slab GEMM.
   {
     const char* se = getenv("DJINN_STEM");
-    const int smode = se ? atoi(se) : 2;
+    const int smode = se ? atoi(se) : 3;
     if (f16 && smode > 0 && ops.size() > 1 && ops[0].kind == OP_PACK && ops[0].xform == 1 &&
         ops[1].kind == OP_GEMM && ops[1].xform == 1) {
       Op& c = ops[1];
@@ -900,6 +900,18 @@ void Net::build(const std::string& desc) {
         ops[0].fused = smode == 1 ? 1 : 0;
         c.out.hx = ops[2].in.hx = g.H - g.OH;
         c.out.wx = ops[2].in.wx = g.W - g.OW;
+        // DJINN_STEM=3 (default): the MAX pool runs in the first-layer kernel's epilogue (its
+        // output goes straight to the pool's output tensor; the conv output never reaches HBM)
+        Op& pl = ops[2];
+        if (smode == 3 && g.epi_lrn && stem_pool_supported(g.N, g.W, g.OH, g.OW, pl.kernel, pl.stride, pl.pad, pl.out.Cp,
+                                                           pl.out.gsz, pl.out.gpitch, pl.out.xu) &&
+            pl.out.H == (g.OH - 3) / 2 + 1 && pl.out.W == (g.OW - 3) / 2 + 1 && pl.out.hx == 0 && pl.out.wx == 0) {
+          c.stem_pool = 1;
+          pl.fused = 1;
+          c.name += "+" + pl.name;
+          c.out = pl.out;
+          c.out_buf = pl.out_buf;
+        }
       }
     }
   }
@@ -965,7 +977,7 @@ void Net::build(const std::string& desc) {
       }
       case OP_LRN: o.bytes_row = 2 * in_e * es; break;
       case OP_LRNPOOL: o.bytes_row = in_e * es + out_e * es; break;
-      case OP_POOL: o.bytes_row = in_e * es + out_e * es; break;
+      case OP_POOL: o.bytes_row = o.fused ? 0.0 : in_e * es + out_e * es; break;
       case OP_SOFTMAX: o.bytes_row = 2.0 * in_e * 4; break;
     }
   }
@@ -1211,7 +1223,7 @@ Workspace* Net::workspace(cudaStream_t st) {
   w->tmY1.resize(ops.size());
   for (size_t i = 0; i < ops.size(); ++i) {
     const Op& o = ops[i];
-    if (!o.stem) continue;
+    if (!o.stem || o.stem_pool) continue;
     // output: the virtual grid [rows * Hs * Ws][Cp]; boxes of 32 pixels x 64 / 32 channels
     const int Cp = o.out.Cp, odt = o.g.out_half ? DT_F16 : dt;
     uint64_t dims[2] = {(uint64_t)Cp, (uint64_t)max_rows * (o.out.H + o.out.hx) * (o.out.W + o.out.wx)};
@@ -1420,6 +1432,14 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
             sg.lrn_alpha_over_n = g.lrn_alpha_over_n; sg.lrn_beta = g.lrn_beta; sg.lrn_k = g.lrn_k;
             sg.gather = o.stem == 1;
             sg.slab_rows = g.slab_rows;
+            if (o.stem_pool) {
+              sg.pool = 1;
+              sg.POH = o.out.H; sg.POW = o.out.W;
+              sg.bands = stem_pool_bands(sg.Nimg, sg.POH);
+              sg.Cpo = o.out.Cp;
+              sg.pool_gp = o.out.gsz >= g.N ? g.N / 2 : o.out.gpitch;
+              sg.obd = o.out.bdr;
+            }
             e = launch_stem_conv(sg, dt, &w->tmA[i], &o.tmB, &w->tmY0[i], &w->tmY1[i], src, (const float*)(ar + o.b_off),
                                  Y, st);
           } else if (dt == DT_F32)
@@ -1451,6 +1471,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
                          o.alpha, o.beta, o.lrn_k, dt, st);
           break;
         case OP_POOL:
+          if (o.fused) { skipped = true; break; }  // in the first-layer kernel's epilogue
           if (dt != DT_F32 && o.is_max && o.kernel <= o.stride + 1)
             e = launch_pool_remap(w->buf[o.in_buf], w->buf[o.out_buf], n, o.in.C, o.in.Cp, o.in.gsz, o.in.gpitch,
                                   o.in.H, o.in.W, o.in.H + o.in.hx, o.in.W + o.in.wx, o.out.H, o.out.W, o.kernel,
@@ -1521,7 +1542,8 @@ std::string Net::plan_string() const {
                                                   std::to_string(o.g.bn) : std::string())
         << (o.ksplit > 1 ? " split-K=" + std::to_string(o.ksplit) + "x" + std::to_string(o.kpb) : std::string())
         << (o.stem == 1 ? " stem(fp32 input, fused pack, resident B, TMA-store epilogue)" : "")
-        << (o.stem == 2 ? " stem(TMA slab, resident B, TMA-store epilogue)" : "")
+        << (o.stem == 2 && !o.stem_pool ? " stem(TMA slab, resident B, TMA-store epilogue)" : "")
+        << (o.stem_pool ? " stem(TMA slab, resident B, LRN + 3x3/2 max pool in the epilogue)" : "")
         << (o.g.epi_lrn ? " lrn-epilogue" : "") << (o.g.out_f32 ? " fp32-out" : "") << (o.g.out_half ? " fp16-out" : "") << "]";
     if (o.kind == OP_PACK && o.embed) s << " [embedding window " << o.eg.window << " tables " << o.eg.T << " D " << o.eg.D << "]";
     if (o.kind != OP_GEMM && o.fused) s << " [fused]";

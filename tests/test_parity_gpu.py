@@ -294,15 +294,18 @@ net.close()
 """
 
 
-@pytest.mark.parametrize("mode", ["1", "2"])
-@pytest.mark.parametrize("prec,n,start", [("fp16", 7, 0), ("bf16", 3, 11), ("fp16", 130, 5)])
+@pytest.mark.parametrize("mode", ["1", "2", "3"])
+@pytest.mark.parametrize("prec,n,start", [("fp16", 7, 0), ("bf16", 3, 11), ("fp16", 130, 5), ("fp16", 149, 2)])
 def test_stem_conv_equals_pack_plus_slab_gemm_bitwise(mode, prec, n, start, tmp_path):
-    """IMC conv1+norm1 as the first-layer kernel with a resident filter bank and a TMA-store
-    epilogue over the virtual grid -- its slab gathered from the fp32 images (DJINN_STEM=1) or
-    loaded from the packed tensor by TMA (2, the default) -- and as the generic slab GEMM
-    (DJINN_STEM=0) give bitwise-equal logits: the same 16-bit operands reach the same MMAs in
-    the same order, and the epilogue arithmetic is the same.  n = 7 / 3 / 130 images: tiles
-    that straddle image boundaries and a ragged last tile."""
+    """IMC conv1+norm1 as the first-layer kernel with a resident filter bank -- its slab
+    gathered from the fp32 images (DJINN_STEM=1), loaded from the packed tensor by TMA with a
+    TMA-store epilogue over the virtual grid (2), or with pool1 fused into the epilogue (3, the
+    default: two conv rows per tile, the partial pool row handed to the next tile) -- and the
+    generic slab GEMM + separate pool (DJINN_STEM=0) give bitwise-equal logits: the same 16-bit
+    operands reach the same MMAs in the same order, the epilogue arithmetic is the same, and a
+    max reorders nothing.  n = 7 / 3 / 130 / 149 images: tiles that straddle image boundaries, a
+    ragged last tile, pool-row bands splitting images (3, 7 images), one image per CTA (130) and
+    CTAs with two images (149)."""
     import os
     import subprocess
     import sys
@@ -316,6 +319,7 @@ def test_stem_conv_equals_pack_plus_slab_gemm_bitwise(mode, prec, n, start, tmp_
         plans.append(r.stdout)
         outs.append(np.load(f))
     assert "stem(" in plans[0] and "stem(" not in plans[1], plans
+    assert ("max pool in the epilogue" in plans[0]) == (mode == "3"), plans
     assert np.array_equal(outs[0], outs[1])
 
 
