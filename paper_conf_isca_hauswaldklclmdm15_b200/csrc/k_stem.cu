@@ -232,10 +232,16 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
   const uint32_t idesc = idesc_f16<BN, BF16, 1>();
   const uint64_t hi = sdesc(0, 128);
   const uint32_t sB16 = (smem_u32(sB) & 0x3FFFFu) >> 4, slab16 = (smem_u32(sSlab) & 0x3FFFFu) >> 4;
+  long long m_te = 0, m_sf = 0, m0 = 0;
+  (void)m0;
   auto issue_tile = [&](int lt) {
     const int slot = lt % NSLOT, sb = lt & 1;
+    SST(m0);
     mbar_wait_sleep(tempty0 + 8 * slot, ((uint32_t)(lt / NSLOT) & 1) ^ 1);
+    SACC(m_te, m0);
+    SST(m0);
     mbar_wait(sfull0 + 8 * sb, (uint32_t)(lt >> 1) & 1);
+    SACC(m_sf, m0);
     tc_fence_after();
     if (elect_one()) {
       const uint32_t d = tmem + (uint32_t)(slot * 128);
@@ -321,6 +327,9 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
     mbar_wait(bfull, 0);
     tc_fence_after();
     for_each_tile([&](int lt, int, int, int, bool, bool) { issue_tile(lt); });
+#ifdef DJINN_STEM_STATS
+    if (blockIdx.x == 0 && lane == 0) printf("[stem mma] wait tempty %lld sfull %lld\n", m_te, m_sf);
+#endif
   } else if (POOL && warp < SC::EPI_WARPS) {
     // ---- epilogue with the fused 3 x 3 / stride-2 MAX pool (POOL): thread = tile row m
     constexpr int HALF = BN / 2, HP = HALF / 8, PSTR = pool_pstr<BN>(), HB = pool_hand_bytes<BN>();
@@ -336,11 +345,16 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
     const int OPH = g.POH + 2 * g.obd, OPW = g.POW + 2 * g.obd;
     uint16_t* Yp = reinterpret_cast<uint16_t*>(Y);
     const float ka = g.lrn_alpha_over_n, kk = g.lrn_k, nb = -g.lrn_beta;
+    long long p_wait = 0, p_hw = 0, p_pool = 0, p_tot = 0, p0 = 0, p1 = 0, p2 = 0;
+    (void)p0; (void)p1; (void)p2;
     for_each_tile([&](int lt, int, int img, int r, bool first, bool last) {
       if (lt % NWG != wg) return;
       const int slot = lt % NSLOT, k = lt & 1, kp = k ^ 1;
+      SST(p2);
+      SST(p0);
       if (lane == 0) mbar_wait_sleep(tfull0 + 8 * slot, (uint32_t)(lt / NSLOT) & 1);
       __syncwarp();
+      SACC(p_wait, p0);
       tc_fence_after();
       const uint32_t tbase = tmem + lane_base + (uint32_t)(slot * 128);
       // pool the staged half h of the tile's channels.  Hand-off buffer k carries this tile's
@@ -350,12 +364,15 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
       // chain between consecutive tiles is one pool step, not a whole epilogue.  Waits sleep in
       // lane 0 (spinning warps would take issue slots from the other warpgroups' LRN math).
       auto pool_half = [&](int h) {
+        SST(p1);
         asm volatile("bar.sync %0, 128;" ::"r"(1 + wg) : "memory");  // half h staged by the warpgroup
+        SST(p0);
         if (lane == 0) {
           mbar_wait_sleep(hempty0 + 8 * (2 * k + h), ((uint32_t)(lt >> 1) & 1) ^ 1);
           if (lt > 0) mbar_wait_sleep(hfull0 + 8 * (2 * kp + h), (uint32_t)((lt - 1) >> 1) & 1);
         }
         __syncwarp();
+        SACC(p_hw, p0);
         const uint32_t hw = hand + (uint32_t)(k * HB + h * HHALF), hr = hand + (uint32_t)(kp * HB + h * HHALF);
         const int64_t orow = ((int64_t)img * OPH + (r - 1) + g.obd) * OPW + g.obd;  // pool row r - 1, column 0
         for (int q = m; q < g.POW * PJ; q += 128) {
@@ -376,6 +393,7 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
           mbar_arrive(hfull0 + 8 * (2 * k + h));
           if (lt > 0) mbar_arrive(hempty0 + 8 * (2 * kp + h));
         }
+        SACC(p_pool, p1);
       };
       auto put_chunk = [&](int i, const float (&o)[16]) {  // 16-bit LRN output -> staged half
         const int p0 = 2 * (i % (HALF / 16));
@@ -451,7 +469,13 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
 #pragma unroll
         for (int j = 0; j < 16; ++j) cur[j] = nxt[j];
       }
+      SACC(p_tot, p2);
     });
+#ifdef DJINN_STEM_STATS
+    if (blockIdx.x == 0 && lane == 0)
+      printf("[stem pool-epi warp %d] total %lld tfull-wait %lld pool(incl hand-off) %lld hand-off wait %lld\n", warp,
+             p_tot, p_wait, p_pool, p_hw);
+#endif
   } else if (!POOL && warp < SC::EPI_WARPS) {
     // ---- epilogue: warpgroup wg drains local tiles lt with lt % NWG == wg; thread = one pixel
     const int quarter = warp & 3, wg = warp >> 2;

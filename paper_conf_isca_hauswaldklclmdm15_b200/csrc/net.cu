@@ -966,13 +966,14 @@ void Net::build(const std::string& desc) {
         if (g.mode == GM_DENSE) kreal = in_e;
         else if (g.mode == GM_LC) kreal = (double)o.orig_k * o.orig_k * oin.C;
         else kreal = (double)o.orig_k * o.orig_k * (oin.C / (g.zf > 1 ? g.zf : g.Z));
-        o.flops_row = 2.0 * out_e * kreal;
+        // a fused pool (stem_pool) makes o.out the pooled tensor: the GEMM's work is the conv's
+        const double gemm_e = o.stem_pool ? (double)g.N * g.OH * g.OW : out_e;
+        o.flops_row = 2.0 * gemm_e * kreal;
         o.bytes_row = in_e * (o.stem == 1 ? 4.0 : es) + out_e * (g.out_f32 ? 4.0 : es);  // stem 1 reads the fp32 images
         const double nb = g.mode == GM_DENSE ? g.N : (double)g.Z * g.bias_zstride;
         o.weight_bytes = (g.mode == GM_LC ? (double)g.Z * g.N * kreal
                                           : (g.mode == GM_CONV ? (double)o.out.C * kreal : (double)g.N * kreal)) * es +
                          nb * 4;
-        if (g.mode == GM_CONV && g.zf > 1) o.flops_row = 2.0 * out_e * kreal;
         break;
       }
       case OP_LRN: o.bytes_row = 2 * in_e * es; break;
