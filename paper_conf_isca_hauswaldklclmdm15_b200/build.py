@@ -12,7 +12,7 @@ ROOT = os.path.dirname(HERE)
 VARIANT = os.environ.get("DJINN_BUILD_VARIANT", "")          # "stats": role-timing instrumentation
 LIB = os.path.join(HERE, "libdjinn%s.so" % ("_" + VARIANT if VARIANT else ""))
 OBJ = os.path.join(HERE, "build" + ("_" + VARIANT if VARIANT else ""))
-SOURCES = ["api.cu", "net.cu", "batcher.cu", "k_misc.cu", "k_simt.cu", "k_tc.cu", "k_stem.cu", "k_mlp.cu"]
+SOURCES = ["api.cu", "net.cu", "batcher.cu", "k_misc.cu", "k_simt.cu", "k_tc.cu", "k_stem.cu", "k_mlp.cu", "k_smx.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "-I", os.path.join(ROOT, "include")] + \

@@ -102,6 +102,13 @@ int djinn_load_net(const char* desc, size_t desc_len, const float* weights, size
       uint32_t box[3] = {64, (uint32_t)(o.bn / o.g.cg), 1};
       djinn::encode_tmap(&o.tmB, n.dt, (uint8_t*)n.arena + o.w_off, 3, dims, strides, box);
     }
+    for (djinn::Op& o : n.ops) {  // dense + softmax cluster kernel: its B map, if clusters fit
+      if (!o.smx) continue;
+      if (djinn::smx_max_active_clusters(n.dt, o.smx_cl) < 1) { o.smx = 0; continue; }
+      uint64_t dims[2] = {(uint64_t)o.g.Kpad, (uint64_t)o.g.N}, strides[1] = {(uint64_t)o.g.Kpad * 2};
+      uint32_t box[2] = {(uint32_t)djinn::smx_bk(), 256};
+      djinn::encode_tmap(&o.tmBs, n.dt, (uint8_t*)n.arena + o.w_off, 2, dims, strides, box, 2 * djinn::smx_bk());
+    }
     for (size_t i = 0; i < n.ops.size(); ++i) {  // fused MLP: W1 / W2 maps for its own tiles
       djinn::Op& o = n.ops[i];
       if (!o.mlp) continue;

@@ -227,6 +227,22 @@ bool mlp2_supported(const MlpGeom& g);
 cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const CUtensorMap* tmW2, const float* x,
                         const float* b1, const float* b2, void* out, cudaStream_t st);
 
+// --- dense layer + row softmax fused over a thread-block cluster (k_smx.cu; ASR's output
+// layer): z = x W^T + b for M rows x N columns (x: 16-bit [rows][>= Kpad], W: the arena's
+// [N][Kpad]), then mode 0 p = softmax(z) fp32 [M][N], 1 argmax int32 [M], 2 z fp32 [M][N].
+// A cluster of CL CTAs owns 128 rows; CTA r computes columns [r NCW, r NCW + NCW) in its tensor
+// memory.  tmA: 2D {Kpad, rows}, box {32, 128 / CL}, SWIZZLE_64B; tmB: 2D {Kpad, N}, box
+// {32, 256}, SWIZZLE_64B.  smx_plan: CL (power of two <= 16) and NCW for N (false: unsupported).
+struct SmxGeom {
+  int64_t M;
+  int N, Kpad, CL, NCW, out_mode;
+};
+bool smx_plan(int N, int Kpad, int* CL, int* NCW);
+int smx_bk();  // K per pipeline stage (the A / B box width)
+int smx_max_active_clusters(int dt, int CL);
+cudaError_t launch_smx(const SmxGeom& g, int dt, const CUtensorMap* tmA, const CUtensorMap* tmB, const float* bias,
+                       void* out, cudaStream_t st);
+
 // --- split-K reduction: y[m][n] = act(bias[n] + sum_s part[s][m][n]) for n < N, 0 for
 // N <= n < write_cols; part fp32 [S][rows][ppitch]; y 16-bit (dt) or fp32 (out_f32) with row
 // pitch out_pitch.  The partial sums are added in split order (deterministic).

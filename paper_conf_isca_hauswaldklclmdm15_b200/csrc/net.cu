@@ -939,6 +939,25 @@ void Net::build(const std::string& desc) {
       }
     }
   }
+  // A wide last dense layer + softmax (ASR's 8000 senones) as one cluster kernel (k_smx.cu) for
+  // forwards of >= smx_min_rows rows: opt-in (DJINN_SMX=1), because on B200 it is slower than
+  // the persistent tc GEMM + softmax kernel (ASR 8192 frames: 449 vs 311 us).
+  // DJINN_SMX_MIN_ROWS overrides the row threshold.
+  {
+    const char* se = getenv("DJINN_SMX");
+    const size_t L = ops.size();
+    int cl = 0, ncw = 0;
+    if (f16 && se && se[0] == '1' && L >= 2 && ops[L - 1].kind == OP_SOFTMAX && ops[L - 2].kind == OP_GEMM &&
+        !ops[L - 2].mlp && ops[L - 2].g.mode == GM_DENSE && ops[L - 2].g.out_f32 && ops[L - 2].g.act == ACT_NONE &&
+        ops[L - 2].g.Z == 1 && smx_plan(ops[L - 2].g.N, ops[L - 2].g.Kpad, &cl, &ncw)) {
+      Op& o = ops[L - 2];
+      o.smx = 1;
+      o.smx_cl = cl;
+      o.smx_ncw = ncw;
+      const char* mr = getenv("DJINN_SMX_MIN_ROWS");
+      o.smx_min_rows = mr ? atoll(mr) : 1024;
+    }
+  }
   out_elems = cur.C;
   arena_bytes = rupz(arena_off, 1024);
   // Centered sigmoid storage on 16-bit paths: a sigmoid layer feeding a dense layer stores
@@ -979,7 +998,9 @@ void Net::build(const std::string& desc) {
       case OP_LRN: o.bytes_row = 2 * in_e * es; break;
       case OP_LRNPOOL: o.bytes_row = in_e * es + out_e * es; break;
       case OP_POOL: o.bytes_row = o.fused ? 0.0 : in_e * es + out_e * es; break;
-      case OP_SOFTMAX: o.bytes_row = 2.0 * in_e * 4; break;
+      case OP_SOFTMAX:  // in the cluster kernel (smx): no traffic of its own
+        o.bytes_row = (&o != &ops[0] && (&o - 1)->smx) ? 0.0 : 2.0 * in_e * 4;
+        break;
     }
   }
   for (const Op& o : ops) {
@@ -1043,7 +1064,7 @@ void Net::choose_tiles() {
       const int nkb = g.Kpad / 64;
       const int64_t tiles = ((g.M + 127) / 128) * ((g.N + o.bn - 1) / o.bn);
       o.ksplit = 1;
-      if (sk_on && !o.mlp && g.mode == GM_DENSE && o.g.cg == 1 && nkb >= 32 && tiles <= 74) {
+      if (sk_on && !o.mlp && !o.smx && g.mode == GM_DENSE && o.g.cg == 1 && nkb >= 32 && tiles <= 74) {
         const int S = (int)std::min<int64_t>(nkb / 8, 148 / tiles);
         if (S >= 2) {
           o.ksplit = S;
@@ -1220,6 +1241,7 @@ Workspace* Net::workspace(cudaStream_t st) {
     if (pb && cudaMalloc(&w->part, pb) != cudaSuccess) throw Error(DJINN_E_NOMEM, "split-K workspace");
   }
   w->tmA.resize(ops.size());
+  w->tmAs.resize(ops.size());
   w->tmY0.resize(ops.size());
   w->tmY1.resize(ops.size());
   for (size_t i = 0; i < ops.size(); ++i) {
@@ -1243,6 +1265,10 @@ Workspace* Net::workspace(cudaStream_t st) {
         uint64_t strides[1] = {(uint64_t)g.a_pitch * 2};
         uint32_t box[2] = {64, 128};
         encode_tmap(&w->tmA[i], dt, w->buf[o.in_buf], 2, dims, strides, box);
+        if (o.smx) {
+          uint32_t bs[2] = {(uint32_t)smx_bk(), (uint32_t)(128 / o.smx_cl)};
+          encode_tmap(&w->tmAs[i], dt, w->buf[o.in_buf], 2, dims, strides, bs, 2 * smx_bk());
+        }
         continue;
       }
       // NHWC input [max_rows][H][W][Cp] viewed as a 4D tensor {C, W, H, N}
@@ -1385,6 +1411,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
         for (size_t i = 0; i <= (pop < 0 ? ops.size() : 1); ++i) pev.push_back(prof_event());
       }
     }
+    bool smx_done = false;  // the cluster kernel wrote this chunk's outputs (softmax not launched)
     for (size_t i = 0; i < ops.size(); ++i) {
       const Op& o = ops[i];
       cudaError_t e = cudaSuccess;
@@ -1403,6 +1430,18 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
           break;
         case OP_GEMM: {
           if (o.fused) { skipped = true; break; }
+          if (o.smx && n >= o.smx_min_rows) {
+            SmxGeom sg{};
+            sg.M = n;
+            sg.N = o.g.N;
+            sg.Kpad = o.g.Kpad;
+            sg.CL = o.smx_cl;
+            sg.NCW = o.smx_ncw;
+            sg.out_mode = mode;
+            e = launch_smx(sg, dt, &w->tmAs[i], &o.tmBs, (const float*)((const uint8_t*)arena + o.b_off), dst, st);
+            smx_done = true;
+            break;
+          }
           if (o.mlp) {
             MlpGeom mg = o.mg;
             mg.rows = n;
@@ -1487,7 +1526,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
                               o.beta, o.lrn_k, dt, st);
           break;
         case OP_SOFTMAX:
-          if (o.fused) { skipped = true; break; }
+          if (o.fused || smx_done) { skipped = true; break; }
           e = launch_softmax((const float*)w->buf[2], n, (int)out_elems, out_pitch, dst, mode, st);
           break;
       }
@@ -1550,6 +1589,9 @@ std::string Net::plan_string() const {
     if (o.kind != OP_GEMM && o.fused) s << " [fused]";
     if (o.kind == OP_GEMM && o.fused) s << " [fused into the MLP kernel]";
     if (o.mlp) s << " [MLP kernel: whole net in one launch, N1p=" << o.mg.N1p << " K0p=" << o.mg.K0p << " N2p=" << o.mg.N2p << "]";
+    if (o.smx)
+      s << " [+softmax: cluster kernel, " << o.smx_cl << " CTAs x " << o.smx_ncw << " columns per 128 rows, rows >= "
+        << o.smx_min_rows << "]";
     if (o.kind == OP_PACK && o.xform) s << " [" << (o.xform == 1 ? "space-to-depth " : "kx-unroll ") << o.xf << (o.xs > 1 ? " step " + std::to_string(o.xs) : std::string()) << "]";
     s << "\n";
   }

@@ -91,6 +91,12 @@ struct Op {
   int ksplit = 1, kpb = 0, npart = 0;
   MlpGeom mg{};
   CUtensorMap tmW1{}, tmW2{};
+  // dense layer + softmax over a thread-block cluster (k_smx.cu): this GEMM op writes the
+  // probabilities itself when a forward has >= smx_min_rows rows (the softmax op is then not
+  // launched); smx_cl CTAs of smx_ncw columns per 128 rows; tmBs: its own B map (SW64 boxes)
+  int smx = 0, smx_cl = 0, smx_ncw = 0;
+  int64_t smx_min_rows = 0;
+  CUtensorMap tmBs{};
   // SENNA window lookup in place of the pack (embed = 1): see EmbedGeom (kernels.h)
   int embed = 0;
   EmbedGeom eg{};
@@ -123,6 +129,7 @@ struct Workspace {
   cudaEvent_t in_ready[2] = {}, in_free[2] = {}, out_ready[2] = {}, out_free[2] = {};
   int64_t pipe_cs = 0;  // chunk rows of the last host-fed call (slot offsets depend on it)
   std::vector<CUtensorMap> tmA;  // per op (dense gemm) over its input buffer
+  std::vector<CUtensorMap> tmAs;  // per op (smx): the same buffer, 32-K SW64 boxes of 128 / CL rows
   std::vector<CUtensorMap> tmY0, tmY1;  // per op (stem): TMA-store maps over its output buffer
   float* part = nullptr;                 // split-K partial sums (the largest need of any op)
   ~Workspace();
