@@ -20,6 +20,7 @@
 #include "tc_common.cuh"
 #include <cfloat>
 #include <cstdio>
+#include <cstdlib>
 #ifdef DJINN_MLP_STATS
 #define MST(i) if (tid == 0) ts[i] = clock64()
 #else
@@ -29,7 +30,11 @@
 namespace djinn {
 namespace {
 
-constexpr int MLP_THREADS = 256;
+#ifndef DJINN_MLP_THREADS
+#define DJINN_MLP_THREADS 512
+#endif
+constexpr int MLP_THREADS = DJINN_MLP_THREADS;  // 16 warps: 4 per TMEM lane quarter drain layer 1
+constexpr int MLP_CG = MLP_THREADS / 128;        // column groups of the layer-1 epilogue
 constexpr int MLP_WSTAGES = 4;            // W1 ring stages
 constexpr int MLP_WK = 32;                // K columns per W1 stage (SWIZZLE_64B rows)
 
@@ -65,8 +70,16 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   const uint32_t w2full = smem_u32(bars), wfull0 = smem_u32(bars + 1), wempty0 = smem_u32(bars + 5);
   const uint32_t d1full = smem_u32(bars + 9), d2full = smem_u32(bars + 10);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, tid = threadIdx.x;
-  const int64_t row0 = (int64_t)blockIdx.x * 128;
-  const int nrows = (int)(g.rows - row0 < 128 ? g.rows - row0 : 128);
+  // rows of this CTA: rpc <= 128 per CTA (the MMAs stay M = 128; rows >= nrows are never
+  // stored): small services spread over more SMs, so the per-CTA chain is shorter
+  const int rpc = g.rpc > 0 ? g.rpc : 128;
+  const int64_t row0 = (int64_t)blockIdx.x * rpc;
+  const int nrows = (int)(g.rows - row0 < rpc ? g.rows - row0 : rpc);
+  // Input row i of the CTA is GEMM row arow(i) = (i % 4) * 32 + i / 4: the rows are spread over
+  // the four TMEM lane quarters, so every epilogue warp has rows to drain when rpc < 128 (a warp
+  // can only read its own quarter's lanes).  Rows arow(i) for i >= nrows are never stored.
+  auto arow = [](int i) { return ((i & 3) << 5) | (i >> 2); };
+  const int nrows4 = (nrows + 3) & ~3;  // input rows loaded (whole quarters' worth of rows)
   const int nkw = g.K0p / MLP_WK;  // W1 ring blocks
 
   if (tid == 0) {
@@ -116,7 +129,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
     // 4 rows per warp iteration with all their loads in flight before any is used (a row at a
     // time serialised ~80 L2 round trips per warp: 12.5 us of the kernel's 29 us, B200)
     constexpr int RB = 4, KMAX = 384 / 64;  // rows per batch; lane pairs per row (K0p <= 384)
-    for (int rb = warp * RB; rb < 128; rb += (MLP_THREADS / 32) * RB) {
+    for (int rb = warp * RB; rb < nrows4; rb += (MLP_THREADS / 32) * RB) {
       float v[RB][KMAX][2];
 #pragma unroll
       for (int i = 0; i < RB; ++i) {
@@ -131,7 +144,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
       }
 #pragma unroll
       for (int i = 0; i < RB; ++i) {
-        const int r = rb + i;
+        const int r = arow(rb + i);
 #pragma unroll
         for (int j = 0; j < KMAX; ++j) {
           const int k = lane * 2 + 64 * j;
@@ -185,10 +198,10 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
     if (lane == 0) mbar_wait(d1full, 0);
     __syncwarp();
     tc_fence_after();
-    const int quarter = warp & 3, half = warp >> 2;
+    const int quarter = warp & 3, cgi = warp >> 2;
     const int r = quarter * 32 + lane;
     const uint32_t tb = tmem + ((uint32_t)(quarter * 32) << 16);
-    const int nch = g.N1p / 16, c0 = half ? (nch + 1) / 2 : 0, c1 = half ? nch : (nch + 1) / 2;
+    const int nch = g.N1p / 16, c0 = cgi * nch / MLP_CG, c1 = (cgi + 1) * nch / MLP_CG;
     uint8_t* a2 = sA;
     // chunk ci: bias + activation -> 16-bit -> A2 (two 16-byte pieces)
     auto emit = [&](int ci, const uint32_t (&rq)[16]) {
@@ -208,7 +221,8 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
       }
     };
     // two chunks per step: the second one's TMEM load is in flight while the first is converted
-    for (int ci = c0; ci < c1; ci += 2) {
+    // (warps whose 32 rows are all past nrows have nothing to produce)
+    for (int ci = c0; ci < c1 && quarter < nrows; ci += 2) {
       uint32_t ra[16], rb2[16];
       tmem_ld16(tb + (uint32_t)(ci * 16), ra);
       if (ci + 1 < c1) tmem_ld16(tb + (uint32_t)((ci + 1) * 16), rb2);
@@ -217,7 +231,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
       if (ci + 1 < c1) emit(ci + 1, rb2);
     }
     // zero K columns [N1p, K1p) of A2 (W2 is zero there too; 0 * garbage could be NaN)
-    for (int k = g.N1p + 8 * half; k < g.K1p; k += 16) {
+    for (int k = g.N1p + 8 * cgi; k < g.K1p && quarter < nrows; k += 8 * MLP_CG) {
       const int kk = k & 63;
       *reinterpret_cast<uint4*>(a2 + (k >> 6) * (128 * 128) + r * 128 + (((kk >> 3) ^ (r & 7)) << 4)) = make_uint4(0, 0, 0, 0);
     }
@@ -249,12 +263,12 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   // coalesced stores of the probabilities / logits; argmax ties -> lowest index
   float* stg = reinterpret_cast<float*>(sA);  // A's space: layer 2's MMAs have completed
   const int N2 = g.N2, sp = N2 + 1;           // odd pitch: conflict-free column writes
-  if (warp < 4) {
+  if (warp < 4 && warp < nrows) {
     if (lane == 0) mbar_wait(d2full, 0);
     __syncwarp();
     MST(9);
     tc_fence_after();
-    const int r = warp * 32 + lane;
+    const int r = 4 * lane + warp;  // the input row of TMEM lane warp * 32 + lane
     const uint32_t tb = d2 + ((uint32_t)(warp * 32) << 16);
     const int nch = g.N2p / 16;
     uint32_t rq[4][16];
@@ -268,37 +282,46 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
 #pragma unroll
         for (int j = 0; j < 16; ++j) {
           const int c = ci * 16 + j;
-          if (c < N2) stg[r * sp + c] = __uint_as_float(rq[ci][j]) + sb2[c];
+          if (c < N2 && r < nrows) stg[r * sp + c] = __uint_as_float(rq[ci][j]) + sb2[c];
         }
       }
   }
   __syncthreads();
   MST(10);
-  // two threads per row (interleaved columns) for the max / exp / sum, in place in shared memory
+  // TPR threads per row (interleaved columns; 2 / 4 / 8 as fewer rows leave threads free) for the
+  // max / exp / sum, in place in shared memory; shuffles stay within the row's aligned lane group
   {
-    const int r = tid >> 1, h = tid & 1;
+    const int rows_max = MLP_THREADS / 2;  // rows covered at 2 threads per row
+    const int lt = nrows > rows_max / 2 ? 1 : (nrows > rows_max / 4 ? 2 : (nrows > rows_max / 8 ? 3 : 4)), TPR = 1 << lt;
+    const int r = tid >> lt, h = tid & (TPR - 1);
+    const bool live = r < nrows;
     float* zr = stg + r * sp;
     float m = -FLT_MAX;
     int mi = 0x7fffffff;
-    for (int c = h; c < N2; c += 2) {
-      const float v = zr[c];
-      if (v > m || (v == m && c < mi)) { m = v; mi = c; }
+    if (live)
+      for (int c = h; c < N2; c += TPR) {
+        const float v = zr[c];
+        if (v > m || (v == m && c < mi)) { m = v; mi = c; }
+      }
+    for (int o = 1; o < TPR; o <<= 1) {
+      const float m2 = __shfl_xor_sync(0xffffffffu, m, o);
+      const int i2 = __shfl_xor_sync(0xffffffffu, mi, o);
+      if (m2 > m || (m2 == m && i2 < mi)) { m = m2; mi = i2; }
     }
-    const float m2 = __shfl_xor_sync(0xffffffffu, m, 1);
-    const int i2 = __shfl_xor_sync(0xffffffffu, mi, 1);
-    if (m2 > m || (m2 == m && i2 < mi)) { m = m2; mi = i2; }
     if (g.out_mode == 1) {
-      if (h == 0 && r < nrows) reinterpret_cast<int*>(out)[row0 + r] = mi;
+      if (h == 0 && live) reinterpret_cast<int*>(out)[row0 + r] = mi;
     } else if (g.out_mode == 0) {
       float sum = 0.f;
-      for (int c = h; c < N2; c += 2) {
-        const float e = expf(zr[c] - m);
-        zr[c] = e;
-        sum += e;
-      }
-      sum += __shfl_xor_sync(0xffffffffu, sum, 1);
+      if (live)
+        for (int c = h; c < N2; c += TPR) {
+          const float e = expf(zr[c] - m);
+          zr[c] = e;
+          sum += e;
+        }
+      for (int o = 1; o < TPR; o <<= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
       const float inv = 1.f / sum;
-      for (int c = h; c < N2; c += 2) zr[c] *= inv;
+      if (live)
+        for (int c = h; c < N2; c += TPR) zr[c] *= inv;
     }
   }
   if (g.out_mode != 1) {
@@ -333,6 +356,18 @@ int mlp2_smem(const MlpGeom& g) {
   return 1024 + abytes + ((MLP_WSTAGES * g.N1p * MLP_WK * 2 + 1023) & ~1023) + KB1 * g.N2p * 128 + 12 * 8 + 16;
 }
 
+int mlp2_rows_per_cta(int64_t rows) {
+  static const int env = [] {
+    const char* e = getenv("DJINN_MLP_RPC");
+    return e ? atoi(e) : 0;
+  }();
+  if (env > 0) return env;
+  const int64_t sms = tc_num_sms();
+  for (int rpc = 32; rpc < 128; rpc *= 2)
+    if ((rows + rpc - 1) / rpc <= sms) return rpc;
+  return 128;
+}
+
 bool mlp2_supported(const MlpGeom& g) {
   return g.K0p % 64 == 0 && g.K1p % 64 == 0 && g.N1p % 16 == 0 && g.N1p >= g.N1 && g.N1p <= 512 &&
          (g.N1p <= 256 || (g.N1p - 256) % 16 == 0) && g.N1p / 2 <= 256 && g.K1p >= g.N1p && g.N2p % 16 == 0 &&
@@ -345,7 +380,9 @@ cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const
   if (g.rows <= 0) return cudaSuccess;
   if (!mlp2_supported(g)) return cudaErrorInvalidValue;
   const int smem = mlp2_smem(g);
-  const unsigned grid = (unsigned)((g.rows + 127) / 128);
+  const int rpc = g.rpc > 0 ? g.rpc : 128;
+  if (rpc > 128 || rpc % 8) return cudaErrorInvalidValue;
+  const unsigned grid = (unsigned)((g.rows + rpc - 1) / rpc);
   // the max-dynamic-smem attribute is set once per (device, kernel): a cudaFuncSetAttribute per
   // call was a measurable part of the ~10 us host cost of a small service's forward
   cudaError_t e = ensure_max_smem(dt == DT_BF16 ? (const void*)mlp2_kernel<true> : (const void*)mlp2_kernel<false>,

@@ -221,7 +221,11 @@ struct MlpGeom {
   int K1p;             // W2's Kpad (layer 1 outputs padded to 64)
   int N2, N2p;         // logits, padded to 16 (<= 64)
   int act1, out_mode;
+  int rpc;             // rows per CTA (<= 128, multiple of 8; 0 = 128)
 };
+// rows per CTA for a forward of `rows` rows: the smallest of 128 / 64 / 32 that keeps the grid
+// within one wave of SMs (DJINN_MLP_RPC overrides)
+int mlp2_rows_per_cta(int64_t rows);
 int mlp2_smem(const MlpGeom& g);
 bool mlp2_supported(const MlpGeom& g);
 cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const CUtensorMap* tmW2, const float* x,

@@ -613,10 +613,16 @@ void Net::build(const std::string& desc) {
           os.C = L.num_output; os.H = OH; os.W = OW;
           os = layout_for(i + 1, os);
           int XB = 1;
+          static const int kx_xb_env = [] {  // DJINN_KX_XB caps the x-block (experiments)
+            const char* e = getenv("DJINN_KX_XB");
+            return e ? atoi(e) : 0;
+          }();
+          const int kx_cap = kx_xb_env > 0 ? kx_xb_env : 8;
           if (os.gsz >= os.C && os.Cp <= 64)
             for (int xbc = 8; xbc >= 2; xbc /= 2)
-              if ((k + xbc - 1) * cur.C <= 64 && xbc * os.Cp <= 256) { XB = xbc; break; }
+              if (xbc <= kx_cap && (k + xbc - 1) * cur.C <= 64 && xbc * os.Cp <= 256) { XB = xbc; break; }
           const int U = k + XB - 1, OWb = (OW + XB - 1) / XB;
+          creal = U * cur.C;  // real channels of a packed tap (the rest of its 64 are zero)
           pk.xform = o.xform = 2;
           pk.xf = o.xf = U;
           pk.xs = o.xs = XB;
@@ -733,7 +739,7 @@ void Net::build(const std::string& desc) {
           // conv2's groups): the 4th 16-channel K sub-step multiplies zero weights, so the
           // kernel variant with 3 MMAs per K block skips it (DJINN_KSKIP=0: off)
           const char* ks = getenv("DJINN_KSKIP");
-          g.kv16 = (g.Cgp == 64 && creal > 32 && creal <= 48 && g.kxs == 1 && g.xb <= 1 && !(ks && ks[0] == '0')) ? 3 : 4;
+          g.kv16 = (g.Cgp == 64 && creal > 32 && creal <= 48 && g.kxs == 1 && !(ks && ks[0] == '0')) ? 3 : 4;
         }
       }
       if (!g.slab && o.in.bdr > 0) {  // a bordered input read by im2col: pad-0 conv over the stored grid
@@ -1446,6 +1452,7 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
             MlpGeom mg = o.mg;
             mg.rows = n;
             mg.out_mode = mode;
+            mg.rpc = mlp2_rows_per_cta(n);
             const uint8_t* ar = (const uint8_t*)arena;
             e = launch_mlp2(mg, dt, &o.tmW1, &o.tmW2, src, (const float*)(ar + o.b_off), (const float*)(ar + ops[i + 1].b_off),
                             dst, st);

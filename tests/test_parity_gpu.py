@@ -341,13 +341,16 @@ net.close()
 """
 
 
-@pytest.mark.parametrize("app,prec,n", [("pos", "fp16", 1000), ("chk", "bf16", 4096), ("ner", "fp16", 129),
-                                        ("ner", "bf16", 3000)])
-def test_mlp_kernel_equals_unfused_path(app, prec, n, tmp_path):
+@pytest.mark.parametrize("app,prec,n,rpc", [("pos", "fp16", 1000, ""), ("chk", "bf16", 4096, ""), ("ner", "fp16", 129, ""),
+                                            ("ner", "bf16", 3000, ""), ("pos", "fp16", 4096, "128"),
+                                            ("chk", "fp16", 1001, "64"), ("ner", "fp16", 70, "32"),
+                                            ("pos", "bf16", 5003, "8")])
+def test_mlp_kernel_equals_unfused_path(app, prec, n, rpc, tmp_path):
     """The one-launch window-MLP kernel (pack + l1 + HardTanh + l2 + softmax on chip) and the four
     separate kernels (DJINN_MLP=0) give bitwise-equal logits and argmax -- the same 16-bit
     operands reach the MMAs in the same K order and the epilogues round the same way -- and
-    probabilities equal to the last ulps (the softmax sums in a different order)."""
+    probabilities equal to the last ulps (the softmax sums in a different order).  rpc: rows per
+    CTA forced by DJINN_MLP_RPC (default: chosen by the batch size), ragged last CTAs included."""
     import os
     import subprocess
     import sys
@@ -356,6 +359,8 @@ def test_mlp_kernel_equals_unfused_path(app, prec, n, tmp_path):
     for mlp in ("1", "0"):
         f = str(tmp_path / f"o{mlp}.npz")
         env = dict(os.environ, DJINN_MLP=mlp)
+        if rpc:
+            env["DJINN_MLP_RPC"] = rpc
         r = subprocess.run([sys.executable, "-c", _MLP_CHILD, root, app, prec, str(n), f], env=env, check=True,
                            timeout=600, capture_output=True, text=True)
         plans.append(r.stdout)
