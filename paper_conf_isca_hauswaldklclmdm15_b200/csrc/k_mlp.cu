@@ -43,11 +43,15 @@ __device__ __forceinline__ uint32_t idesc_rt(int n, bool bf16) {  // kind::f16, 
   return (1u << 4) | (ab << 7) | (ab << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
 }
 
-template <bool BF16>
+// AT = false: layer 1's A is built from the fp32 query rows x (the window nets' input);
+// AT = true: A is a 16-bit activation tensor (the tail of a larger net, e.g. DIG's pool2 output)
+// read by TMA (tmA: 2D {K0p, rows}, box {32, 128}, SWIZZLE_64B) through the W1 ring -- each stage
+// carries its 32-column A block beside the W1 block -- and layer 2's A operand reuses the ring.
+template <bool BF16, bool AT>
 __global__ void __launch_bounds__(MLP_THREADS, 1)
-    mlp2_kernel(const __grid_constant__ CUtensorMap tmW1, const __grid_constant__ CUtensorMap tmW2, const MlpGeom g,
-                const float* __restrict__ x, const float* __restrict__ b1, const float* __restrict__ b2,
-                void* __restrict__ out) {
+    mlp2_kernel(const __grid_constant__ CUtensorMap tmW1, const __grid_constant__ CUtensorMap tmW2,
+                const __grid_constant__ CUtensorMap tmA, const MlpGeom g, const float* __restrict__ x,
+                const float* __restrict__ b1, const float* __restrict__ b2, void* __restrict__ out) {
   pdl_trigger();
 #ifdef DJINN_MLP_STATS
   long long ts[12] = {0};
@@ -57,11 +61,14 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int KB0 = g.K0p / 64, KB1 = g.K1p / 64;  // 64-column blocks of the two A operands
-  const int abytes = (KB0 > KB1 ? KB0 : KB1) * 128 * 128;
+  constexpr int ABLK = 128 * MLP_WK * 2;         // AT: one stage's A block (128 rows of 64 B)
   const int wstage = g.N1p * MLP_WK * 2;          // one W1 ring stage (N1p rows of 64 B)
-  uint8_t* sA = smem;                             // A1, then A2
-  uint8_t* sW = sA + abytes;                      // W1 ring
-  uint8_t* sW2 = sW + ((MLP_WSTAGES * wstage + 1023) & ~1023);
+  const int sstride = AT ? ABLK + wstage : wstage;  // ring stage stride
+  const int abytes = AT ? 0 : (KB0 > KB1 ? KB0 : KB1) * 128 * 128;
+  const int ring = (MLP_WSTAGES * sstride + 1023) & ~1023;
+  uint8_t* sW = smem + abytes;                    // W1 ring (AT: A block + W1 block per stage)
+  uint8_t* sA = AT ? sW : smem;                   // A1 (not AT), then A2 (AT: over the drained ring)
+  uint8_t* sW2 = sW + ring;
   uint64_t* bars = reinterpret_cast<uint64_t*>(sW2 + KB1 * g.N2p * 128);
   // bars: w2full, wfull[4], wempty[4], d1full, d2full
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 11);
@@ -78,6 +85,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   // Input row i of the CTA is GEMM row arow(i) = (i % 4) * 32 + i / 4: the rows are spread over
   // the four TMEM lane quarters, so every epilogue warp has rows to drain when rpc < 128 (a warp
   // can only read its own quarter's lanes).  Rows arow(i) for i >= nrows are never stored.
+  // (AT: the TMA rows are contiguous, so GEMM row = input row and rpc is 128)
   auto arow = [](int i) { return ((i & 3) << 5) | (i >> 2); };
   const int nrows4 = (nrows + 3) & ~3;  // input rows loaded (whole quarters' worth of rows)
   const int nkw = g.K0p / MLP_WK;  // W1 ring blocks
@@ -105,13 +113,17 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
   // weights: W2 whole, and the first ring stages of W1 (never written by earlier kernels)
-  auto load_w1 = [&](int kb) {
+  auto load_w1 = [&](int kb) {  // (AT: the stage's barrier also expects its A block, load_a)
     const int s = kb % MLP_WSTAGES;
-    const uint32_t dst = smem_u32(sW) + (uint32_t)(s * wstage);
-    mbar_arrive_expect_tx(wfull0 + 8 * s, (uint32_t)wstage);
+    const uint32_t dst = smem_u32(sW) + (uint32_t)(s * sstride + (AT ? ABLK : 0));
+    mbar_arrive_expect_tx(wfull0 + 8 * s, (uint32_t)(wstage + (AT ? ABLK : 0)));
     const int half = g.N1p / 2;  // two boxes of N1p / 2 rows
     tma_2d(dst, &tmW1, wfull0 + 8 * s, kb * MLP_WK, 0);
     tma_2d(dst + (uint32_t)(half * MLP_WK * 2), &tmW1, wfull0 + 8 * s, kb * MLP_WK, half);
+  };
+  auto load_a = [&](int kb) {  // AT: rows [row0, row0 + 128) x K columns [32 kb, 32 kb + 32)
+    const int s = kb % MLP_WSTAGES;
+    tma_2d(smem_u32(sW) + (uint32_t)(s * sstride), &tmA, wfull0 + 8 * s, kb * MLP_WK, (int)row0);
   };
   if (tid == 0) {
     mbar_arrive_expect_tx(w2full, (uint32_t)(KB1 * g.N2p * 128));
@@ -121,11 +133,13 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   MST(1);
   pdl_wait();  // the input rows and the output buffer belong to earlier kernels of the stream
   MST(2);
+  if (AT && tid == 0)
+    for (int kb = 0; kb < MLP_WSTAGES && kb < nkw; ++kb) load_a(kb);
 
   // ---- 1. fp32 rows -> 16-bit A1 (K-major, 128B swizzle: element (r, k) of block k / 64 at
   // r * 128 + (((k % 64) / 8) ^ (r % 8)) * 16 + (k % 8) * 2); a warp reads one row's floats
   // contiguously, so the global reads are coalesced
-  {
+  if (!AT) {
     // 4 rows per warp iteration with all their loads in flight before any is used (a row at a
     // time serialised ~80 L2 round trips per warp: 12.5 us of the kernel's 29 us, B200)
     constexpr int RB = 4, KMAX = 384 / 64;  // rows per batch; lane pairs per row (K0p <= 384)
@@ -175,8 +189,9 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
 #pragma unroll
       for (int k = 0; k < MLP_WK / 16; ++k) {
         const int kk = kb * MLP_WK + k * 16;  // first K column of this step
-        const uint64_t ad = hi128 | (uint64_t)(a16 + (uint32_t)((kk >> 6) * (128 * 128 / 16) + ((kk & 63) * 2) / 16));
-        const uint32_t wb = w16 + (uint32_t)(s * (wstage >> 4)) + (uint32_t)(k * 2);
+        const uint64_t ad = AT ? hi64 | (uint64_t)(w16 + (uint32_t)(s * (sstride >> 4)) + (uint32_t)(k * 2))
+                               : hi128 | (uint64_t)(a16 + (uint32_t)((kk >> 6) * (128 * 128 / 16) + ((kk & 63) * 2) / 16));
+        const uint32_t wb = w16 + (uint32_t)(s * (sstride >> 4) + (AT ? ABLK >> 4 : 0)) + (uint32_t)(k * 2);
         mma_f16(tmem, ad, hi64 | (uint64_t)wb, ida, (kb | k) != 0);
         if (nb) mma_f16(tmem + (uint32_t)na, ad, hi64 | (uint64_t)(wb + (uint32_t)((na * 64) >> 4)), idb, (kb | k) != 0);
       }
@@ -188,6 +203,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
     for (int kb = 0; kb + MLP_WSTAGES < nkw; ++kb) {
       mbar_wait(wempty0 + 8 * (kb % MLP_WSTAGES), (uint32_t)(kb / MLP_WSTAGES) & 1);
       load_w1(kb + MLP_WSTAGES);
+      if (AT) load_a(kb + MLP_WSTAGES);
     }
   }
   MST(4);
@@ -222,7 +238,8 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
     };
     // two chunks per step: the second one's TMEM load is in flight while the first is converted
     // (warps whose 32 rows are all past nrows have nothing to produce)
-    for (int ci = c0; ci < c1 && quarter < nrows; ci += 2) {
+    const bool act_rows = AT ? quarter * 32 < nrows : quarter < nrows;  // this warp has rows to drain
+    for (int ci = c0; ci < c1 && act_rows; ci += 2) {
       uint32_t ra[16], rb2[16];
       tmem_ld16(tb + (uint32_t)(ci * 16), ra);
       if (ci + 1 < c1) tmem_ld16(tb + (uint32_t)((ci + 1) * 16), rb2);
@@ -231,7 +248,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
       if (ci + 1 < c1) emit(ci + 1, rb2);
     }
     // zero K columns [N1p, K1p) of A2 (W2 is zero there too; 0 * garbage could be NaN)
-    for (int k = g.N1p + 8 * cgi; k < g.K1p && quarter < nrows; k += 8 * MLP_CG) {
+    for (int k = g.N1p + 8 * cgi; k < g.K1p && act_rows; k += 8 * MLP_CG) {
       const int kk = k & 63;
       *reinterpret_cast<uint4*>(a2 + (k >> 6) * (128 * 128) + r * 128 + (((kk >> 3) ^ (r & 7)) << 4)) = make_uint4(0, 0, 0, 0);
     }
@@ -263,12 +280,12 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   // coalesced stores of the probabilities / logits; argmax ties -> lowest index
   float* stg = reinterpret_cast<float*>(sA);  // A's space: layer 2's MMAs have completed
   const int N2 = g.N2, sp = N2 + 1;           // odd pitch: conflict-free column writes
-  if (warp < 4 && warp < nrows) {
+  if (warp < 4 && (AT ? warp * 32 : warp) < nrows) {
     if (lane == 0) mbar_wait(d2full, 0);
     __syncwarp();
     MST(9);
     tc_fence_after();
-    const int r = 4 * lane + warp;  // the input row of TMEM lane warp * 32 + lane
+    const int r = AT ? warp * 32 + lane : 4 * lane + warp;  // the input row of TMEM lane warp * 32 + lane
     const uint32_t tb = d2 + ((uint32_t)(warp * 32) << 16);
     const int nch = g.N2p / 16;
     uint32_t rq[4][16];
@@ -352,8 +369,9 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
 
 int mlp2_smem(const MlpGeom& g) {
   const int KB0 = g.K0p / 64, KB1 = g.K1p / 64;
-  const int abytes = (KB0 > KB1 ? KB0 : KB1) * 128 * 128;
-  return 1024 + abytes + ((MLP_WSTAGES * g.N1p * MLP_WK * 2 + 1023) & ~1023) + KB1 * g.N2p * 128 + 12 * 8 + 16;
+  const int abytes = g.a_tma ? 0 : (KB0 > KB1 ? KB0 : KB1) * 128 * 128;
+  const int sstride = g.N1p * MLP_WK * 2 + (g.a_tma ? 128 * MLP_WK * 2 : 0);
+  return 1024 + abytes + ((MLP_WSTAGES * sstride + 1023) & ~1023) + KB1 * g.N2p * 128 + 12 * 8 + 16;
 }
 
 int mlp2_rows_per_cta(int64_t rows) {
@@ -371,26 +389,28 @@ int mlp2_rows_per_cta(int64_t rows) {
 bool mlp2_supported(const MlpGeom& g) {
   return g.K0p % 64 == 0 && g.K1p % 64 == 0 && g.N1p % 16 == 0 && g.N1p >= g.N1 && g.N1p <= 512 &&
          (g.N1p <= 256 || (g.N1p - 256) % 16 == 0) && g.N1p / 2 <= 256 && g.K1p >= g.N1p && g.N2p % 16 == 0 &&
-         g.N2p >= g.N2 && g.N2p <= 64 && g.N1c % 16 == 0 && g.N1c >= g.N1p && g.N1c + g.N2p <= 512 &&
+         g.N2p >= g.N2 && g.N2p <= 64 && g.N1c % 16 == 0 && (g.N1c >= g.N1p || g.N1c == 0) &&
+         g.N1c + g.N2p <= 512 && (!g.a_tma || MLP_WSTAGES * (g.N1p + 128) * MLP_WK * 2 >= g.K1p / 64 * 128 * 128) &&
          mlp2_smem(g) <= 227 * 1024 - 3 * 1024;
 }
 
-cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const CUtensorMap* tmW2, const float* x,
-                        const float* b1, const float* b2, void* out, cudaStream_t st) {
+cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const CUtensorMap* tmW2, const CUtensorMap* tmA,
+                        const float* x, const float* b1, const float* b2, void* out, cudaStream_t st) {
   if (g.rows <= 0) return cudaSuccess;
   if (!mlp2_supported(g)) return cudaErrorInvalidValue;
   const int smem = mlp2_smem(g);
   const int rpc = g.rpc > 0 ? g.rpc : 128;
-  if (rpc > 128 || rpc % 8) return cudaErrorInvalidValue;
+  if (rpc > 128 || rpc % 8 || (g.a_tma && rpc != 128)) return cudaErrorInvalidValue;
   const unsigned grid = (unsigned)((g.rows + rpc - 1) / rpc);
   // the max-dynamic-smem attribute is set once per (device, kernel): a cudaFuncSetAttribute per
   // call was a measurable part of the ~10 us host cost of a small service's forward
-  cudaError_t e = ensure_max_smem(dt == DT_BF16 ? (const void*)mlp2_kernel<true> : (const void*)mlp2_kernel<false>,
-                                  227 * 1024 - 3 * 1024);
+  if (g.a_tma && !tmA) return cudaErrorInvalidValue;
+  auto kern = dt == DT_BF16 ? (g.a_tma ? mlp2_kernel<true, true> : mlp2_kernel<true, false>)
+                            : (g.a_tma ? mlp2_kernel<false, true> : mlp2_kernel<false, false>);
+  cudaError_t e = ensure_max_smem((const void*)kern, 227 * 1024 - 3 * 1024);
   if (e != cudaSuccess) return e;
-  if (dt == DT_BF16)
-    return launch_pdl(mlp2_kernel<true>, dim3(grid), dim3(MLP_THREADS), smem, st, *tmW1, *tmW2, g, x, b1, b2, out);
-  return launch_pdl(mlp2_kernel<false>, dim3(grid), dim3(MLP_THREADS), smem, st, *tmW1, *tmW2, g, x, b1, b2, out);
+  return launch_pdl(kern, dim3(grid), dim3(MLP_THREADS), smem, st, *tmW1, *tmW2, g.a_tma ? *tmA : *tmW1, g, x, b1, b2,
+                    out);
 }
 
 }  // namespace djinn

@@ -222,14 +222,16 @@ struct MlpGeom {
   int N2, N2p;         // logits, padded to 16 (<= 64)
   int act1, out_mode;
   int rpc;             // rows per CTA (<= 128, multiple of 8; 0 = 128)
+  int a_tma;           // 1: layer 1's A is a 16-bit tensor [rows][K0p] read by TMA (tmA), x unused;
+                       //    N1c = 0 then lets layer 2 reuse layer 1's TMEM columns
 };
 // rows per CTA for a forward of `rows` rows: the smallest of 128 / 64 / 32 that keeps the grid
 // within one wave of SMs (DJINN_MLP_RPC overrides)
 int mlp2_rows_per_cta(int64_t rows);
 int mlp2_smem(const MlpGeom& g);
 bool mlp2_supported(const MlpGeom& g);
-cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const CUtensorMap* tmW2, const float* x,
-                        const float* b1, const float* b2, void* out, cudaStream_t st);
+cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const CUtensorMap* tmW2, const CUtensorMap* tmA,
+                        const float* x, const float* b1, const float* b2, void* out, cudaStream_t st);
 
 // --- dense layer + row softmax fused over a thread-block cluster (k_smx.cu; ASR's output
 // layer): z = x W^T + b for M rows x N columns (x: 16-bit [rows][>= Kpad], W: the arena's

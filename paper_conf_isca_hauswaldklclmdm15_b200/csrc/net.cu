@@ -944,6 +944,33 @@ void Net::build(const std::string& desc) {
         ops[0].fused = ops[2].fused = ops[3].fused = 1;
       }
     }
+    // The same kernel as the tail of a larger net (DIG's ip1 + ReLU + ip2 + softmax): layer 1
+    // reads the 16-bit activations of the layer before it by TMA (a_tma).
+    const size_t L = ops.size();
+    if (f16 && !(me && me[0] == '0') && L >= 4 && !ops[L - 3].mlp && ops[L - 3].kind == OP_GEMM &&
+        ops[L - 3].g.mode == GM_DENSE && ops[L - 3].in_buf >= 0 && !ops[L - 3].g.out_f32 && !ops[L - 3].g.out_half &&
+        ops[L - 3].g.Z == 1 && ops[L - 2].kind == OP_GEMM && ops[L - 2].g.mode == GM_DENSE && ops[L - 2].g.out_f32 &&
+        ops[L - 2].g.Z == 1 && ops[L - 1].kind == OP_SOFTMAX && ops[L - 4].kind != OP_PACK) {
+      const Op& a = ops[L - 3];
+      const Op& b = ops[L - 2];
+      MlpGeom m{};
+      m.a_tma = 1;
+      m.K0 = a.g.Kpad;
+      m.K0p = a.g.Kpad;
+      m.N1 = a.g.N;
+      m.N1p = rup(m.N1, 16);
+      m.K1p = b.g.Kpad;
+      m.N2 = b.g.N;
+      m.N2p = rup(m.N2, 16);
+      m.N1c = m.N1p + m.N2p <= 512 ? m.N1p : 0;
+      m.act1 = a.g.act;
+      if (a.g.a_pitch <= a.g.Kpad && a.g.a_pitch % 8 == 0 && a.out.Cp <= m.K1p && m.N1p <= 512 && (m.N1p <= 256 || m.N1p % 32 == 0) &&
+          mlp2_supported(m)) {
+        ops[L - 3].mlp = 1;
+        ops[L - 3].mg = m;
+        ops[L - 2].fused = ops[L - 1].fused = 1;
+      }
+    }
   }
   // A wide last dense layer + softmax (ASR's 8000 senones) as one cluster kernel (k_smx.cu) for
   // forwards of >= smx_min_rows rows: opt-in (DJINN_SMX=1), because on B200 it is slower than
@@ -1275,6 +1302,10 @@ Workspace* Net::workspace(cudaStream_t st) {
           uint32_t bs[2] = {(uint32_t)smx_bk(), (uint32_t)(128 / o.smx_cl)};
           encode_tmap(&w->tmAs[i], dt, w->buf[o.in_buf], 2, dims, strides, bs, 2 * smx_bk());
         }
+        if (o.mlp && o.mg.a_tma) {  // the fused MLP tail: 32-column blocks of 128 rows (SW64)
+          uint32_t bs[2] = {32, 128};
+          encode_tmap(&w->tmAs[i], dt, w->buf[o.in_buf], 2, dims, strides, bs, 64);
+        }
         continue;
       }
       // NHWC input [max_rows][H][W][Cp] viewed as a 4D tensor {C, W, H, N}
@@ -1452,10 +1483,10 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
             MlpGeom mg = o.mg;
             mg.rows = n;
             mg.out_mode = mode;
-            mg.rpc = mlp2_rows_per_cta(n);
+            mg.rpc = mg.a_tma ? 128 : mlp2_rows_per_cta(n);
             const uint8_t* ar = (const uint8_t*)arena;
-            e = launch_mlp2(mg, dt, &o.tmW1, &o.tmW2, src, (const float*)(ar + o.b_off), (const float*)(ar + ops[i + 1].b_off),
-                            dst, st);
+            e = launch_mlp2(mg, dt, &o.tmW1, &o.tmW2, mg.a_tma ? &w->tmAs[i] : nullptr, src, (const float*)(ar + o.b_off),
+                            (const float*)(ar + ops[i + 1].b_off), dst, st);
             break;
           }
           GemmGeom g = o.g;
@@ -1595,7 +1626,10 @@ std::string Net::plan_string() const {
     if (o.kind == OP_PACK && o.embed) s << " [embedding window " << o.eg.window << " tables " << o.eg.T << " D " << o.eg.D << "]";
     if (o.kind != OP_GEMM && o.fused) s << " [fused]";
     if (o.kind == OP_GEMM && o.fused) s << " [fused into the MLP kernel]";
-    if (o.mlp) s << " [MLP kernel: whole net in one launch, N1p=" << o.mg.N1p << " K0p=" << o.mg.K0p << " N2p=" << o.mg.N2p << "]";
+    if (o.mlp)
+      s << (o.mg.a_tma ? " [MLP tail kernel: this layer + the next + softmax in one launch, A by TMA, N1p="
+                       : " [MLP kernel: whole net in one launch, N1p=")
+        << o.mg.N1p << " K0p=" << o.mg.K0p << " N2p=" << o.mg.N2p << "]";
     if (o.smx)
       s << " [+softmax: cluster kernel, " << o.smx_cl << " CTAs x " << o.smx_ncw << " columns per 128 rows, rows >= "
         << o.smx_min_rows << "]";

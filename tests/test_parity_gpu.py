@@ -344,13 +344,16 @@ net.close()
 @pytest.mark.parametrize("app,prec,n,rpc", [("pos", "fp16", 1000, ""), ("chk", "bf16", 4096, ""), ("ner", "fp16", 129, ""),
                                             ("ner", "bf16", 3000, ""), ("pos", "fp16", 4096, "128"),
                                             ("chk", "fp16", 1001, "64"), ("ner", "fp16", 70, "32"),
-                                            ("pos", "bf16", 5003, "8")])
+                                            ("pos", "bf16", 5003, "8"), ("dig", "fp16", 1600, ""),
+                                            ("dig", "bf16", 333, "")])
 def test_mlp_kernel_equals_unfused_path(app, prec, n, rpc, tmp_path):
     """The one-launch window-MLP kernel (pack + l1 + HardTanh + l2 + softmax on chip) and the four
     separate kernels (DJINN_MLP=0) give bitwise-equal logits and argmax -- the same 16-bit
     operands reach the MMAs in the same K order and the epilogues round the same way -- and
     probabilities equal to the last ulps (the softmax sums in a different order).  rpc: rows per
-    CTA forced by DJINN_MLP_RPC (default: chosen by the batch size), ragged last CTAs included."""
+    CTA forced by DJINN_MLP_RPC (default: chosen by the batch size), ragged last CTAs included.
+    DIG: the same kernel as the tail of a conv net (ip1 + ReLU + ip2 + softmax, A read by TMA
+    from pool2's 16-bit output, layer 2 reusing layer 1's 512 TMEM columns)."""
     import os
     import subprocess
     import sys
