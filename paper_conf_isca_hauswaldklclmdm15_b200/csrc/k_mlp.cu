@@ -328,14 +328,32 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
     if (g.out_mode == 1) {
       if (h == 0 && live) reinterpret_cast<int*>(out)[row0 + r] = mi;
     } else if (g.out_mode == 0) {
-      float sum = 0.f;
+      // The row sum in an order that does not depend on TPR (so a row's probabilities are bitwise
+      // the same whatever the batch size or rows per CTA): 16 partial sums over the columns
+      // c = p (mod 16), each in increasing c, then a fixed binary tree (p + 8, p + 4, p + 2, p + 1);
+      // the tree levels of stride >= TPR run inside the thread, the rest by shuffles.
+      float part[8];
+      const int PPT = 16 / TPR;  // partials per thread: p = h + TPR * j
+#pragma unroll
+      for (int j = 0; j < 8; ++j) part[j] = 0.f;
       if (live)
         for (int c = h; c < N2; c += TPR) {
           const float e = expf(zr[c] - m);
           zr[c] = e;
-          sum += e;
+          const int j = (c & 15) / TPR;
+#pragma unroll
+          for (int q = 0; q < 8; ++q)
+            if (q == j) part[q] += e;
         }
-      for (int o = 1; o < TPR; o <<= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+#pragma unroll
+      for (int st = 8; st >= 1; st >>= 1)
+        if (st >= TPR) {
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            if (j < st / TPR && j < PPT) part[j] = part[j] + part[j + st / TPR];
+        }
+      float sum = part[0];
+      for (int o = TPR / 2; o >= 1; o >>= 1) sum = sum + __shfl_xor_sync(0xffffffffu, sum, o);
       const float inv = 1.f / sum;
       if (live)
         for (int c = h; c < N2; c += TPR) zr[c] *= inv;
