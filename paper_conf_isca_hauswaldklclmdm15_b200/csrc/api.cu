@@ -101,6 +101,12 @@ int djinn_load_net(const char* desc, size_t desc_len, const float* weights, size
       uint64_t strides[2] = {(uint64_t)g.Kpad * 2, (uint64_t)g.N * g.Kpad * 2};
       uint32_t box[3] = {64, (uint32_t)(o.bn / o.g.cg), 1};
       djinn::encode_tmap(&o.tmB, n.dt, (uint8_t*)n.arena + o.w_off, 3, dims, strides, box);
+      if (o.stem && djinn::stem_dense_b()) {  // K-dense resident filter bank (kernels.h)
+        const int kd = (g.KH * g.KW * o.xf * o.xf * o.orig_in.C + 63) / 64 * 64;
+        uint64_t d2[2] = {(uint64_t)kd, (uint64_t)g.N}, s2[1] = {(uint64_t)g.Kpad * 2};
+        uint32_t b2[2] = {64, (uint32_t)(g.N / 2)};
+        djinn::encode_tmap(&o.tmBc, n.dt, (uint8_t*)n.arena + o.w_off, 2, d2, s2, b2, 128);
+      }
     }
     for (djinn::Op& o : n.ops) {  // dense + softmax cluster kernel: its B map, if clusters fit
       if (!o.smx) continue;

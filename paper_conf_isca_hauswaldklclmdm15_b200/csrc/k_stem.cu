@@ -56,11 +56,23 @@ namespace {
 constexpr int ST_SLAB_ROWS = 256;  // slab buffer rows (>= 128 + (KS-1)*Ws + KS-1)
 constexpr int ST_SLAB_BYTES = ST_SLAB_ROWS * 128;
 
-template <bool GATHER>
+#ifndef DJINN_STEM_NWG
+#define DJINN_STEM_NWG 4
+#endif
+// CB (K-dense B): the resident filter bank is stored dense in K -- tap t's F*F*C0 channels at K
+// t*F*F*C0 .. -- in whole 64-channel SW128 blocks (IMC: 9 x 48 = 432 -> 7 blocks, 84 KB) instead
+// of one 64-channel block per tap with 16 zero channels (9 blocks, 108 KB), which leaves room for
+// a 4th epilogue warpgroup in the pooled variant.  (An SW32 block per 16-channel K step was
+// measured first: 27 us slower at 3 warpgroups, 445 vs 418 us.)
+#ifndef DJINN_STEM_CB
+#define DJINN_STEM_CB 1
+#endif
+template <bool GATHER, bool POOL = false>
 struct StemCfg {
-  static constexpr int NWG = GATHER ? 2 : 3;                // epilogue warpgroups
+  static constexpr bool CB = DJINN_STEM_CB;
+  static constexpr int NWG = GATHER ? 2 : (POOL ? DJINN_STEM_NWG : 3);  // epilogue warpgroups
   static constexpr int EPI_WARPS = 4 * NWG;
-  static constexpr int NSLOT = GATHER ? 4 : 3;              // TMEM accumulator slots (128 columns each)
+  static constexpr int NSLOT = GATHER ? 4 : NWG;            // TMEM accumulator slots (128 columns each)
   static constexpr int GATHER_WARP0 = EPI_WARPS, GATHER_WARPS = GATHER ? 8 : 0;
   static constexpr int PROD_WARP = EPI_WARPS;               // SLAB: TMA producer; GATHER: first gather warp
   static constexpr int MMA_WARP = GATHER ? EPI_WARPS : EPI_WARPS + 1;
@@ -98,11 +110,15 @@ template <int BN>
 __host__ __device__ constexpr int pool_pstr() { return ((BN / 2) / 8 + 1) * 16; }
 template <int BN>
 __host__ __device__ constexpr int pool_hand_bytes() { return 2 * POW_MAX * ((BN / 2) / 8) * 16; }
-template <int BN, int KS, bool GATHER, bool POOL>
+template <int BN, int KS, int CH, bool GATHER>
+__host__ __device__ constexpr int stem_b_bytes() {  // K-dense: ceil(KS*KS*CH / 64) blocks
+  return StemCfg<GATHER>::CB ? (KS * KS * CH + 63) / 64 * BN * 128 : KS * KS * BN * 128;
+}
+template <int BN, int KS, int CH, bool GATHER, bool POOL>
 __host__ __device__ constexpr int stem_smem() {
-  return 1024 + ((KS * KS * BN * 128 + 1023) & ~1023) + 2 * ST_SLAB_BYTES +
-         (POOL ? StemCfg<GATHER>::NWG * 128 * pool_pstr<BN>() + 2 * pool_hand_bytes<BN>()
-               : StemCfg<GATHER>::EPI_WARPS * stem_stage_bytes<BN, GATHER>()) +
+  return 1024 + ((stem_b_bytes<BN, KS, CH, GATHER>() + 1023) & ~1023) + 2 * ST_SLAB_BYTES +
+         (POOL ? StemCfg<GATHER, POOL>::NWG * 128 * pool_pstr<BN>() + 2 * pool_hand_bytes<BN>()
+               : StemCfg<GATHER, POOL>::EPI_WARPS * stem_stage_bytes<BN, GATHER>()) +
          32 * 8 + 16;
 }
 __device__ __forceinline__ uint4 lds128(uint32_t addr) {
@@ -130,30 +146,39 @@ __device__ __forceinline__ uint4 hmax8(uint4 a, uint4 b) {  // packed 16-bit max
 }
 
 template <int BN, bool BF16, int F, int C0, int KS, bool GATHER, bool POOL>
-__global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
+__global__ void __launch_bounds__(StemCfg<GATHER, POOL>::THREADS, 1)
     stem_conv_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                     const __grid_constant__ CUtensorMap tmY0, const __grid_constant__ CUtensorMap tmY1,
+                     const __grid_constant__ CUtensorMap tmBc, const __grid_constant__ CUtensorMap tmY0,
+                     const __grid_constant__ CUtensorMap tmY1,
                      const StemGeom g, const float* __restrict__ x, const float* __restrict__ bias,
                      void* __restrict__ Y) {
-  using SC = StemCfg<GATHER>;
+  using SC = StemCfg<GATHER, POOL>;
   constexpr int KB = KS * KS;                   // K blocks: one 64-channel block per tap
   constexpr int CH = F * F * C0;                // real channels of a space-to-depth pixel
   constexpr int KSUB = (CH + 15) / 16;          // 16-channel MMA K steps per tap (IMC: 3 of 4)
-  constexpr int B_BLK = BN * 128;               // bytes of one K block of B
+  constexpr int B_BLK = BN * 128;               // bytes of one K block of B (SW128 layout)
+  constexpr int KBD = (KB * CH + 63) / 64;      // CB: K-dense blocks of B
   constexpr int NB64 = BN / 64, HAS32 = (BN % 64) == 32;
   constexpr int STG = stem_stage_bytes<BN, GATHER>();
   constexpr int NCH = BN / 16;                  // 16-column accumulator chunks
   constexpr int NSLOT = SC::NSLOT, NWG = SC::NWG;
   static_assert(CH <= 64 && CH % 8 == 0, "space-to-depth pixel must fill whole 8-channel chunks of one K block");
+  static_assert(!SC::CB || CH % 16 == 0, "K-dense bank: every 16-channel K step inside one 64-channel block");
   static_assert(BN % 32 == 0 && BN <= 128, "tile width");
 
   pdl_trigger();
   const int cid = blockIdx.x, ncl = gridDim.x;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+#ifdef DJINN_STEM_SLAB_FIRST  // layout experiment: the two slab buffers at the base, then B
+  uint8_t* sSlab = smem;
+  uint8_t* sB = sSlab + 2 * ST_SLAB_BYTES;
+  uint8_t* sOut = sB + ((stem_b_bytes<BN, KS, CH, GATHER>() + 1023) & ~1023);
+#else
   uint8_t* sB = smem;
-  uint8_t* sSlab = sB + ((KB * B_BLK + 1023) & ~1023);
+  uint8_t* sSlab = sB + ((stem_b_bytes<BN, KS, CH, GATHER>() + 1023) & ~1023);
   uint8_t* sOut = sSlab + 2 * ST_SLAB_BYTES;
+#endif
   uint8_t* sHand = sOut + (POOL ? NWG * 128 * pool_pstr<BN>() : SC::EPI_WARPS * STG);  // POOL: partial pool rows
   uint64_t* bars = reinterpret_cast<uint64_t*>(sHand + (POOL ? 2 * pool_hand_bytes<BN>() : 0));
   // bars: bfull, sfull[2], sempty[2], tfull[4], tempty[4], (tmem slot), POOL: hfull[2][2] at 16, hempty[2][2] at 20
@@ -204,7 +229,7 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");  // (cluster of one)
     fence_proxy_async();
     if (!GATHER) asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmA) : "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmB) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)(SC::CB ? &tmBc : &tmB)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmY0) : "memory");
     if (HAS32 && GATHER) asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmY1) : "memory");
   }
@@ -222,9 +247,15 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
   if (warp == SC::PROD_WARP && lane == 0) {
     // the whole filter bank, resident for the kernel: K block kb = tap kb, all BN rows (the
     // tensor map's box holds BN / 2 rows: two boxes per block)
-    mbar_arrive_expect_tx(bfull, (uint32_t)(KB * B_BLK));
-    for (int kb = 0; kb < KB; ++kb)
-      for (int h = 0; h < 2; ++h) tma_3d(smem_u32(sB) + kb * B_BLK + h * (B_BLK / 2), &tmB, bfull, kb * 64, h * (BN / 2), 0);
+    if (SC::CB) {  // K-dense bank: KBD blocks of 64 channels, two boxes of BN / 2 rows each
+      mbar_arrive_expect_tx(bfull, (uint32_t)(KBD * B_BLK));
+      for (int kb = 0; kb < KBD; ++kb)
+        for (int h = 0; h < 2; ++h) tma_2d(smem_u32(sB) + kb * B_BLK + h * (B_BLK / 2), &tmBc, bfull, kb * 64, h * (BN / 2));
+    } else {
+      mbar_arrive_expect_tx(bfull, (uint32_t)(KB * B_BLK));
+      for (int kb = 0; kb < KB; ++kb)
+        for (int h = 0; h < 2; ++h) tma_3d(smem_u32(sB) + kb * B_BLK + h * (B_BLK / 2), &tmB, bfull, kb * 64, h * (BN / 2), 0);
+    }
   }
   pdl_wait();  // the input rows and the output buffer belong to earlier kernels of the stream
 
@@ -251,7 +282,12 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
         const uint64_t ad = hi | (uint64_t)(abase + (uint32_t)(((tap / KS) * g.Ws + tap % KS) * 8));
         const uint64_t bd = hi | (uint64_t)(sB16 + (uint32_t)tap * (B_BLK >> 4));
 #pragma unroll
-        for (int k = 0; k < KSUB; ++k) mma_f16(d, ad + 2 * k, bd + 2 * k, idesc, (tap | k) != 0);
+        for (int k = 0; k < KSUB; ++k) {
+          const int kk = tap * CH + 16 * k;  // CB: the K index of this step in the dense bank
+          const uint64_t bk =
+              SC::CB ? hi | (uint64_t)(sB16 + (uint32_t)(kk >> 6) * (B_BLK >> 4) + (uint32_t)(((kk & 63) * 2) >> 4)) : bd + 2 * k;
+          mma_f16(d, ad + 2 * k, bk, idesc, (tap | k) != 0);
+        }
       }
       mma_commit(sempty0 + 8 * sb);
       mma_commit(tfull0 + 8 * slot);
@@ -640,19 +676,23 @@ __global__ void __launch_bounds__(StemCfg<GATHER>::THREADS, 1)
 }
 
 template <int BN, bool BF16, int F, int C0, int KS, bool GATHER, bool POOL>
-cudaError_t launch_stem_inst(const StemGeom& g, const CUtensorMap* tmA, const CUtensorMap* tmB, const CUtensorMap* tmY0,
-                             const CUtensorMap* tmY1, const float* x, const float* bias, void* Y, cudaStream_t st) {
+cudaError_t launch_stem_inst(const StemGeom& g, const CUtensorMap* tmA, const CUtensorMap* tmB, const CUtensorMap* tmBc,
+                             const CUtensorMap* tmY0, const CUtensorMap* tmY1, const float* x, const float* bias, void* Y,
+                             cudaStream_t st) {
   auto kern = stem_conv_kernel<BN, BF16, F, C0, KS, GATHER, POOL>;
-  constexpr int smem = stem_smem<BN, KS, GATHER, POOL>();
+  constexpr int smem = stem_smem<BN, KS, F * F * C0, GATHER, POOL>();
   static_assert(smem <= 227 * 1024 - BN * 4, "stem kernel shared memory");
   cudaError_t e = ensure_max_smem((const void*)kern, smem);
   if (e != cudaSuccess) return e;
   const int64_t work = POOL ? (int64_t)g.Nimg * g.bands : ((int64_t)g.Nimg * g.Hs * g.Ws + 127) / 128;
   const int grid = (int)(work < tc_num_sms() ? work : tc_num_sms());
-  return launch_pdl(kern, dim3(grid), dim3(StemCfg<GATHER>::THREADS), smem, st, *tmA, *tmB, *tmY0, *tmY1, g, x, bias, Y);
+  return launch_pdl(kern, dim3(grid), dim3(StemCfg<GATHER, POOL>::THREADS), smem, st, *tmA, *tmB, *tmBc, *tmY0, *tmY1, g, x,
+                    bias, Y);
 }
 
 }  // namespace
+
+bool stem_dense_b() { return StemCfg<false>::CB; }
 
 bool stem_supported(int bn, int f, int c0, int ks, int out_pitch) {
   return bn == 96 && out_pitch == 96 && f == 4 && c0 == 3 && ks == 3;
@@ -684,23 +724,23 @@ int stem_pool_bands(int nimg, int poh) {
 }
 
 cudaError_t launch_stem_conv(const StemGeom& g, int dt, const CUtensorMap* tmA, const CUtensorMap* tmB,
-                             const CUtensorMap* tmY0, const CUtensorMap* tmY1, const float* x, const float* bias, void* Y,
-                             cudaStream_t st) {
+                             const CUtensorMap* tmBc, const CUtensorMap* tmY0, const CUtensorMap* tmY1, const float* x,
+                             const float* bias, void* Y, cudaStream_t st) {
   if (g.Nimg <= 0) return cudaSuccess;
   if (g.N != 96 || (!g.gather && (g.slab_rows < 128 + 2 * g.Ws + 2 || g.slab_rows > ST_SLAB_ROWS)))
     return cudaErrorInvalidValue;
   if (g.pool) {
     if (g.gather || g.out_half || !g.epi_lrn || g.bands < 1 || g.bands > g.POH || g.POW > POW_MAX || 2 * g.Ws > 128)
       return cudaErrorInvalidValue;
-    if (dt == DT_BF16) return launch_stem_inst<96, true, 4, 3, 3, false, true>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
-    return launch_stem_inst<96, false, 4, 3, 3, false, true>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
+    if (dt == DT_BF16) return launch_stem_inst<96, true, 4, 3, 3, false, true>(g, tmA, tmB, tmBc, tmY0, tmY1, x, bias, Y, st);
+    return launch_stem_inst<96, false, 4, 3, 3, false, true>(g, tmA, tmB, tmBc, tmY0, tmY1, x, bias, Y, st);
   }
   if (g.gather) {
-    if (dt == DT_BF16) return launch_stem_inst<96, true, 4, 3, 3, true, false>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
-    return launch_stem_inst<96, false, 4, 3, 3, true, false>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
+    if (dt == DT_BF16) return launch_stem_inst<96, true, 4, 3, 3, true, false>(g, tmA, tmB, tmBc, tmY0, tmY1, x, bias, Y, st);
+    return launch_stem_inst<96, false, 4, 3, 3, true, false>(g, tmA, tmB, tmBc, tmY0, tmY1, x, bias, Y, st);
   }
-  if (dt == DT_BF16) return launch_stem_inst<96, true, 4, 3, 3, false, false>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
-  return launch_stem_inst<96, false, 4, 3, 3, false, false>(g, tmA, tmB, tmY0, tmY1, x, bias, Y, st);
+  if (dt == DT_BF16) return launch_stem_inst<96, true, 4, 3, 3, false, false>(g, tmA, tmB, tmBc, tmY0, tmY1, x, bias, Y, st);
+  return launch_stem_inst<96, false, 4, 3, 3, false, false>(g, tmA, tmB, tmBc, tmY0, tmY1, x, bias, Y, st);
 }
 
 }  // namespace djinn

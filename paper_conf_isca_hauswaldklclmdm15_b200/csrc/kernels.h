@@ -205,9 +205,14 @@ bool stem_supported(int bn, int f, int c0, int ks, int out_pitch);
 bool stem_pool_supported(int n, int ws, int oh, int ow, int kernel, int stride, int pad, int cpo, int gsz, int gpitch,
                          int xu);
 int stem_pool_bands(int nimg, int poh);
+// stem_dense_b(): the filter bank of a stem op is stored dense in K (tap t, channel c at K index
+// t * F*F*C0 + c, zeros from KS*KS*F*F*C0 to Kpad) instead of one 64-channel block per tap; tmBc is
+// then a 2D {rup(KS*KS*F*F*C0, 64), N} map of it (row pitch Kpad), box {64, N / 2}, SWIZZLE_128B
+// (IMC: 7 resident K blocks, 84 KB, instead of 9, 108 KB).
+bool stem_dense_b();
 cudaError_t launch_stem_conv(const StemGeom& g, int dt, const CUtensorMap* tmA, const CUtensorMap* tmB,
-                             const CUtensorMap* tmY0, const CUtensorMap* tmY1, const float* x, const float* bias, void* Y,
-                             cudaStream_t st);
+                             const CUtensorMap* tmBc, const CUtensorMap* tmY0, const CUtensorMap* tmY1, const float* x,
+                             const float* bias, void* Y, cudaStream_t st);
 
 // --- fused two-layer MLP + softmax (k_mlp.cu; the SENNA window nets): fp32 rows x [rows][K0]
 // -> h = act1(x W1^T + b1) (N1) -> z = h W2^T + b2 (N2) -> out (mode 0 prob fp32 [rows][N2],

@@ -1168,7 +1168,9 @@ void Net::load_weights(const float* w, size_t n, int mem) {
               int64_t kk;
               if (o.xform == 1) {  // space-to-depth: tap (ky/f, kx/f), channel ((ky%f)*f + kx%f)*C0 + c
                 const int f = o.xf;
-                kk = (int64_t)((ky / f) * g.KW + kx / f) * g.Cgp + ((ky % f) * f + kx % f) * C0 + c;
+                // the first-layer kernel keeps B dense in K (tap * f*f*C0 + channel, no per-tap pad)
+                const int64_t tstride = (o.stem && stem_dense_b()) ? (int64_t)f * f * C0 : g.Cgp;
+                kk = (int64_t)((ky / f) * g.KW + kx / f) * tstride + ((ky % f) * f + kx % f) * C0 + c;
               } else if (o.in.xu > 1) {  // x-unrolled input + x-block: tap group j, slot i
                 for (int dx = 0; dx < g.xb; ++dx) {
                   const int e = dx + kx, jj = e / g.kxs, ii = e % g.kxs;
@@ -1518,8 +1520,8 @@ void Net::forward(const float* in, int64_t rows, int in_mem, void* out, int out_
               sg.pool_gp = o.out.gsz >= g.N ? g.N / 2 : o.out.gpitch;
               sg.obd = o.out.bdr;
             }
-            e = launch_stem_conv(sg, dt, &w->tmA[i], &o.tmB, &w->tmY0[i], &w->tmY1[i], src, (const float*)(ar + o.b_off),
-                                 Y, st);
+            e = launch_stem_conv(sg, dt, &w->tmA[i], &o.tmB, &o.tmBc, &w->tmY0[i], &w->tmY1[i], src,
+                                 (const float*)(ar + o.b_off), Y, st);
           } else if (dt == DT_F32)
             e = launch_simt_gemm(g, (const float*)A, (const float*)(ar + o.w_off), (const float*)(ar + o.b_off),
                                  (float*)Y, st);

@@ -83,6 +83,7 @@ struct Op {
   // it is not launched (fused = 1)
   int stem = 0, fused = 0;
   int stem_pool = 0;            // stem = 2 with the following MAX pool in its epilogue (the pool op is fused)
+  CUtensorMap tmBc{};           // stem: the filter bank as 16-channel SW32 boxes (compact resident B)
   // fused two-layer MLP + softmax (k_mlp.cu): this GEMM op runs the whole net (mlp = 1); the
   // pack, the second GEMM and the softmax ops are not launched (fused = 1)
   int mlp = 0;
