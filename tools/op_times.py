@@ -13,7 +13,7 @@ from datagen import recipes  # noqa: E402
 
 app = sys.argv[1]
 prec = sys.argv[2] if len(sys.argv) > 2 else "bf16"
-rows = int(sys.argv[3]) if len(sys.argv) > 3 else {"imc": 1024, "face": 256, "asr": 8192, "dig": 1600}.get(app, 4096)
+rows = int(sys.argv[3]) if len(sys.argv) > 3 and int(sys.argv[3]) > 0 else {"imc": 1024, "face": 256, "asr": 8192, "dig": 1600}.get(app, 4096)
 iters = int(sys.argv[4]) if len(sys.argv) > 4 else 10
 net = dj.DjinnNet(dj.net_description(app), recipes.flat_blob(recipes.gen_weights(app, prec)), prec, rows)
 x = torch.from_numpy(recipes.gen_input_rows(app, 0, rows, prec)).cuda()
