@@ -130,3 +130,25 @@ def test_dense_tiles_at_the_bench_batches():
     assert _tiles("pos", 4096)["l1"] == (64, 1)                    # 32 x 5 = 160 tiles
     dig = _tiles("dig", 1600)
     assert dig["ip1"] == (64, 1) and dig["ip2"] == (16, 1)
+
+
+def test_plan_fused_tails_and_cluster_softmax(monkeypatch):
+    """SURVEY 8(f) f4 plan decisions: DIG's ip1 + ReLU + ip2 + softmax run as one MLP tail kernel
+    (A read by TMA, layer 2 reusing layer 1's TMEM columns: N1p 512 + N2p 16 > 512); the window
+    nets keep the whole-net MLP kernel; ASR's dense + softmax cluster kernel is opt-in
+    (DJINN_SMX=1: 16 CTAs x 512 columns per 128 rows) because it measured slower on B200."""
+    dig = dj.djinn_describe(dj.net_description("dig"), dj.DJINN_FP16, 1600)[0]
+    assert "MLP tail kernel" in dig and "N1p=512 K0p=1024 N2p=16" in dig
+    assert dig.count("[fused") == 2                          # ip2 and the softmax are not launched
+    pos = dj.djinn_describe(dj.net_description("pos"), dj.DJINN_FP16, 4096)[0]
+    assert "MLP kernel: whole net in one launch" in pos
+    monkeypatch.setenv("DJINN_MLP", "0")
+    assert "MLP" not in dj.djinn_describe(dj.net_description("dig"), dj.DJINN_FP16, 1600)[0]
+    monkeypatch.delenv("DJINN_MLP")
+    asr = dj.djinn_describe(dj.net_description("asr"), dj.DJINN_FP16, 8192)[0]
+    assert "cluster kernel" not in asr
+    monkeypatch.setenv("DJINN_SMX", "1")
+    asr1 = dj.djinn_describe(dj.net_description("asr"), dj.DJINN_FP16, 8192)[0]
+    assert "cluster kernel, 16 CTAs x 512 columns per 128 rows, rows >= 1024" in asr1
+    # fp32 path: neither fused kernel (plain SIMT plan)
+    assert "cluster" not in dj.djinn_describe(dj.net_description("asr"), dj.DJINN_FP32, 8192)[0]
