@@ -120,8 +120,9 @@ int djinn_load_net(const char* desc, size_t desc_len, const float* weights, size
       if (!o.mlp) continue;
       const djinn::Op& o2 = n.ops[i + 1];
       uint64_t d1[2] = {(uint64_t)o.g.Kpad, (uint64_t)o.g.N}, s1[1] = {(uint64_t)o.g.Kpad * 2};
-      uint32_t b1[2] = {32, (uint32_t)(o.mg.N1p / 2)};
-      djinn::encode_tmap(&o.tmW1, n.dt, (uint8_t*)n.arena + o.w_off, 2, d1, s1, b1, 64);
+      const int wk = djinn::mlp2_wk(o.mg.a_tma);
+      uint32_t b1[2] = {(uint32_t)wk, (uint32_t)(o.mg.N1p / (o.mg.nsplit > 1 ? o.mg.nsplit : 1) / 2)};
+      djinn::encode_tmap(&o.tmW1, n.dt, (uint8_t*)n.arena + o.w_off, 2, d1, s1, b1, 2 * wk);
       uint64_t d2[2] = {(uint64_t)o2.g.Kpad, (uint64_t)o2.g.N}, s2[1] = {(uint64_t)o2.g.Kpad * 2};
       uint32_t b2[2] = {64, (uint32_t)o.mg.N2p};
       djinn::encode_tmap(&o.tmW2, n.dt, (uint8_t*)n.arena + o2.w_off, 2, d2, s2, b2, 128);

@@ -35,8 +35,19 @@ namespace {
 #endif
 constexpr int MLP_THREADS = DJINN_MLP_THREADS;  // 16 warps: 4 per TMEM lane quarter drain layer 1
 constexpr int MLP_CG = MLP_THREADS / 128;        // column groups of the layer-1 epilogue
-constexpr int MLP_WSTAGES = 4;            // W1 ring stages
-constexpr int MLP_WK = 32;                // K columns per W1 stage (SWIZZLE_64B rows)
+constexpr int MLP_WSTAGES = 4;            // W1 ring stages (whole-net kernel)
+constexpr int MLP_MAXST = 12;             // AT: ring stages fitted to MLP_RING_BYTES (smaller stages when split)
+constexpr int MLP_RING_BYTES = 160 * 1024;
+// ring stages of a launch (host and device agree): the TMA-fed tail keeps ~160 KB in flight
+__host__ __device__ inline int mlp_stages(bool at, int sstride) {
+  if (!at) return MLP_WSTAGES;
+  const int n = MLP_RING_BYTES / sstride;
+  return n < 2 ? 2 : (n > MLP_MAXST ? MLP_MAXST : n);
+}
+constexpr int MLP_WK = 32;                // K columns per W1 stage (SWIZZLE_64B rows), whole-net kernel
+constexpr int MLP_WK_AT = 64;             // TMA-fed tail: 128-byte rows (SWIZZLE_128B) -- 64-byte TMA rows
+                                          // had capped its stream at ~23 B/clock per SM (DIG: 12 us of layer 1)
+__host__ __device__ constexpr int mlp_wk(bool at) { return at ? MLP_WK_AT : MLP_WK; }
 
 __device__ __forceinline__ uint32_t idesc_rt(int n, bool bf16) {  // kind::f16, D fp32, K-major A/B, M = 128
   const uint32_t ab = bf16 ? 1u : 0u;
@@ -60,27 +71,39 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
 #endif
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  const int KB0 = g.K0p / 64, KB1 = g.K1p / 64;  // 64-column blocks of the two A operands
-  constexpr int ABLK = 128 * MLP_WK * 2;         // AT: one stage's A block (128 rows of 64 B)
-  const int wstage = g.N1p * MLP_WK * 2;          // one W1 ring stage (N1p rows of 64 B)
+  // Split (AT only, nsplit = S > 1): a cluster of S CTAs shares a block of 128 rows; CTA q owns
+  // layer 1's columns [q N1p, (q + 1) N1p) (N1p = g.N1p / S) -- its slice of W1 -- and computes the
+  // partial logits of layer 2 over that K slice; CTA 0 adds the S partials (in rank order, through
+  // DSMEM) and the bias, then runs the softmax.  The per-CTA layer-1 work drops S-fold.
+  const int S = AT && g.nsplit > 1 ? g.nsplit : 1;
+  const uint32_t q = S > 1 ? cluster_rank() : 0u;
+  const int N1p = g.N1p / S, n1o = (int)q * N1p;
+  const int N1 = min(N1p, g.N1 - n1o);            // real layer-1 columns of this CTA
+  const int K1p = S > 1 ? (N1p + 63) / 64 * 64 : g.K1p;
+  const int N1c = S > 1 ? (N1p + g.N2p <= 512 ? N1p : 0) : g.N1c;
+  const int KB0 = g.K0p / 64, KB1 = K1p / 64;    // 64-column blocks of the two A operands
+  constexpr int WK = mlp_wk(AT);                 // K columns per ring stage
+  constexpr int ABLK = 128 * WK * 2;             // AT: one stage's A block (128 rows of 128 B)
+  const int wstage = N1p * WK * 2;                // one W1 ring stage (N1p rows of 2 WK bytes)
   const int sstride = AT ? ABLK + wstage : wstage;  // ring stage stride
   const int abytes = AT ? 0 : (KB0 > KB1 ? KB0 : KB1) * 128 * 128;
-  const int ring = (MLP_WSTAGES * sstride + 1023) & ~1023;
+  const int NST = mlp_stages(AT, sstride);
+  const int ring = (NST * sstride + 1023) & ~1023;
   uint8_t* sW = smem + abytes;                    // W1 ring (AT: A block + W1 block per stage)
   uint8_t* sA = AT ? sW : smem;                   // A1 (not AT), then A2 (AT: over the drained ring)
   uint8_t* sW2 = sW + ring;
   uint64_t* bars = reinterpret_cast<uint64_t*>(sW2 + KB1 * g.N2p * 128);
-  // bars: w2full, wfull[4], wempty[4], d1full, d2full
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 11);
+  // bars: w2full, wfull[NST], wempty[NST], d1full, d2full, tmem slot
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 3 + 2 * NST);
   __shared__ __align__(16) float sb1[512];
   __shared__ __align__(16) float sb2[256];
-  const uint32_t w2full = smem_u32(bars), wfull0 = smem_u32(bars + 1), wempty0 = smem_u32(bars + 5);
-  const uint32_t d1full = smem_u32(bars + 9), d2full = smem_u32(bars + 10);
+  const uint32_t w2full = smem_u32(bars), wfull0 = smem_u32(bars + 1), wempty0 = smem_u32(bars + 1 + NST);
+  const uint32_t d1full = smem_u32(bars + 1 + 2 * NST), d2full = smem_u32(bars + 2 + 2 * NST);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, tid = threadIdx.x;
   // rows of this CTA: rpc <= 128 per CTA (the MMAs stay M = 128; rows >= nrows are never
   // stored): small services spread over more SMs, so the per-CTA chain is shorter
   const int rpc = g.rpc > 0 ? g.rpc : 128;
-  const int64_t row0 = (int64_t)blockIdx.x * rpc;
+  const int64_t row0 = (int64_t)(blockIdx.x / S) * rpc;
   const int nrows = (int)(g.rows - row0 < rpc ? g.rows - row0 : rpc);
   // Input row i of the CTA is GEMM row arow(i) = (i % 4) * 32 + i / 4: the rows are spread over
   // the four TMEM lane quarters, so every epilogue warp has rows to drain when rpc < 128 (a warp
@@ -88,11 +111,11 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   // (AT: the TMA rows are contiguous, so GEMM row = input row and rpc is 128)
   auto arow = [](int i) { return ((i & 3) << 5) | (i >> 2); };
   const int nrows4 = (nrows + 3) & ~3;  // input rows loaded (whole quarters' worth of rows)
-  const int nkw = g.K0p / MLP_WK;  // W1 ring blocks
+  const int nkw = g.K0p / WK;  // W1 ring blocks
 
   if (tid == 0) {
     mbar_init(w2full, 1);
-    for (int s = 0; s < MLP_WSTAGES; ++s) {
+    for (int s = 0; s < NST; ++s) {
       mbar_init(wfull0 + 8 * s, 1);
       mbar_init(wempty0 + 8 * s, 1);
     }
@@ -106,7 +129,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
                  : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
-  for (int c = tid; c < 512; c += MLP_THREADS) sb1[c] = c < g.N1 ? __ldg(b1 + c) : 0.f;
+  for (int c = tid; c < 512; c += MLP_THREADS) sb1[c] = c < N1 ? __ldg(b1 + n1o + c) : 0.f;
   for (int c = tid; c < 256; c += MLP_THREADS) sb2[c] = c < g.N2 ? __ldg(b2 + c) : 0.f;
   tc_fence_before();
   __syncthreads();
@@ -114,27 +137,27 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   const uint32_t tmem = *tmem_slot;
   // weights: W2 whole, and the first ring stages of W1 (never written by earlier kernels)
   auto load_w1 = [&](int kb) {  // (AT: the stage's barrier also expects its A block, load_a)
-    const int s = kb % MLP_WSTAGES;
+    const int s = kb % NST;
     const uint32_t dst = smem_u32(sW) + (uint32_t)(s * sstride + (AT ? ABLK : 0));
     mbar_arrive_expect_tx(wfull0 + 8 * s, (uint32_t)(wstage + (AT ? ABLK : 0)));
-    const int half = g.N1p / 2;  // two boxes of N1p / 2 rows
-    tma_2d(dst, &tmW1, wfull0 + 8 * s, kb * MLP_WK, 0);
-    tma_2d(dst + (uint32_t)(half * MLP_WK * 2), &tmW1, wfull0 + 8 * s, kb * MLP_WK, half);
+    const int half = N1p / 2;  // two boxes of N1p / 2 rows
+    tma_2d(dst, &tmW1, wfull0 + 8 * s, kb * WK, n1o);
+    tma_2d(dst + (uint32_t)(half * WK * 2), &tmW1, wfull0 + 8 * s, kb * WK, n1o + half);
   };
   auto load_a = [&](int kb) {  // AT: rows [row0, row0 + 128) x K columns [32 kb, 32 kb + 32)
-    const int s = kb % MLP_WSTAGES;
-    tma_2d(smem_u32(sW) + (uint32_t)(s * sstride), &tmA, wfull0 + 8 * s, kb * MLP_WK, (int)row0);
+    const int s = kb % NST;
+    tma_2d(smem_u32(sW) + (uint32_t)(s * sstride), &tmA, wfull0 + 8 * s, kb * WK, (int)row0);
   };
   if (tid == 0) {
     mbar_arrive_expect_tx(w2full, (uint32_t)(KB1 * g.N2p * 128));
-    for (int kb = 0; kb < KB1; ++kb) tma_2d(smem_u32(sW2) + (uint32_t)(kb * g.N2p * 128), &tmW2, w2full, kb * 64, 0);
-    for (int kb = 0; kb < MLP_WSTAGES && kb < nkw; ++kb) load_w1(kb);
+    for (int kb = 0; kb < KB1; ++kb) tma_2d(smem_u32(sW2) + (uint32_t)(kb * g.N2p * 128), &tmW2, w2full, n1o + kb * 64, 0);
+    for (int kb = 0; kb < NST && kb < nkw; ++kb) load_w1(kb);
   }
   MST(1);
   pdl_wait();  // the input rows and the output buffer belong to earlier kernels of the stream
   MST(2);
   if (AT && tid == 0)
-    for (int kb = 0; kb < MLP_WSTAGES && kb < nkw; ++kb) load_a(kb);
+    for (int kb = 0; kb < NST && kb < nkw; ++kb) load_a(kb);
 
   // ---- 1. fp32 rows -> 16-bit A1 (K-major, 128B swizzle: element (r, k) of block k / 64 at
   // r * 128 + (((k % 64) / 8) ^ (r % 8)) * 16 + (k % 8) * 2); a warp reads one row's floats
@@ -179,31 +202,32 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   const bool bf = BF16;
   // ---- 2. layer 1 MMAs (thread 0): K steps of 16 over the W1 ring
   if (tid == 0) {
-    const int na = g.N1p > 256 ? 256 : g.N1p, nb = g.N1p - na;
+    const int na = N1p > 256 ? 256 : N1p, nb = N1p - na;
     const uint32_t ida = idesc_rt(na, bf), idb = nb ? idesc_rt(nb, bf) : 0u;
     const uint32_t a16 = (smem_u32(sA) & 0x3FFFFu) >> 4, w16 = (smem_u32(sW) & 0x3FFFFu) >> 4;
     for (int kb = 0; kb < nkw; ++kb) {
-      const int s = kb % MLP_WSTAGES;
-      mbar_wait(wfull0 + 8 * s, (uint32_t)(kb / MLP_WSTAGES) & 1);
+      const int s = kb % NST;
+      mbar_wait(wfull0 + 8 * s, (uint32_t)(kb / NST) & 1);
       tc_fence_after();
 #pragma unroll
-      for (int k = 0; k < MLP_WK / 16; ++k) {
-        const int kk = kb * MLP_WK + k * 16;  // first K column of this step
-        const uint64_t ad = AT ? hi64 | (uint64_t)(w16 + (uint32_t)(s * (sstride >> 4)) + (uint32_t)(k * 2))
+      for (int k = 0; k < WK / 16; ++k) {
+        const int kk = kb * WK + k * 16;  // first K column of this step
+        const uint64_t hw = AT ? hi128 : hi64;  // the ring's swizzle (WK * 2-byte rows)
+        const uint64_t ad = AT ? hi128 | (uint64_t)(w16 + (uint32_t)(s * (sstride >> 4)) + (uint32_t)(k * 2))
                                : hi128 | (uint64_t)(a16 + (uint32_t)((kk >> 6) * (128 * 128 / 16) + ((kk & 63) * 2) / 16));
         const uint32_t wb = w16 + (uint32_t)(s * (sstride >> 4) + (AT ? ABLK >> 4 : 0)) + (uint32_t)(k * 2);
-        mma_f16(tmem, ad, hi64 | (uint64_t)wb, ida, (kb | k) != 0);
-        if (nb) mma_f16(tmem + (uint32_t)na, ad, hi64 | (uint64_t)(wb + (uint32_t)((na * 64) >> 4)), idb, (kb | k) != 0);
+        mma_f16(tmem, ad, hw | (uint64_t)wb, ida, (kb | k) != 0);
+        if (nb) mma_f16(tmem + (uint32_t)na, ad, hw | (uint64_t)(wb + (uint32_t)((na * WK * 2) >> 4)), idb, (kb | k) != 0);
       }
       mma_commit(wempty0 + 8 * s);
     }
     mma_commit(d1full);
   } else if (tid == 32) {
     // W1 ring refills: stage kb % S is reloaded with block kb + S once its MMAs have completed
-    for (int kb = 0; kb + MLP_WSTAGES < nkw; ++kb) {
-      mbar_wait(wempty0 + 8 * (kb % MLP_WSTAGES), (uint32_t)(kb / MLP_WSTAGES) & 1);
-      load_w1(kb + MLP_WSTAGES);
-      if (AT) load_a(kb + MLP_WSTAGES);
+    for (int kb = 0; kb + NST < nkw; ++kb) {
+      mbar_wait(wempty0 + 8 * (kb % NST), (uint32_t)(kb / NST) & 1);
+      load_w1(kb + NST);
+      if (AT) load_a(kb + NST);
     }
   }
   MST(4);
@@ -217,7 +241,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
     const int quarter = warp & 3, cgi = warp >> 2;
     const int r = quarter * 32 + lane;
     const uint32_t tb = tmem + ((uint32_t)(quarter * 32) << 16);
-    const int nch = g.N1p / 16, c0 = cgi * nch / MLP_CG, c1 = (cgi + 1) * nch / MLP_CG;
+    const int nch = N1p / 16, c0 = cgi * nch / MLP_CG, c1 = (cgi + 1) * nch / MLP_CG;
     uint8_t* a2 = sA;
     // chunk ci: bias + activation -> 16-bit -> A2 (two 16-byte pieces)
     auto emit = [&](int ci, const uint32_t (&rq)[16]) {
@@ -226,7 +250,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
       bias_act16(v, rq, bq, g.act1);
       const int k = ci * 16;
 #pragma unroll
-      for (int j = 0; j < 16; ++j) v[j] = k + j < g.N1 ? v[j] : 0.f;
+      for (int j = 0; j < 16; ++j) v[j] = k + j < N1 ? v[j] : 0.f;
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         const int kk = (k + 8 * h) & 63;
@@ -248,7 +272,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
       if (ci + 1 < c1) emit(ci + 1, rb2);
     }
     // zero K columns [N1p, K1p) of A2 (W2 is zero there too; 0 * garbage could be NaN)
-    for (int k = g.N1p + 8 * cgi; k < g.K1p && act_rows; k += 8 * MLP_CG) {
+    for (int k = N1p + 8 * cgi; k < K1p && act_rows; k += 8 * MLP_CG) {
       const int kk = k & 63;
       *reinterpret_cast<uint4*>(a2 + (k >> 6) * (128 * 128) + r * 128 + (((kk >> 3) ^ (r & 7)) << 4)) = make_uint4(0, 0, 0, 0);
     }
@@ -259,13 +283,13 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   MST(5);
 
   // ---- 4. layer 2 MMAs (thread 0) into columns [N1c, N1c + N2p)
-  const uint32_t d2 = tmem + (uint32_t)g.N1c;
+  const uint32_t d2 = tmem + (uint32_t)N1c;
   if (tid == 0) {
     tc_fence_after();
     mbar_wait(w2full, 0);
     const uint32_t id2 = idesc_rt(g.N2p, bf);
     const uint32_t a16 = (smem_u32(sA) & 0x3FFFFu) >> 4, w16 = (smem_u32(sW2) & 0x3FFFFu) >> 4;
-    for (int k = 0; k < g.K1p; k += 16) {
+    for (int k = 0; k < K1p; k += 16) {
       const uint64_t ad = hi128 | (uint64_t)(a16 + (uint32_t)((k >> 6) * (128 * 128 / 16) + ((k & 63) * 2) / 16));
       const uint64_t bd = hi128 | (uint64_t)(w16 + (uint32_t)((k >> 6) * (g.N2p * 128 / 16) + ((k & 63) * 2) / 16));
       mma_f16(d2, ad, bd, id2, k != 0);
@@ -299,15 +323,34 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
 #pragma unroll
         for (int j = 0; j < 16; ++j) {
           const int c = ci * 16 + j;
-          if (c < N2 && r < nrows) stg[r * sp + c] = __uint_as_float(rq[ci][j]) + sb2[c];
+          if (c < N2 && r < nrows) stg[r * sp + c] = __uint_as_float(rq[ci][j]) + (S > 1 ? 0.f : sb2[c]);
         }
       }
   }
   __syncthreads();
+  if (S > 1) {
+    // split: CTA 0 adds the cluster's partial logits in rank order (DSMEM), then the bias
+    cluster_sync();
+    if (q == 0)
+      for (int e = tid; e < nrows * N2; e += MLP_THREADS) {
+        const int r = e / N2, c = e - r * N2;
+        const uint32_t a = smem_u32(stg + r * sp + c);
+        float z = stg[r * sp + c];
+        for (int p = 1; p < S; ++p) {
+          uint32_t ra;
+          float v;
+          asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(a), "r"(p));
+          asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(ra) : "memory");
+          z += v;
+        }
+        stg[r * sp + c] = z + sb2[c];
+      }
+    __syncthreads();
+  }
   MST(10);
   // TPR threads per row (interleaved columns; 2 / 4 / 8 as fewer rows leave threads free) for the
   // max / exp / sum, in place in shared memory; shuffles stay within the row's aligned lane group
-  {
+  if (q == 0) {
     const int rows_max = MLP_THREADS / 2;  // rows covered at 2 threads per row
     const int lt = nrows > rows_max / 2 ? 1 : (nrows > rows_max / 4 ? 2 : (nrows > rows_max / 8 ? 3 : 4)), TPR = 1 << lt;
     const int r = tid >> lt, h = tid & (TPR - 1);
@@ -359,7 +402,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
         for (int c = h; c < N2; c += TPR) zr[c] *= inv;
     }
   }
-  if (g.out_mode != 1) {
+  if (g.out_mode != 1 && q == 0) {
     __syncthreads();
     // coalesced stores: a warp writes whole rows (lanes over columns)
     for (int r = warp; r < nrows; r += MLP_THREADS / 32) {
@@ -369,6 +412,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
   }
   MST(6);
   tc_fence_before();
+  if (S > 1) cluster_sync();  // CTA 0 has read every peer's partial logits
   __syncthreads();
   MST(7);
 #ifdef DJINN_MLP_STATS
@@ -388,8 +432,10 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
 int mlp2_smem(const MlpGeom& g) {
   const int KB0 = g.K0p / 64, KB1 = g.K1p / 64;
   const int abytes = g.a_tma ? 0 : (KB0 > KB1 ? KB0 : KB1) * 128 * 128;
-  const int sstride = g.N1p * MLP_WK * 2 + (g.a_tma ? 128 * MLP_WK * 2 : 0);
-  return 1024 + abytes + ((MLP_WSTAGES * sstride + 1023) & ~1023) + KB1 * g.N2p * 128 + 12 * 8 + 16;
+  const int wk = mlp_wk(g.a_tma);
+  const int sstride = g.N1p * wk * 2 + (g.a_tma ? 128 * wk * 2 : 0);
+  return 1024 + abytes + ((mlp_stages(g.a_tma, sstride) * sstride + 1023) & ~1023) + KB1 * g.N2p * 128 +
+         (4 + 2 * MLP_MAXST) * 8 + 16;
 }
 
 int mlp2_rows_per_cta(int64_t rows) {
@@ -404,11 +450,15 @@ int mlp2_rows_per_cta(int64_t rows) {
   return 128;
 }
 
+int mlp2_wk(int a_tma) { return mlp_wk(a_tma != 0); }
+
 bool mlp2_supported(const MlpGeom& g) {
+  const int S = g.nsplit > 1 ? g.nsplit : 1;
+  if (S > 1 && (!g.a_tma || S > 8 || g.N1p % (16 * S) || g.N1p / S > 256 || g.N1p / S < 32)) return false;
   return g.K0p % 64 == 0 && g.K1p % 64 == 0 && g.N1p % 16 == 0 && g.N1p >= g.N1 && g.N1p <= 512 &&
          (g.N1p <= 256 || (g.N1p - 256) % 16 == 0) && g.N1p / 2 <= 256 && g.K1p >= g.N1p && g.N2p % 16 == 0 &&
          g.N2p >= g.N2 && g.N2p <= 64 && g.N1c % 16 == 0 && (g.N1c >= g.N1p || g.N1c == 0) &&
-         g.N1c + g.N2p <= 512 && (!g.a_tma || MLP_WSTAGES * (g.N1p + 128) * MLP_WK * 2 >= g.K1p / 64 * 128 * 128) &&
+         g.N1c + g.N2p <= 512 && (!g.a_tma || mlp_stages(true, (g.N1p + 128) * MLP_WK_AT * 2) * (g.N1p + 128) * MLP_WK_AT * 2 >= g.K1p / 64 * 128 * 128) &&
          mlp2_smem(g) <= 227 * 1024 - 3 * 1024;
 }
 
@@ -427,8 +477,25 @@ cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const
                             : (g.a_tma ? mlp2_kernel<false, true> : mlp2_kernel<false, false>);
   cudaError_t e = ensure_max_smem((const void*)kern, 227 * 1024 - 3 * 1024);
   if (e != cudaSuccess) return e;
-  return launch_pdl(kern, dim3(grid), dim3(MLP_THREADS), smem, st, *tmW1, *tmW2, g.a_tma ? *tmA : *tmW1, g, x, b1, b2,
-                    out);
+  const int S = g.nsplit > 1 ? g.nsplit : 1;
+  if (S == 1)
+    return launch_pdl(kern, dim3(grid), dim3(MLP_THREADS), smem, st, *tmW1, *tmW2, g.a_tma ? *tmA : *tmW1, g, x, b1, b2,
+                      out);
+  cudaLaunchConfig_t cfg = {};  // split: clusters of S CTAs per 128-row block
+  cfg.gridDim = dim3(grid * (unsigned)S);
+  cfg.blockDim = dim3(MLP_THREADS);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = (unsigned)S;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl_enabled() ? 2 : 1;
+  return cudaLaunchKernelEx(&cfg, kern, *tmW1, *tmW2, *tmA, g, x, b1, b2, out);
 }
 
 }  // namespace djinn

@@ -229,11 +229,14 @@ struct MlpGeom {
   int rpc;             // rows per CTA (<= 128, multiple of 8; 0 = 128)
   int a_tma;           // 1: layer 1's A is a 16-bit tensor [rows][K0p] read by TMA (tmA), x unused;
                        //    N1c = 0 then lets layer 2 reuse layer 1's TMEM columns
+  int nsplit;          // a_tma: clusters of nsplit CTAs split layer 1's N1p columns (tmW1's box is
+                       //    then {32, N1p / nsplit / 2}); CTA 0 sums the partial logits (0/1: no split)
 };
 // rows per CTA for a forward of `rows` rows: the smallest of 128 / 64 / 32 that keeps the grid
 // within one wave of SMs (DJINN_MLP_RPC overrides)
 int mlp2_rows_per_cta(int64_t rows);
 int mlp2_smem(const MlpGeom& g);
+int mlp2_wk(int a_tma);  // K columns per ring stage: 32 (SW64 boxes) or, TMA-fed, 64 (SW128)
 bool mlp2_supported(const MlpGeom& g);
 cudaError_t launch_mlp2(const MlpGeom& g, int dt, const CUtensorMap* tmW1, const CUtensorMap* tmW2, const CUtensorMap* tmA,
                         const float* x, const float* b1, const float* b2, void* out, cudaStream_t st);

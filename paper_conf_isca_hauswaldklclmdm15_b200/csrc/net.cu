@@ -964,6 +964,11 @@ void Net::build(const std::string& desc) {
       m.N2p = rup(m.N2, 16);
       m.N1c = m.N1p + m.N2p <= 512 ? m.N1p : 0;
       m.act1 = a.g.act;
+      // split layer 1's columns over a cluster (128 per CTA) when it is wide: each CTA then streams
+      // 1 / S of W1 (DIG: 512 -> 4 x 128).  DJINN_MLP_SPLIT overrides (1: no split).
+      const char* ms = getenv("DJINN_MLP_SPLIT");
+      m.nsplit = ms ? atoi(ms) : (m.N1p >= 256 && m.N1p % 128 == 0 ? m.N1p / 128 : 1);
+      if (m.nsplit > 1 && !mlp2_supported(m)) m.nsplit = 1;
       if (a.g.a_pitch <= a.g.Kpad && a.g.a_pitch % 8 == 0 && a.out.Cp <= m.K1p && m.N1p <= 512 && (m.N1p <= 256 || m.N1p % 32 == 0) &&
           mlp2_supported(m)) {
         ops[L - 3].mlp = 1;
@@ -1304,9 +1309,9 @@ Workspace* Net::workspace(cudaStream_t st) {
           uint32_t bs[2] = {(uint32_t)smx_bk(), (uint32_t)(128 / o.smx_cl)};
           encode_tmap(&w->tmAs[i], dt, w->buf[o.in_buf], 2, dims, strides, bs, 2 * smx_bk());
         }
-        if (o.mlp && o.mg.a_tma) {  // the fused MLP tail: 32-column blocks of 128 rows (SW64)
-          uint32_t bs[2] = {32, 128};
-          encode_tmap(&w->tmAs[i], dt, w->buf[o.in_buf], 2, dims, strides, bs, 64);
+        if (o.mlp && o.mg.a_tma) {  // the fused MLP tail: 64-column blocks of 128 rows (SW128)
+          uint32_t bs[2] = {(uint32_t)mlp2_wk(1), 128};
+          encode_tmap(&w->tmAs[i], dt, w->buf[o.in_buf], 2, dims, strides, bs, 2 * mlp2_wk(1));
         }
         continue;
       }
@@ -1631,7 +1636,8 @@ std::string Net::plan_string() const {
     if (o.mlp)
       s << (o.mg.a_tma ? " [MLP tail kernel: this layer + the next + softmax in one launch, A by TMA, N1p="
                        : " [MLP kernel: whole net in one launch, N1p=")
-        << o.mg.N1p << " K0p=" << o.mg.K0p << " N2p=" << o.mg.N2p << "]";
+        << o.mg.N1p << " K0p=" << o.mg.K0p << " N2p=" << o.mg.N2p
+        << (o.mg.nsplit > 1 ? " split over " + std::to_string(o.mg.nsplit) + "-CTA clusters" : std::string()) << "]";
     if (o.smx)
       s << " [+softmax: cluster kernel, " << o.smx_cl << " CTAs x " << o.smx_ncw << " columns per 128 rows, rows >= "
         << o.smx_min_rows << "]";

@@ -341,19 +341,25 @@ net.close()
 """
 
 
-@pytest.mark.parametrize("app,prec,n,rpc", [("pos", "fp16", 1000, ""), ("chk", "bf16", 4096, ""), ("ner", "fp16", 129, ""),
-                                            ("ner", "bf16", 3000, ""), ("pos", "fp16", 4096, "128"),
-                                            ("chk", "fp16", 1001, "64"), ("ner", "fp16", 70, "32"),
-                                            ("pos", "bf16", 5003, "8"), ("dig", "fp16", 1600, ""),
-                                            ("dig", "bf16", 333, "")])
-def test_mlp_kernel_equals_unfused_path(app, prec, n, rpc, tmp_path):
+@pytest.mark.parametrize("app,prec,n,env", [("pos", "fp16", 1000, {}), ("chk", "bf16", 4096, {}), ("ner", "fp16", 129, {}),
+                                            ("ner", "bf16", 3000, {}), ("pos", "fp16", 4096, {"DJINN_MLP_RPC": "128"}),
+                                            ("chk", "fp16", 1001, {"DJINN_MLP_RPC": "64"}),
+                                            ("ner", "fp16", 70, {"DJINN_MLP_RPC": "32"}),
+                                            ("pos", "bf16", 5003, {"DJINN_MLP_RPC": "8"}),
+                                            ("dig", "fp16", 1600, {"DJINN_MLP_SPLIT": "1"}),
+                                            ("dig", "bf16", 333, {"DJINN_MLP_SPLIT": "1"}),
+                                            ("dig", "fp16", 1600, {}), ("dig", "bf16", 333, {}),
+                                            ("dig", "fp16", 700, {"DJINN_MLP_SPLIT": "2"})])
+def test_mlp_kernel_equals_unfused_path(app, prec, n, env, tmp_path):
     """The one-launch window-MLP kernel (pack + l1 + HardTanh + l2 + softmax on chip) and the four
     separate kernels (DJINN_MLP=0) give bitwise-equal logits and argmax -- the same 16-bit
     operands reach the MMAs in the same K order and the epilogues round the same way -- and
     probabilities equal to the last ulps (the softmax sums in a different order).  rpc: rows per
     CTA forced by DJINN_MLP_RPC (default: chosen by the batch size), ragged last CTAs included.
     DIG: the same kernel as the tail of a conv net (ip1 + ReLU + ip2 + softmax, A read by TMA
-    from pool2's 16-bit output, layer 2 reusing layer 1's 512 TMEM columns)."""
+    from pool2's 16-bit output, layer 2 reusing layer 1's 512 TMEM columns) -- bitwise when not
+    split (DJINN_MLP_SPLIT=1); split over a cluster (default: 4 CTAs x 128 of ip1's columns) the
+    logits are the sum of per-CTA partial sums (a different fp32 order): equal to ~1e-6."""
     import os
     import subprocess
     import sys
@@ -361,14 +367,19 @@ def test_mlp_kernel_equals_unfused_path(app, prec, n, rpc, tmp_path):
     res, plans = [], []
     for mlp in ("1", "0"):
         f = str(tmp_path / f"o{mlp}.npz")
-        env = dict(os.environ, DJINN_MLP=mlp)
-        if rpc:
-            env["DJINN_MLP_RPC"] = rpc
-        r = subprocess.run([sys.executable, "-c", _MLP_CHILD, root, app, prec, str(n), f], env=env, check=True,
+        env_c = dict(os.environ, DJINN_MLP=mlp)
+        env_c.update(env)
+        r = subprocess.run([sys.executable, "-c", _MLP_CHILD, root, app, prec, str(n), f], env=env_c, check=True,
                            timeout=600, capture_output=True, text=True)
         plans.append(r.stdout)
         res.append(np.load(f))
-    assert "MLP kernel" in plans[0] and "MLP kernel" not in plans[1], plans
+    assert "MLP" in plans[0] and "MLP" not in plans[1], plans
+    if "split over" in plans[0]:
+        lg0, lg1 = res[0]["lg"], res[1]["lg"]
+        assert np.abs(lg0 - lg1).max() <= 1e-5 * np.abs(lg1).max(), np.abs(lg0 - lg1).max()
+        assert np.array_equal(res[0]["am"], lg0.argmax(1)) and (res[0]["am"] == res[1]["am"]).mean() >= 0.995
+        np.testing.assert_allclose(res[0]["pr"], res[1]["pr"], rtol=1e-4, atol=1e-6)
+        return
     assert np.array_equal(res[0]["lg"], res[1]["lg"])
     assert np.array_equal(res[0]["am"], res[1]["am"])
     np.testing.assert_allclose(res[0]["pr"], res[1]["pr"], rtol=2e-6, atol=1e-7)
