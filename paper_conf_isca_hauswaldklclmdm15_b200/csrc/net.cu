@@ -1075,7 +1075,23 @@ void Net::choose_tiles() {
         const int64_t t64 = ((g.M + 127) / 128) * ((g.N + 63) / 64) * g.Z;  // tiles after the cap (cg = 1)
         cap = (mt * nt * g.Z < 148 && t64 <= 2 * 148) ? 64 : 0;
       }
-      if (g.mode == GM_DENSE && cap >= 16 && o.bn > cap) {
+      // A long-K dense GEMM of at most two row tiles under one wave keeps 128-wide single-CTA tiles
+      // and is split over K instead (below): half the K chain per CTA at twice the per-MMA width
+      // (N = 64 MMAs run at the 52-cycle floor).  Measured on B200: IMC 16 images 160.8 -> 157.8 us
+      // per batch, FACE 2 images 191.0 -> 180.1, FACE F7 at 256 35.2 -> 33.8; IMC fc8 at 1024
+      // images was slower (27.1 -> 35.7 us incl. the reduction), hence the row limit.
+      // DJINN_SPLITK_WIDE=0 disables.
+      static const bool wide_sk = [] {
+        const char* e = getenv("DJINN_SPLITK_WIDE");
+        return !(e && e[0] == '0');
+      }();
+      const int64_t t128 = ((g.M + 127) / 128) * ((g.N + 127) / 128) * g.Z;
+      const bool wide = env_cap < 0 && wide_sk && g.mode == GM_DENSE && cap == 64 && g.Kpad / 64 >= 32 && t128 <= 74 &&
+                        (g.M + 127) / 128 <= 2 && !o.mlp && !o.smx;
+      if (wide) {
+        o.bn = 128;
+        o.g.cg = 1;
+      } else if (g.mode == GM_DENSE && cap >= 16 && o.bn > cap) {
         o.bn = cap;
         o.g.cg = tc_pick_cg(g, o.bn);
       }
