@@ -122,7 +122,7 @@ def test_dense_tiles_at_the_bench_batches():
     assert imc["fc8"] == (64, 1)                                   # 8 x 16 = 128 tiles
     face = _tiles("face", 256)
     # FACE F7 (2 row tiles, 111 K blocks): 128-wide tiles split over K (the "wide split-K" rule)
-    assert face["F7"] == (128, 1) and face["F8"] == (64, 1)
+    assert face["F7"] == (128, 1) and face["F8"] == (128, 1)
     asr = _tiles("asr", 8192)
     # > one wave: CTA pairs; the 2048-wide layers take 192-wide tiles (5 waves of 192 beat 4 of
     # 256 over 74 pairs: wave quantisation), the 8000-wide output layer keeps 256
