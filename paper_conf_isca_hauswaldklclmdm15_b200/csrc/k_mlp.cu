@@ -40,14 +40,22 @@ constexpr int MLP_MAXST = 12;             // AT: ring stages fitted to MLP_RING_
 constexpr int MLP_RING_BYTES = 160 * 1024;
 // ring stages of a launch (host and device agree): the TMA-fed tail keeps ~160 KB in flight
 __host__ __device__ inline int mlp_stages(bool at, int sstride) {
+#ifdef DJINN_MLP_WK64
+  if (!at) return 2;
+#else
   if (!at) return MLP_WSTAGES;
+#endif
   const int n = MLP_RING_BYTES / sstride;
   return n < 2 ? 2 : (n > MLP_MAXST ? MLP_MAXST : n);
 }
 constexpr int MLP_WK = 32;                // K columns per W1 stage (SWIZZLE_64B rows), whole-net kernel
 constexpr int MLP_WK_AT = 64;             // TMA-fed tail: 128-byte rows (SWIZZLE_128B) -- 64-byte TMA rows
                                           // had capped its stream at ~23 B/clock per SM (DIG: 12 us of layer 1)
+#ifdef DJINN_MLP_WK64  // experiment: 128-byte W1 rows for the whole-net kernel too (2 ring stages)
+__host__ __device__ constexpr int mlp_wk(bool at) { return MLP_WK_AT; }
+#else
 __host__ __device__ constexpr int mlp_wk(bool at) { return at ? MLP_WK_AT : MLP_WK; }
+#endif
 
 __device__ __forceinline__ uint32_t idesc_rt(int n, bool bf16) {  // kind::f16, D fp32, K-major A/B, M = 128
   const uint32_t ab = bf16 ? 1u : 0u;
@@ -212,7 +220,7 @@ __global__ void __launch_bounds__(MLP_THREADS, 1)
 #pragma unroll
       for (int k = 0; k < WK / 16; ++k) {
         const int kk = kb * WK + k * 16;  // first K column of this step
-        const uint64_t hw = AT ? hi128 : hi64;  // the ring's swizzle (WK * 2-byte rows)
+        const uint64_t hw = WK == 64 ? hi128 : hi64;  // the ring's swizzle (WK * 2-byte rows)
         const uint64_t ad = AT ? hi128 | (uint64_t)(w16 + (uint32_t)(s * (sstride >> 4)) + (uint32_t)(k * 2))
                                : hi128 | (uint64_t)(a16 + (uint32_t)((kk >> 6) * (128 * 128 / 16) + ((kk & 63) * 2) / 16));
         const uint32_t wb = w16 + (uint32_t)(s * (sstride >> 4) + (AT ? ABLK >> 4 : 0)) + (uint32_t)(k * 2);
