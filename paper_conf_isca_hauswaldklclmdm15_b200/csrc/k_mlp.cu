@@ -40,10 +40,10 @@ constexpr int MLP_MAXST = 12;             // AT: ring stages fitted to MLP_RING_
 constexpr int MLP_RING_BYTES = 160 * 1024;
 // ring stages of a launch (host and device agree): the TMA-fed tail keeps ~160 KB in flight
 __host__ __device__ inline int mlp_stages(bool at, int sstride) {
-#ifdef DJINN_MLP_WK64
-  if (!at) return 2;
-#else
+#ifdef DJINN_MLP_WK32
   if (!at) return MLP_WSTAGES;
+#else
+  if (!at) return 2;
 #endif
   const int n = MLP_RING_BYTES / sstride;
   return n < 2 ? 2 : (n > MLP_MAXST ? MLP_MAXST : n);
@@ -51,10 +51,13 @@ __host__ __device__ inline int mlp_stages(bool at, int sstride) {
 constexpr int MLP_WK = 32;                // K columns per W1 stage (SWIZZLE_64B rows), whole-net kernel
 constexpr int MLP_WK_AT = 64;             // TMA-fed tail: 128-byte rows (SWIZZLE_128B) -- 64-byte TMA rows
                                           // had capped its stream at ~23 B/clock per SM (DIG: 12 us of layer 1)
-#ifdef DJINN_MLP_WK64  // experiment: 128-byte W1 rows for the whole-net kernel too (2 ring stages)
-__host__ __device__ constexpr int mlp_wk(bool at) { return MLP_WK_AT; }
-#else
+// 128-byte W1 rows for the whole-net kernel too (2 ring stages of N1p x 128 B; its A is resident):
+// POS 4096 windows 14.5 -> 13.5 us, 65536 75.7 -> 72.4 us on B200.  DJINN_MLP_WK32 restores the
+// 4-stage ring of 64-byte rows.
+#ifdef DJINN_MLP_WK32
 __host__ __device__ constexpr int mlp_wk(bool at) { return at ? MLP_WK_AT : MLP_WK; }
+#else
+__host__ __device__ constexpr int mlp_wk(bool at) { return MLP_WK_AT; }
 #endif
 
 __device__ __forceinline__ uint32_t idesc_rt(int n, bool bf16) {  // kind::f16, D fp32, K-major A/B, M = 128
