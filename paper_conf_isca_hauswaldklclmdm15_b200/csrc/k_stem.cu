@@ -53,7 +53,16 @@
 namespace djinn {
 namespace {
 
-constexpr int ST_SLAB_ROWS = 256;  // slab buffer rows (>= 128 + (KS-1)*Ws + KS-1)
+constexpr int ST_SLAB_ROWS = 248;  // slab buffer rows (>= 128 + (KS-1)*Ws + KS-1; IMC: 244)
+// POOL: staged rows per warpgroup -- the pool reads conv rows 2r (tile rows 0 .. Ws-1) and 2r + 1
+// (Ws .. 2 Ws - 1) up to column 2 (POW - 1) + 2, i.e. rows < Ws + 2 POW <= POOL_STG_ROWS
+constexpr int POOL_STG_ROWS = 112;
+// POOL: one hand-off buffer per half (tile lt + 1 reads each item of tile lt's partial pool row and
+// then overwrites it with its own, same thread), so no "empty" barrier and half the space
+#ifndef DJINN_STEM_HAND1
+#define DJINN_STEM_HAND1 1
+#endif
+constexpr int POOL_HBUF = DJINN_STEM_HAND1 ? 1 : 2;
 constexpr int ST_SLAB_BYTES = ST_SLAB_ROWS * 128;
 
 #ifndef DJINN_STEM_NWG
@@ -65,7 +74,7 @@ constexpr int ST_SLAB_BYTES = ST_SLAB_ROWS * 128;
 // a 4th epilogue warpgroup in the pooled variant.  (An SW32 block per 16-channel K step was
 // measured first: 27 us slower at 3 warpgroups, 445 vs 418 us.)
 #ifndef DJINN_STEM_CB
-#define DJINN_STEM_CB 1
+#define DJINN_STEM_CB 0
 #endif
 template <bool GATHER, bool POOL = false>
 struct StemCfg {
@@ -109,15 +118,19 @@ constexpr int POW_MAX = 28;
 template <int BN>
 __host__ __device__ constexpr int pool_pstr() { return ((BN / 2) / 8 + 1) * 16; }
 template <int BN>
-__host__ __device__ constexpr int pool_hand_bytes() { return 2 * POW_MAX * ((BN / 2) / 8) * 16; }
+__host__ __device__ constexpr int pool_hand_bytes() { return 2 * POW_MAX * ((BN / 2) / 8) * 16; }  // one buffer
 template <int BN, int KS, int CH, bool GATHER>
 __host__ __device__ constexpr int stem_b_bytes() {  // K-dense: ceil(KS*KS*CH / 64) blocks
+#ifdef DJINN_STEM_BPAD  // diagnostic: the per-tap bank's footprint whatever the layout
+  return KS * KS * BN * 128;
+#else
   return StemCfg<GATHER>::CB ? (KS * KS * CH + 63) / 64 * BN * 128 : KS * KS * BN * 128;
+#endif
 }
 template <int BN, int KS, int CH, bool GATHER, bool POOL>
 __host__ __device__ constexpr int stem_smem() {
   return 1024 + ((stem_b_bytes<BN, KS, CH, GATHER>() + 1023) & ~1023) + 2 * ST_SLAB_BYTES +
-         (POOL ? StemCfg<GATHER, POOL>::NWG * 128 * pool_pstr<BN>() + 2 * pool_hand_bytes<BN>()
+         (POOL ? StemCfg<GATHER, POOL>::NWG * POOL_STG_ROWS * pool_pstr<BN>() + POOL_HBUF * pool_hand_bytes<BN>()
                : StemCfg<GATHER, POOL>::EPI_WARPS * stem_stage_bytes<BN, GATHER>()) +
          32 * 8 + 16;
 }
@@ -179,14 +192,18 @@ __global__ void __launch_bounds__(StemCfg<GATHER, POOL>::THREADS, 1)
   uint8_t* sSlab = sB + ((stem_b_bytes<BN, KS, CH, GATHER>() + 1023) & ~1023);
   uint8_t* sOut = sSlab + 2 * ST_SLAB_BYTES;
 #endif
-  uint8_t* sHand = sOut + (POOL ? NWG * 128 * pool_pstr<BN>() : SC::EPI_WARPS * STG);  // POOL: partial pool rows
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sHand + (POOL ? 2 * pool_hand_bytes<BN>() : 0));
+  uint8_t* sHand = sOut + (POOL ? NWG * POOL_STG_ROWS * pool_pstr<BN>() : SC::EPI_WARPS * STG);  // POOL: partial pool rows
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sHand + (POOL ? POOL_HBUF * pool_hand_bytes<BN>() : 0));
   // bars: bfull, sfull[2], sempty[2], tfull[4], tempty[4], (tmem slot), POOL: hfull[2][2] at 16, hempty[2][2] at 20
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 13);
   __shared__ __align__(16) float sbias[BN];
   const uint32_t bfull = smem_u32(bars), sfull0 = smem_u32(bars + 1), sempty0 = smem_u32(bars + 3);
   const uint32_t tfull0 = smem_u32(bars + 5), tempty0 = smem_u32(bars + 9);
   const uint32_t hfull0 = smem_u32(bars + 16), hempty0 = smem_u32(bars + 20);
+  // single hand-off buffer: per half, the local index of the last tile that published its partial
+  // pool row (a counter, not an mbarrier phase: warpgroups run up to NSLOT tiles apart, so a
+  // parity wait could alias a phase two tiles old)
+  const uint32_t hseq0 = smem_u32(bars + 24);
   static_assert(!POOL || !GATHER, "the fused pool runs on the TMA-slab variant");
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -221,11 +238,13 @@ __global__ void __launch_bounds__(StemCfg<GATHER, POOL>::THREADS, 1)
       mbar_init(tfull0 + 8 * s, 1);
       mbar_init(tempty0 + 8 * s, 4);  // the draining warpgroup
     }
-    if (POOL)
+    if (POOL) {
       for (int s = 0; s < 4; ++s) {
         mbar_init(hfull0 + 8 * s, 1);   // writer warpgroup, per (buffer, half)
         mbar_init(hempty0 + 8 * s, 1);  // reader warpgroup, per (buffer, half)
       }
+      for (int h = 0; h < 2; ++h) asm volatile("st.shared.s32 [%0], %1;" ::"r"(hseq0 + 4 * h), "r"(-1) : "memory");
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");  // (cluster of one)
     fence_proxy_async();
     if (!GATHER) asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmA) : "memory");
@@ -374,7 +393,7 @@ __global__ void __launch_bounds__(StemCfg<GATHER, POOL>::THREADS, 1)
     const int quarter = warp & 3, wg = warp >> 2;
     const int m = quarter * 32 + lane;
     const uint32_t lane_base = (uint32_t)(quarter * 32) << 16;
-    const uint32_t stg = smem_u32(sOut) + (uint32_t)(wg * 128 * PSTR);
+    const uint32_t stg = smem_u32(sOut) + (uint32_t)(wg * POOL_STG_ROWS * PSTR);
     const uint32_t my_row = stg + (uint32_t)(m * PSTR);
     const uint32_t hand = smem_u32(sHand);
     const int PJ = g.pool_gp / 8;  // output pieces per half (grouped: the group pitch, pads written 0)
@@ -385,7 +404,7 @@ __global__ void __launch_bounds__(StemCfg<GATHER, POOL>::THREADS, 1)
     (void)p0; (void)p1; (void)p2;
     for_each_tile([&](int lt, int, int img, int r, bool first, bool last) {
       if (lt % NWG != wg) return;
-      const int slot = lt % NSLOT, k = lt & 1, kp = k ^ 1;
+      const int slot = lt % NSLOT, k = POOL_HBUF == 2 ? (lt & 1) : 0, kp = POOL_HBUF == 2 ? (k ^ 1) : 0;
       SST(p2);
       SST(p0);
       if (lane == 0) mbar_wait_sleep(tfull0 + 8 * slot, (uint32_t)(lt / NSLOT) & 1);
@@ -404,8 +423,18 @@ __global__ void __launch_bounds__(StemCfg<GATHER, POOL>::THREADS, 1)
         asm volatile("bar.sync %0, 128;" ::"r"(1 + wg) : "memory");  // half h staged by the warpgroup
         SST(p0);
         if (lane == 0) {
-          mbar_wait_sleep(hempty0 + 8 * (2 * k + h), ((uint32_t)(lt >> 1) & 1) ^ 1);
-          if (lt > 0) mbar_wait_sleep(hfull0 + 8 * (2 * kp + h), (uint32_t)((lt - 1) >> 1) & 1);
+          if (POOL_HBUF == 2) {
+            mbar_wait_sleep(hempty0 + 8 * (2 * k + h), ((uint32_t)(lt >> 1) & 1) ^ 1);
+            if (lt > 0) mbar_wait_sleep(hfull0 + 8 * (2 * kp + h), (uint32_t)((lt - 1) >> 1) & 1);
+          } else if (lt > 0) {  // tile lt - 1 has read the buffer and written its own partial row
+            int seen, iters = 0;
+            for (;;) {
+              asm volatile("ld.acquire.cta.shared.s32 %0, [%1];" : "=r"(seen) : "r"(hseq0 + 4 * h) : "memory");
+              if (seen >= lt - 1) break;
+              if (++iters > (1 << 24)) __trap();  // a lost publication must fault, never hang
+              __nanosleep(64);
+            }
+          }
         }
         __syncwarp();
         SACC(p_hw, p0);
@@ -419,20 +448,26 @@ __global__ void __launch_bounds__(StemCfg<GATHER, POOL>::THREADS, 1)
             const uint4 va = hmax8<BF16>(hmax8<BF16>(lds128(a), lds128(a + PSTR)), lds128(a + 2 * PSTR));
             const uint32_t b = a + (uint32_t)(g.Ws * PSTR);
             const uint4 vb = hmax8<BF16>(hmax8<BF16>(lds128(b), lds128(b + PSTR)), lds128(b + 2 * PSTR));
-            if (!last) sts128(hw + (uint32_t)((pc * HP + j) * 16), hmax8<BF16>(va, vb));
+            // read the previous tile's partial row before overwriting it (one buffer: hr == hw)
             if (!first) res = hmax8<BF16>(lds128(hr + (uint32_t)((pc * HP + j) * 16)), va);
+            if (!last) sts128(hw + (uint32_t)((pc * HP + j) * 16), hmax8<BF16>(va, vb));
           }
           if (!first) *reinterpret_cast<uint4*>(Yp + (orow + pc) * g.Cpo + h * g.pool_gp + 8 * j) = res;
         }
         asm volatile("bar.sync %0, 128;" ::"r"(1 + wg) : "memory");  // staging read, hand-off half written
         if (m == 0) {
-          mbar_arrive(hfull0 + 8 * (2 * k + h));
-          if (lt > 0) mbar_arrive(hempty0 + 8 * (2 * kp + h));
+          if (POOL_HBUF == 2) {
+            mbar_arrive(hfull0 + 8 * (2 * k + h));
+            if (lt > 0) mbar_arrive(hempty0 + 8 * (2 * kp + h));
+          } else {
+            asm volatile("st.release.cta.shared.s32 [%0], %1;" ::"r"(hseq0 + 4 * h), "r"(lt) : "memory");
+          }
         }
         SACC(p_pool, p1);
       };
       auto put_chunk = [&](int i, const float (&o)[16]) {  // 16-bit LRN output -> staged half
         const int p0 = 2 * (i % (HALF / 16));
+        if (m >= POOL_STG_ROWS) return;  // rows the pool never reads
 #pragma unroll
         for (int hh = 0; hh < 2; ++hh)
           sts128(my_row + (uint32_t)((p0 + hh) * 16),
@@ -703,6 +738,7 @@ bool stem_pool_supported(int n, int ws, int oh, int ow, int kernel, int stride, 
   // tile = two conv rows; pool rows exactly cover the conv rows (no clipped ceil window);
   // output plain at pitch n, or two groups of n / 2 channels at a group pitch (pads written 0)
   if (kernel != 3 || stride != 2 || pad != 0 || xu != 1 || 2 * ws > 128 || oh < 3 || ow < 3) return false;
+  if (ws + 2 * ((ow - 3) / 2 + 1) > POOL_STG_ROWS) return false;  // the pooled rows fit the staging
   if ((oh - 3) % 2 || (ow - 3) % 2 || (ow - 3) / 2 + 1 > POW_MAX || ow > ws) return false;
   const bool plain = cpo == n && gsz >= n;
   const bool grouped = gsz == n / 2 && gpitch >= gsz && gpitch % 8 == 0 && cpo == 2 * gpitch;
