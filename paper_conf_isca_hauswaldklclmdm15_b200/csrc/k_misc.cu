@@ -102,19 +102,22 @@ __global__ void pack_xform_kernel(const float* __restrict__ x, T* __restrict__ y
     for (int pix = blockIdx.x * blockDim.x + threadIdx.x; pix < per_row; pix += gridDim.x * blockDim.x) {
       const int yo = pix / Wo, xo = pix - (pix / Wo) * Wo;
       T* dst = y + (r * per_row + pix) * (int64_t)Cp;
-      int a = 0, b = 0, c = 0;  // mode 1: (dy, dx, c); mode 2: (kx, -, c)
+      int a = 0, b = 0, c = 0;  // mode 1: (dy, dx, c); mode 2: (kx, -, c); mode 3: (kx, ky, c)
+      const int kh = H - Ho + 1;  // mode 3: window rows
       for (int ch = 0; ch < Cp; ch += 8) {
         __align__(16) T v[8];
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
-          const int yy = mode == 1 ? yo * f + a : yo;
+          const int yy = mode == 1 ? yo * f + a : (mode == 3 ? yo + b : yo);
           const int xx = mode == 1 ? xo * f + b : xo * xs + a;
-          const bool ok = a < f && yy < H && xx < W;
+          const bool ok = (mode == 3 ? b < kh : a < f) && yy < H && xx < W;
           v[j] = cvt<T>(ok ? __ldg(src + ((int64_t)c * H + yy) * W + xx) : 0.f);
           if (++c == C) {
             c = 0;
             if (mode == 1) {
               if (++b == f) { b = 0; ++a; }
+            } else if (mode == 3) {
+              if (++a == f) { a = 0; ++b; }
             } else {
               ++a;
             }
@@ -162,6 +165,9 @@ __global__ void pack_xform_fixed_kernel(const float* __restrict__ x, T* __restri
             if (MODE == 1) {
               const int d = cc / C, c = cc % C, dy = d / F, dx = d % F;
               if (d < F * F && y0 + dy < H && x0 + dx < W) val = __ldg(p0 + ((int64_t)c * H + dy) * W + dx);
+            } else if (MODE == 3) {  // window unroll: channel (ky * F + kx) * C + c, KH = H - Ho + 1 rows
+              const int ky = cc / (F * C), rr = cc % (F * C), kx = rr / C, c = rr % C;
+              if (ky < H - Ho + 1 && x0 + kx < W) val = __ldg(p0 + ((int64_t)c * H + ky) * W + kx);
             } else {
               const int kx = cc / C, c = cc % C;
               if (kx < F && x0 + kx < W) val = __ldg(p0 + (int64_t)c * H * W + kx);
@@ -193,6 +199,8 @@ static bool launch_pack_fixed(const float* x, void* y, int64_t rows, int C, int 
     launch_pdl(pack_xform_fixed_kernel<T, 2, 3, 18, 64, 8>, dim3(g), dim3(128), 0, st, x, (T*)y, rows, H, W, Ho, Wo);
   else if (mode == 2 && C == 1 && f == 12 && xs == 8 && Cp == 16)
     launch_pdl(pack_xform_fixed_kernel<T, 2, 1, 12, 16, 8>, dim3(g), dim3(128), 0, st, x, (T*)y, rows, H, W, Ho, Wo);
+  else if (mode == 3 && C == 1 && f == 12 && xs == 8 && Cp == 64)
+    launch_pdl(pack_xform_fixed_kernel<T, 3, 1, 12, 64, 8>, dim3(g), dim3(128), 0, st, x, (T*)y, rows, H, W, Ho, Wo);
   else if (mode == 1 && C == 3 && f == 4 && Cp == 64)
     launch_pdl(pack_xform_fixed_kernel<T, 1, 3, 4, 64, 1>, dim3(g), dim3(128), 0, st, x, (T*)y, rows, H, W, Ho, Wo);
   else

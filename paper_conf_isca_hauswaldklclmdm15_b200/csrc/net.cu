@@ -623,13 +623,25 @@ void Net::build(const std::string& desc) {
               if (xbc <= kx_cap && (k + xbc - 1) * cur.C <= 64 && xbc * os.Cp <= 256) { XB = xbc; break; }
           const int U = k + XB - 1, OWb = (OW + XB - 1) / XB;
           creal = U * cur.C;  // real channels of a packed tap (the rest of its 64 are zero)
-          pk.xform = o.xform = 2;
+          // window unroll (xform 3): when the whole k x U window fits one 64-channel pixel (DIG
+          // conv1: 5 x 12 x 1 = 60), the packed pixel holds all k rows too and the conv becomes a
+          // 1 x 1 conv over the OH x OWb grid -- one 128-byte TMA row per GEMM row instead of k
+          // 32-byte ones.  Opt-in (DJINN_WINDOW_UNROLL=1): correct, but measured slower on B200
+          // (DIG conv1 41.5 -> 40.0 us, its pack 9.9 -> 15.9 us: conv1 is bound by its epilogue).
+          static const bool wu_on = [] {
+            const char* e = getenv("DJINN_WINDOW_UNROLL");
+            return e && e[0] == '1';
+          }();
+          const bool wu = wu_on && k > 1 && k * U * cur.C <= 64 && k * U * cur.C > 32;
+          pk.xform = o.xform = wu ? 3 : 2;
           pk.xf = o.xf = U;
           pk.xs = o.xs = XB;
           pk.out = Shape();
-          pk.out.C = U * cur.C; pk.out.H = cur.H; pk.out.W = OWb; pk.out.Cp = tap_pitch(U * cur.C);
-          g.H = cur.H; g.W = pk.out.W; g.Cp_in = g.Cgp = pk.out.Cp;
-          g.KH = k; g.KW = 1;
+          pk.out.C = (wu ? k : 1) * U * cur.C; pk.out.H = wu ? OH : cur.H; pk.out.W = OWb;
+          pk.out.Cp = tap_pitch(pk.out.C);
+          if (wu) creal = pk.out.C;
+          g.H = pk.out.H; g.W = pk.out.W; g.Cp_in = g.Cgp = pk.out.Cp;
+          g.KH = wu ? 1 : k; g.KW = 1;
           if (XB > 1) {
             g.xb = XB;
             g.OWb = OWb;
@@ -1201,6 +1213,11 @@ void Net::load_weights(const float* w, size_t n, int mem) {
                   if (dx > 0) put(0, dx * g.out_pitch + co, ki, w[off]);
                   else kk = ki;
                 }
+              } else if (o.xform == 3) {  // window unroll: one tap, channel (ky*U + kx)*C0 + c (+ x-block copies)
+                const int U = o.xf;
+                for (int dx = 1; dx < g.xb; ++dx)
+                  put(0, dx * g.out_pitch + co, (int64_t)(ky * U + dx + kx) * C0 + c, w[off]);
+                kk = (int64_t)(ky * U + kx) * C0 + c;
               } else if (o.xform == 2) {  // kx-unroll: tap ky, channel kx*C0 + c (+ x-block copies)
                 for (int dx = 1; dx < g.xb; ++dx)
                   put(0, dx * g.out_pitch + co, (int64_t)ky * g.Cgp + (dx + kx) * C0 + c, w[off]);
@@ -1659,7 +1676,9 @@ std::string Net::plan_string() const {
     if (o.smx)
       s << " [+softmax: cluster kernel, " << o.smx_cl << " CTAs x " << o.smx_ncw << " columns per 128 rows, rows >= "
         << o.smx_min_rows << "]";
-    if (o.kind == OP_PACK && o.xform) s << " [" << (o.xform == 1 ? "space-to-depth " : "kx-unroll ") << o.xf << (o.xs > 1 ? " step " + std::to_string(o.xs) : std::string()) << "]";
+    if (o.kind == OP_PACK && o.xform)
+      s << " [" << (o.xform == 1 ? "space-to-depth " : o.xform == 3 ? "window-unroll " : "kx-unroll ") << o.xf
+        << (o.xs > 1 ? " step " + std::to_string(o.xs) : std::string()) << "]";
     s << "\n";
   }
   return s.str();
