@@ -191,9 +191,61 @@ __global__ void pack_xform_fixed_kernel(const float* __restrict__ x, T* __restri
   }
 }
 
+// kx-unroll (mode 2) with one WARP per input row: the warp reads the row's C x W floats with
+// coalesced loads into shared memory, then writes the row's Wo packed pixels as whole 16-byte
+// chunks (consecutive lanes, consecutive chunks).  The per-pixel kernel above reads each input
+// float from up to U / XS pixels' threads with 32-byte-strided lanes (FACE: ~32 sectors per load
+// instruction).  FACE's 152 x 3 rows: 62.5 -> 51.0 us on B200.
+template <typename T, int C, int U, int CP, int XS>
+__global__ void __launch_bounds__(256) pack_kx_rows_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows,
+                                                           int H, int W, int Wo) {
+  pdl_trigger();
+  pdl_wait();
+  extern __shared__ float srow[];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  float* sr = srow + wid * C * W;
+  const int64_t total = rows * H;  // (image, row) pairs: kx-unroll keeps the rows
+  constexpr int CPC = CP / 8;
+  for (int64_t t = (int64_t)blockIdx.x * nw + wid; t < total; t += (int64_t)gridDim.x * nw) {
+    const int64_t img = t / H;
+    const int yy = (int)(t - img * H);
+    const float* src = x + (img * C * H + yy) * (int64_t)W;
+#pragma unroll
+    for (int c = 0; c < C; ++c)
+      for (int i = lane; i < W; i += 32) sr[c * W + i] = __ldg(src + (int64_t)c * H * W + i);
+    __syncwarp();
+    uint4* dst = reinterpret_cast<uint4*>(y + t * (int64_t)Wo * CP);
+    for (int e = lane; e < Wo * CPC; e += 32) {
+      const int xo = e / CPC, j = e - xo * CPC;
+      __align__(16) T v[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const int cc = 8 * j + q, kx = cc / C, c = cc - kx * C, xx = xo * XS + kx;
+        v[q] = cvt<T>(kx < U && xx < W ? sr[c * W + xx] : 0.f);
+      }
+      dst[e] = *reinterpret_cast<const uint4*>(v);
+    }
+    __syncwarp();
+  }
+}
+
 template <typename T>
 static bool launch_pack_fixed(const float* x, void* y, int64_t rows, int C, int H, int W, int mode, int f, int xs, int Ho,
                               int Wo, int Cp, cudaStream_t st) {
+  static const bool rows_on = [] {  // DJINN_PACK_ROWS=0: the per-pixel kx-unroll kernel
+    const char* e = getenv("DJINN_PACK_ROWS");
+    return !(e && e[0] == '0');
+  }();
+  if (rows_on && mode == 2 && Ho == H && C * W * 4 * 8 <= 48 * 1024) {
+    const int64_t total = rows * H;
+    const unsigned gb = (unsigned)std::min<int64_t>((total + 7) / 8, 148 * 16);
+    const size_t smem = (size_t)8 * C * W * 4;
+    if (C == 3 && f == 18 && xs == 8 && Cp == 64) {
+      launch_pdl(pack_kx_rows_kernel<T, 3, 18, 64, 8>, dim3(gb), dim3(256), smem, st, x, (T*)y, rows, H, W, Wo);
+      return true;
+    }
+    // (DIG's 28 x 1 rows: 16.2 us vs 10.0 for the per-pixel kernel, so it keeps that one)
+  }
   dim3 g(min(nblocks(Ho * Wo, 128), 1024), (unsigned)(rows < 65535 ? rows : 65535));
   if (mode == 2 && C == 3 && f == 18 && xs == 8 && Cp == 64)
     launch_pdl(pack_xform_fixed_kernel<T, 2, 3, 18, 64, 8>, dim3(g), dim3(128), 0, st, x, (T*)y, rows, H, W, Ho, Wo);
