@@ -31,6 +31,36 @@ static inline int nblocks(int64_t n, int t) { return (int)((n + t - 1) / t); }
 // K0: fp32 NCHW [rows][C][H][W] -> NHWC [rows][Ho][Wo][Cp] (16-bit), 8 channels per thread,
 // with the optional first-layer transforms (space-to-depth, kx-unroll) that give the first
 // convolution a dense, 16-element-aligned K (DESIGN.md sec 5 "first layer").
+// Vector inputs (C x 1 x 1: ASR frames, NLP windows): one thread per 8-channel chunk of the
+// flattened (row, chunk) space, two float4 loads when the row is 16-byte aligned.  The general
+// kernel below gives each row its own block, and a 448-channel row is only 56 chunks (ASR pack
+// 13.5 us for 8192 frames: mostly idle warps).
+template <typename T>
+__global__ void pack16_vec_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int C, int Cp) {
+  pdl_trigger();
+  pdl_wait();
+  const int chunks = Cp / 8;
+  const int64_t total = rows * chunks;
+  const bool vec = (C % 4) == 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / chunks;
+    const int c0 = (int)(i - r * chunks) * 8;
+    const float* src = x + r * C + c0;
+    float f[8];
+    if (vec && c0 + 8 <= C) {
+      const float4 a = __ldg(reinterpret_cast<const float4*>(src)), b = __ldg(reinterpret_cast<const float4*>(src + 4));
+      f[0] = a.x; f[1] = a.y; f[2] = a.z; f[3] = a.w; f[4] = b.x; f[5] = b.y; f[6] = b.z; f[7] = b.w;
+    } else {
+#pragma unroll
+      for (int j = 0; j < 8; ++j) f[j] = c0 + j < C ? __ldg(src + j) : 0.f;
+    }
+    __align__(16) T v[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) v[j] = cvt<T>(f[j]);
+    reinterpret_cast<uint4*>(y)[i] = *reinterpret_cast<const uint4*>(v);
+  }
+}
+
 template <typename T>
 __global__ void pack16_kernel(const float* __restrict__ x, T* __restrict__ y, int64_t rows, int C, int H, int W,
                               int mode, int f, int xs, int Ho, int Wo, int Cp) {
@@ -277,6 +307,13 @@ cudaError_t launch_pack_input(const float* x, void* y, int64_t rows, int C, int 
       launch_pdl(pack_xform_kernel<__half>, dim3(g), dim3(T), 0, st, x, (__half*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
     else
       launch_pdl(pack_xform_kernel<__nv_bfloat16>, dim3(g), dim3(T), 0, st, x, (__nv_bfloat16*)y, rows, C, H, W, mode, f, xs, Ho, Wo, Cp);
+  } else if (mode == 0 && H == 1 && W == 1 && Ho == 1 && Wo == 1) {
+    const int64_t total = rows * (Cp / 8);
+    const unsigned g = (unsigned)std::min<int64_t>((total + T - 1) / T, 148 * 16);
+    if (dt == DT_F16)
+      launch_pdl(pack16_vec_kernel<__half>, dim3(g), dim3(T), 0, st, x, (__half*)y, rows, C, Cp);
+    else
+      launch_pdl(pack16_vec_kernel<__nv_bfloat16>, dim3(g), dim3(T), 0, st, x, (__nv_bfloat16*)y, rows, C, Cp);
   } else {
     const int per_row = Ho * Wo * (Cp / 8);
     dim3 g(min(nblocks(per_row, T), 1024), (unsigned)(rows < 65535 ? rows : 65535));
