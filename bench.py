@@ -120,8 +120,10 @@ class ClockSampler:
         try:
             self.nv = self._nvml_handle()
             self.src = "nvml 2 ms"
+            self.ready = threading.Event()
             self.t = threading.Thread(target=self._poll, daemon=True)
             self.t.start()
+            self.ready.wait(2.0)     # the poll loop is running before the timed region starts
             return self
         except Exception:
             self.nv = None
@@ -137,17 +139,22 @@ class ClockSampler:
             self.proc = None
         return self
 
+    def _sample(self):
+        pm, h = self.nv
+        sm = pm.nvmlDeviceGetClockInfo(h, pm.NVML_CLOCK_SM)
+        pw = pm.nvmlDeviceGetPowerUsage(h) / 1000.0
+        rs = pm.nvmlDeviceGetCurrentClocksEventReasons(h)
+        act = ["Active" if rs & self.NVML_BITS[n] else "Not Active" for n in self.NAMES]
+        self.rows.append((time.time(), [str(sm), str(self.mx), f"{pw:.1f}"] + act))
+
     def _poll(self):
         pm, h = self.nv
-        mx = pm.nvmlDeviceGetMaxClockInfo(h, pm.NVML_CLOCK_SM)
+        self.mx = pm.nvmlDeviceGetMaxClockInfo(h, pm.NVML_CLOCK_SM)
+        self.ready.set()
         while not self.stop:
             if self.active:
                 try:
-                    sm = pm.nvmlDeviceGetClockInfo(h, pm.NVML_CLOCK_SM)
-                    pw = pm.nvmlDeviceGetPowerUsage(h) / 1000.0
-                    rs = pm.nvmlDeviceGetCurrentClocksEventReasons(h)
-                    act = ["Active" if rs & self.NVML_BITS[n] else "Not Active" for n in self.NAMES]
-                    self.rows.append((time.time(), [str(sm), str(mx), f"{pw:.1f}"] + act))
+                    self._sample()
                 except Exception:
                     pass
                 time.sleep(0.002)
@@ -165,6 +172,14 @@ class ClockSampler:
     def mark_end(self):
         self.active = False
         self.t1 = time.time()
+        if self.nv and not any(self.t0 <= t <= self.t1 for t, _ in self.rows):
+            # the poll thread got no GIL slot inside a short region: one sample at its end
+            try:
+                self._sample()
+                self.t1 = self.rows[-1][0]
+                self.src = "nvml (1 sample at the end of the timed region)"
+            except Exception:
+                pass
         if self.proc:
             time.sleep(0.1)
 
